@@ -1,0 +1,1277 @@
+/*
+ * triosim_oracle.c -- TEST INFRASTRUCTURE ONLY.
+ *
+ * A plain, slow, single-threaded CPU discrete-event simulator of TrioSim's
+ * per-design-point method (Li et al., "TrioSim", ISCA'25; PAPER.md = P:N line
+ * refs).  Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+ * --impl reference leg may load this library.  It shares NO code, header,
+ * table or helper with the CUDA product path (paper_conf_isca_libwmvgjbj025_b200/):
+ * it restates the binary record layouts itself and re-derives everything
+ * (routes, partitions, buckets, task graph) from the paper and the readings in
+ * DESIGN.md ("Semantics" R1-R19; readings Q1-Q31).
+ *
+ * Structure, in the paper's order (Sec. 4.3-4.5):
+ *   1. trace checks + producer table
+ *   2. operator-time model t' = t * rho                   (R4)
+ *   3. trace extrapolation into an explicit task graph    (R6-R11)
+ *        nodes: compute TASKs (per-GPU in-order queues),
+ *               FLOWs (data movement / collective steps),
+ *               BARRIERs (zero-time joins: collective start, "done on GPU g")
+ *   4. routing: BFS shortest path, lexicographic tie break (R12)
+ *   5. event-driven timeline (R13-R17) with the
+ *      flow-based network model: route -> bandwidth allocation (max-min
+ *      progressive filling) -> progress update -> delivery, re-allocating every
+ *      in-transit flow whenever one starts or completes (Fig. 5).
+ *   6. outputs (R18-R19).
+ *
+ * Arithmetic: IEEE binary64, compiled with -O2 -ffp-contract=off (no FMA
+ * contraction), no fast-math; every sum is a left fold in the stated order.
+ *
+ * Parity pins (tests/test_oracle_*.py): closed forms CF1-CF14 (DESIGN.md
+ * "Pins"), brute-force routing and partitioning, max-min invariants of the
+ * progressive filling, and an exact-rational Python re-simulation of exported
+ * task graphs.  Unpinned: absolute accuracy vs real hardware (P:244-300,
+ * needs the paper's traces and machines) -- "parity unpinned" for that only.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <math.h>
+#include <stdio.h>
+
+/* ------------------------------------------------------------------ */
+/* Record layouts (the binary formats of DESIGN.md "Inputs"),          */
+/* restated here independently of include/triosim.h.                   */
+/* ------------------------------------------------------------------ */
+typedef struct {
+    uint32_t kind, layer;
+    uint8_t phase, tp_role;
+    uint16_t flags;
+    uint32_t io_off;
+    uint16_t n_in, n_out;
+    uint32_t pad;
+    double time_s, flops;
+} OOp; /* 40 B */
+
+typedef struct {
+    uint64_t bytes_b0;
+    uint8_t category, batch_scaled;
+    uint16_t pad;
+    uint32_t param_id;
+} OTensor; /* 16 B */
+
+typedef struct {
+    uint32_t src, dst;
+    double bw, lat;
+} OLink; /* 24 B */
+
+typedef struct {
+    uint32_t topo;
+    uint8_t strategy, tp_mode, coll_algo, pad0;
+    uint16_t dp, tp, pp, pad1;
+    uint32_t microbatches, global_batch;
+    int32_t stage_plan;
+    uint32_t pad2;
+    uint64_t bucket_bytes;
+    double bw_scale, lat_scale;
+} OPoint; /* 56 B */
+
+typedef struct {
+    double iter_time_s, compute_busy_max_s, comm_busy_s, exposed_comm_s, coll_payload_bytes;
+    uint64_t n_compute, n_flows, n_collectives, n_p2p, n_instants, n_wf_calls, n_wf_rounds, order_hash;
+    int32_t status;
+    uint32_t max_active_flows;
+} OResult; /* 112 B */
+
+_Static_assert(sizeof(OOp) == 40, "op record");
+_Static_assert(sizeof(OTensor) == 16, "tensor record");
+_Static_assert(sizeof(OLink) == 24, "link record");
+_Static_assert(sizeof(OPoint) == 56, "point record");
+_Static_assert(sizeof(OResult) == 112, "result record");
+
+enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
+enum { CAT_INPUT = 0, CAT_WEIGHT = 1, CAT_WGRAD = 2, CAT_ACT = 3, CAT_AGRAD = 4, CAT_OTHER = 5 };
+enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4 };
+enum { TPM_PAPER = 0, TPM_MEGATRON = 1 };
+enum { ALG_RING = 0, ALG_TREE = 1 };
+enum { ROLE_NONE = 0, ROLE_COL = 1, ROLE_ROW = 2, ROLE_LOCAL = 3, ROLE_GATHER = 4 };
+enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
+#define OPF_BATCH_SCALED 1u
+
+#define O_OK 0
+#define O_EINVAL (-1)
+#define O_ENOMEM (-2)
+
+enum { PT_OK = 0, PT_BAD_BATCH = 1, PT_BAD_DEGREES = 2, PT_NO_ROUTE = 3, PT_TOO_LARGE = 4,
+       PT_DEADLOCK = 5, PT_BAD_PLAN = 6, PT_BAD_CONFIG = 7 };
+
+/* event kinds of the order hash (R19) */
+enum { EV_COLL_START = 1, EV_RELEASE = 2, EV_ACTIVATE = 3, EV_DELIVER = 4, EV_TASK_START = 5, EV_TASK_END = 6 };
+
+/* ------------------------------------------------------------------ */
+/* small growable arrays                                               */
+/* ------------------------------------------------------------------ */
+typedef struct { int *v; long n, cap; } IVec;
+static int iv_push(IVec *a, int x) {
+    if (a->n == a->cap) {
+        long nc = a->cap ? a->cap * 2 : 64;
+        int *p = (int *)realloc(a->v, (size_t)nc * sizeof(int));
+        if (!p) return -1;
+        a->v = p; a->cap = nc;
+    }
+    a->v[a->n++] = x;
+    return 0;
+}
+static void iv_free(IVec *a) { free(a->v); a->v = NULL; a->n = a->cap = 0; }
+
+/* ------------------------------------------------------------------ */
+/* Trace checks: SSA tensors, producers precede readers,*/
+/* phases FWD* BWD* OPT*, layers numbered by first FWD appearance.     */
+/* ------------------------------------------------------------------ */
+typedef struct {
+    const OOp *ops; uint32_t n_ops;
+    const OTensor *ts; uint32_t n_ts;
+    const uint32_t *io; uint32_t n_io;
+    uint32_t b0;
+    int *prod;        /* producing op of each tensor, -1 = none (resident input/weight) */
+    uint32_t n_layers;
+} Trace;
+
+static int trace_check(Trace *T) {
+    if (T->n_ops == 0 || T->b0 == 0) return O_EINVAL;
+    T->prod = (int *)malloc(sizeof(int) * (T->n_ts ? T->n_ts : 1));
+    if (!T->prod) return O_ENOMEM;
+    for (uint32_t x = 0; x < T->n_ts; x++) {
+        T->prod[x] = -1;
+        if (T->ts[x].category > CAT_OTHER) return O_EINVAL;
+    }
+    int last_phase = 0;
+    uint32_t next_layer = 0;
+    for (uint32_t o = 0; o < T->n_ops; o++) {
+        const OOp *op = &T->ops[o];
+        if (op->phase > PH_OPT || op->phase < last_phase) return O_EINVAL;
+        last_phase = op->phase;
+        if (!(op->time_s >= 0.0) || isinf(op->time_s)) return O_EINVAL;
+        if ((uint64_t)op->io_off + op->n_in + op->n_out > T->n_io) return O_EINVAL;
+        if (op->tp_role > 7) return O_EINVAL;
+        if (op->phase == PH_FWD) {
+            if (op->layer == next_layer) next_layer++;
+            else if (op->layer > next_layer) return O_EINVAL;
+        } else if (op->layer >= next_layer) {
+            return O_EINVAL;
+        }
+        for (uint32_t k = 0; k < op->n_in; k++) {
+            uint32_t x = T->io[op->io_off + k];
+            if (x >= T->n_ts) return O_EINVAL;
+            if (T->prod[x] == (int)o) return O_EINVAL; /* read-own-output */
+        }
+        for (uint32_t k = 0; k < op->n_out; k++) {
+            uint32_t x = T->io[op->io_off + op->n_in + k];
+            if (x >= T->n_ts) return O_EINVAL;
+            if (T->prod[x] != -1) return O_EINVAL; /* each tensor produced once */
+            T->prod[x] = (int)o;
+        }
+    }
+    /* a reader must come after the producer (checked after all producers are known) */
+    for (uint32_t o = 0; o < T->n_ops; o++) {
+        const OOp *op = &T->ops[o];
+        for (uint32_t k = 0; k < op->n_in; k++) {
+            uint32_t x = T->io[op->io_off + k];
+            if (T->prod[x] >= (int)o) return O_EINVAL;
+        }
+    }
+    T->n_layers = next_layer;
+    if (T->n_layers == 0) return O_EINVAL;
+    return O_OK;
+}
+
+/* ------------------------------------------------------------------ */
+/* Operator-time model (R4; P:178 batch change, P:200 trace time when   */
+/* nothing changes, P:202 FLOPs-ratio rescale).                        */
+/* ------------------------------------------------------------------ */
+static int op_split(const OOp *op, int tp_mode) {
+    if (tp_mode == TPM_PAPER) return (op->tp_role & ROLE_GATHER) != 0;   /* conv/linear/embedding */
+    return (op->tp_role & 3) != 0;                                      /* Megatron COL/ROW/LOCAL */
+}
+
+static double op_time(const Trace *T, uint32_t o, double r_b, int tp, int tp_mode) {
+    const OOp *op = &T->ops[o];
+    double rho = 1.0;
+    if (op->flags & OPF_BATCH_SCALED) rho = r_b;
+    if (tp > 1 && op_split(op, tp_mode)) rho = rho / (double)tp;
+    if (rho == 1.0) return op->time_s;      /* the trace time itself */
+    return op->time_s * rho;                /* FLOPs-ratio rescale */
+}
+
+/* R5: bytes of a tensor instance under the point's batch and TP split */
+static double tensor_bytes(const Trace *T, uint32_t x, double r_b, int tp, int tp_mode) {
+    const OTensor *t = &T->ts[x];
+    double b = (double)t->bytes_b0;
+    if (t->batch_scaled) b = b * r_b;
+    if (tp > 1 && t->category == CAT_WGRAD && T->prod[x] >= 0 && op_split(&T->ops[T->prod[x]], tp_mode))
+        b = b / (double)tp;
+    return b;
+}
+
+/* ------------------------------------------------------------------ */
+/* Task graph                                                          */
+/* ------------------------------------------------------------------ */
+enum { N_TASK = 0, N_FLOW = 1, N_BARRIER = 2 };
+#define NF_COLL_START 1 /* barrier that is a collective start (hashed) */
+#define NF_P2P 2        /* flow is a point-to-point data movement */
+
+typedef struct {
+    int type;
+    int gpu;          /* task: simulated GPU node */
+    double dur;       /* task: t' */
+    int src, dst;     /* flow endpoints (GPU nodes) */
+    double bytes;     /* flow size */
+    uint64_t code;    /* canonical id for the order hash */
+    int flags;
+} GNode;
+
+typedef struct {
+    GNode *n; long count, cap;
+    IVec dep_from, dep_to;   /* edge list: node dep_from[i] waits for node dep_to[i] */
+    int n_coll;
+    double coll_payload;     /* left fold of collective payloads in creation order */
+} Graph;
+
+static int g_add(Graph *G, GNode nd) {
+    if (G->count == G->cap) {
+        long nc = G->cap ? G->cap * 2 : 256;
+        GNode *p = (GNode *)realloc(G->n, (size_t)nc * sizeof(GNode));
+        if (!p) return -1;
+        G->n = p; G->cap = nc;
+    }
+    G->n[G->count] = nd;
+    return (int)G->count++;
+}
+static int g_dep(Graph *G, int node, int on) {
+    if (iv_push(&G->dep_from, node) || iv_push(&G->dep_to, on)) return -1;
+    return 0;
+}
+static void g_free(Graph *G) {
+    free(G->n); G->n = NULL; G->count = G->cap = 0;
+    iv_free(&G->dep_from); iv_free(&G->dep_to);
+}
+static int add_task(Graph *G, int gpu, long prog, double dur) {
+    GNode n; memset(&n, 0, sizeof n);
+    n.type = N_TASK; n.gpu = gpu; n.dur = dur;
+    n.code = ((uint64_t)(uint32_t)gpu << 40) | (uint64_t)prog;
+    return g_add(G, n);
+}
+static int add_barrier(Graph *G, int flags, uint64_t code) {
+    GNode n; memset(&n, 0, sizeof n);
+    n.type = N_BARRIER; n.flags = flags; n.code = code;
+    return g_add(G, n);
+}
+static int add_flow(Graph *G, int src, int dst, double bytes, uint64_t code, int flags) {
+    GNode n; memset(&n, 0, sizeof n);
+    n.type = N_FLOW; n.src = src; n.dst = dst; n.bytes = bytes; n.code = code; n.flags = flags;
+    return g_add(G, n);
+}
+static uint64_t coll_flow_code(int c, int step, int member) {
+    return ((uint64_t)(uint32_t)c << 32) | ((uint64_t)(uint32_t)step << 16) | (uint64_t)(uint32_t)member;
+}
+static uint64_t p2p_flow_code(uint32_t x, int j, int dst) {
+    return (1ull << 59) | ((uint64_t)x << 32) | ((uint64_t)(uint32_t)j << 16) | (uint64_t)(uint32_t)dst;
+}
+
+/*
+ * One collective (R10; P:87-89 ring AllReduce, P:174 reduce/scatter/gather,
+ * P:192 ring tasks handed to the network model).  members[] are GPU nodes in
+ * ring order.  trig[i] = task whose completion makes member i's input ready;
+ * prev_done[i] = "previous collective of this group done on member i" (FIFO
+ * per (GPU, group), reading Q24) or NULL.  Writes done[i] = barrier "this
+ * collective is done on member i" (last flow touching it delivered).
+ */
+static int build_collective(Graph *G, const int *members, int p, int kind, int algo, double S,
+                            const int *trig, const int *prev_done, int *done) {
+    int c = G->n_coll++;
+    G->coll_payload = G->coll_payload + S;
+    int sb = add_barrier(G, NF_COLL_START, (uint64_t)c);
+    if (sb < 0) return -1;
+    for (int i = 0; i < p; i++) {
+        if (g_dep(G, sb, trig[i])) return -1;
+        if (prev_done && g_dep(G, sb, prev_done[i])) return -1;
+    }
+    IVec fl = {0}; /* all flows of this collective */
+    if (algo == ALG_RING || kind != CK_AR) {
+        /* ring: K steps; flow (i,k) goes m_i -> m_(i+1); released at start if k == 0,
+         * else when (i-1,k-1) [predecessor's chunk arrived] and (i,k-1) [own previous
+         * send] are both delivered (reading Q21). */
+        int K = (kind == CK_AR) ? 2 * (p - 1) : (p - 1);
+        double chunk = S / (double)p;
+        int *id = (int *)malloc(sizeof(int) * (size_t)(p * (K > 0 ? K : 1)));
+        if (!id) return -1;
+        for (int k = 0; k < K; k++)
+            for (int i = 0; i < p; i++) {
+                int f = add_flow(G, members[i], members[(i + 1) % p], chunk, coll_flow_code(c, k, i), 0);
+                if (f < 0) { free(id); return -1; }
+                id[k * p + i] = f;
+                iv_push(&fl, f);
+                if (k == 0) {
+                    g_dep(G, f, sb);
+                } else {
+                    g_dep(G, f, id[(k - 1) * p + (i - 1 + p) % p]);
+                    g_dep(G, f, id[(k - 1) * p + i]);
+                }
+            }
+        free(id);
+    } else {
+        /* tree AllReduce (extension, reading Q25): binary heap over member index,
+         * reduce i -> parent(i) carrying S once all children's reduces arrived;
+         * broadcast parent(i) -> i once parent(i) holds the result. */
+        int *up = (int *)malloc(sizeof(int) * (size_t)p), *dn = (int *)malloc(sizeof(int) * (size_t)p);
+        if (!up || !dn) { free(up); free(dn); return -1; }
+        for (int i = 0; i < p; i++) up[i] = dn[i] = -1;
+        for (int i = p - 1; i >= 1; i--) {
+            up[i] = add_flow(G, members[i], members[(i - 1) / 2], S, coll_flow_code(c, 0, i), 0);
+            iv_push(&fl, up[i]);
+        }
+        for (int i = 1; i < p; i++) {
+            dn[i] = add_flow(G, members[(i - 1) / 2], members[i], S, coll_flow_code(c, 1, i), 0);
+            iv_push(&fl, dn[i]);
+        }
+        for (int i = 1; i < p; i++) {
+            int nch = 0;
+            for (int ch = 2 * i + 1; ch <= 2 * i + 2 && ch < p; ch++) { g_dep(G, up[i], up[ch]); nch++; }
+            if (nch == 0) g_dep(G, up[i], sb);
+            int par = (i - 1) / 2;
+            if (par == 0) {
+                for (int ch = 1; ch <= 2 && ch < p; ch++) g_dep(G, dn[i], up[ch]);
+            } else {
+                g_dep(G, dn[i], dn[par]);
+            }
+        }
+        free(up); free(dn);
+    }
+    for (int i = 0; i < p; i++) {
+        done[i] = add_barrier(G, 0, 0);
+        if (done[i] < 0) { iv_free(&fl); return -1; }
+        /* done on member i: every flow with src or dst = m_i delivered (R10) */
+        int any = 0;
+        for (long q = 0; q < fl.n; q++) {
+            const GNode *f = &G->n[fl.v[q]];
+            if (f->src == members[i] || f->dst == members[i]) { g_dep(G, done[i], fl.v[q]); any = 1; }
+        }
+        if (!any) g_dep(G, done[i], sb);
+    }
+    iv_free(&fl);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Routing (R12; "we use the shortest path algorithm"):           */
+/* BFS by hop count, neighbours expanded in ascending node id, first    */
+/* discovery fixes the parent -> lexicographically smallest node path.  */
+/* ------------------------------------------------------------------ */
+typedef struct {
+    uint32_t n_nodes, n_gpus, n_links;
+    const OLink *links;
+    int *adj_off, *adj_link;   /* per node, out-links sorted by dst */
+} Topo;
+
+static const OLink *g_sort_links;
+static int cmp_by_dst(const void *a, const void *b) {
+    int la = *(const int *)a, lb = *(const int *)b;
+    uint32_t da = g_sort_links[la].dst, db = g_sort_links[lb].dst;
+    return (da > db) - (da < db);
+}
+
+static int topo_init(Topo *tp, uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links) {
+    tp->n_nodes = n_nodes; tp->n_gpus = n_gpus; tp->n_links = n_links; tp->links = links;
+    if (n_gpus == 0 || n_gpus > n_nodes) return O_EINVAL;
+    tp->adj_off = (int *)calloc(n_nodes + 1, sizeof(int));
+    tp->adj_link = (int *)malloc(sizeof(int) * (n_links ? n_links : 1));
+    if (!tp->adj_off || !tp->adj_link) return O_ENOMEM;
+    for (uint32_t e = 0; e < n_links; e++) {
+        const OLink *l = &links[e];
+        if (l->src >= n_nodes || l->dst >= n_nodes || l->src == l->dst) return O_EINVAL;
+        if (!(l->bw > 0.0) || isinf(l->bw) || !(l->lat >= 0.0) || isinf(l->lat)) return O_EINVAL;
+        for (uint32_t f = 0; f < e; f++)
+            if (links[f].src == l->src && links[f].dst == l->dst) return O_EINVAL; /* one link per ordered pair */
+        tp->adj_off[l->src + 1]++;
+    }
+    for (uint32_t v = 0; v < n_nodes; v++) tp->adj_off[v + 1] += tp->adj_off[v];
+    int *fill = (int *)calloc(n_nodes, sizeof(int));
+    if (!fill) return O_ENOMEM;
+    for (uint32_t e = 0; e < n_links; e++) {
+        uint32_t s = links[e].src;
+        tp->adj_link[tp->adj_off[s] + fill[s]++] = (int)e;
+    }
+    free(fill);
+    g_sort_links = links;
+    for (uint32_t v = 0; v < n_nodes; v++)
+        qsort(tp->adj_link + tp->adj_off[v], (size_t)(tp->adj_off[v + 1] - tp->adj_off[v]), sizeof(int), cmp_by_dst);
+    return O_OK;
+}
+static void topo_free(Topo *tp) { free(tp->adj_off); free(tp->adj_link); tp->adj_off = tp->adj_link = NULL; }
+
+/* returns hop count (>=0) and writes link ids src->dst into out[]; -1 = no route */
+static int bfs_route(const Topo *tp, int src, int dst, int *out, int out_cap) {
+    if (src == dst) return 0;
+    int n = (int)tp->n_nodes;
+    int *par_link = (int *)malloc(sizeof(int) * (size_t)n), *queue = (int *)malloc(sizeof(int) * (size_t)n);
+    char *seen = (char *)calloc((size_t)n, 1);
+    if (!par_link || !queue || !seen) { free(par_link); free(queue); free(seen); return -2; }
+    int qh = 0, qt = 0;
+    queue[qt++] = src; seen[src] = 1; par_link[src] = -1;
+    while (qh < qt && !seen[dst]) {
+        int u = queue[qh++];
+        for (int a = tp->adj_off[u]; a < tp->adj_off[u + 1]; a++) {
+            int e = tp->adj_link[a];
+            int v = (int)tp->links[e].dst;
+            if (!seen[v]) { seen[v] = 1; par_link[v] = e; queue[qt++] = v; }
+        }
+    }
+    int hops = -1;
+    if (seen[dst]) {
+        int len = 0;
+        for (int v = dst; v != src; v = (int)tp->links[par_link[v]].src) len++;
+        if (len <= out_cap) {
+            int v = dst;
+            for (int k = len - 1; k >= 0; k--) { out[k] = par_link[v]; v = (int)tp->links[par_link[v]].src; }
+            hops = len;
+        } else {
+            hops = -3;
+        }
+    }
+    free(par_link); free(queue); free(seen);
+    return hops;
+}
+
+/* ------------------------------------------------------------------ */
+/* PP stage partition (R8; P:188 user-specified, "automatically   */
+/* assigns layers to GPUs to balance workloads"): contiguous layers,    */
+/* minimise the max stage cost (left fold of trace times t), ties to    */
+/* the lexicographically smallest boundary vector.                      */
+/* ------------------------------------------------------------------ */
+static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
+    int L = (int)T->n_layers;
+    if (S < 1 || S > L) return -1;
+    double *lc = (double *)calloc((size_t)L, sizeof(double));
+    double *cost = (double *)malloc(sizeof(double) * (size_t)L * (size_t)L); /* cost[a*L+b] = layers a..b */
+    double *best = (double *)malloc(sizeof(double) * (size_t)(S + 1) * (size_t)(L + 1));
+    if (!lc || !cost || !best) { free(lc); free(cost); free(best); return -2; }
+    for (uint32_t o = 0; o < T->n_ops; o++) lc[T->ops[o].layer] = lc[T->ops[o].layer] + T->ops[o].time_s;
+    for (int a = 0; a < L; a++) {
+        double s = 0.0;
+        for (int b = a; b < L; b++) { s = s + lc[b]; cost[a * L + b] = s; }
+    }
+    /* best[s][i]: min over partitions of layers i..L-1 into s stages of the max stage cost */
+#define BEST(s, i) best[(size_t)(s) * (size_t)(L + 1) + (size_t)(i)]
+    for (int i = 0; i < L; i++) BEST(1, i) = cost[i * L + L - 1];
+    for (int s = 2; s <= S; s++)
+        for (int i = 0; i + s <= L; i++) {
+            double b = INFINITY;
+            for (int j = i + 1; L - j >= s - 1; j++) {
+                double a = cost[i * L + j - 1];
+                double r = BEST(s - 1, j);
+                double m = a > r ? a : r;
+                if (m < b) b = m;
+            }
+            BEST(s, i) = b;
+        }
+    double V = BEST(S, 0);
+    int i = 0;
+    first_layer[0] = 0;
+    for (int s = S; s >= 2; s--) {
+        int jj = -1;
+        for (int j = i + 1; L - j >= s - 1; j++)
+            if (cost[i * L + j - 1] <= V && BEST(s - 1, j) <= V) { jj = j; break; }
+        if (jj < 0) { free(lc); free(cost); free(best); return -3; }
+        first_layer[S - s + 1] = (uint32_t)jj;
+        i = jj;
+    }
+#undef BEST
+    free(lc); free(cost); free(best);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Point validation (R3) -- same order of checks as DESIGN.md R3.       */
+/* ------------------------------------------------------------------ */
+static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
+                       int have_plan) {
+    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_TREE) return PT_BAD_CONFIG;
+    if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
+        return PT_BAD_CONFIG;
+    uint32_t dp = pt->dp, tpd = pt->tp, pp = pt->pp, m = pt->microbatches;
+    if (dp == 0 || tpd == 0 || pp == 0) return PT_BAD_DEGREES;
+    switch (pt->strategy) {
+    case ST_DP: case ST_DDP: if (tpd != 1 || pp != 1) return PT_BAD_DEGREES; break;
+    case ST_TP: if (dp != 1 || pp != 1) return PT_BAD_DEGREES; break;
+    case ST_PP: if (dp != 1 || tpd != 1) return PT_BAD_DEGREES; break;
+    default: break;
+    }
+    int piped = (pt->strategy == ST_PP || pt->strategy == ST_HYBRID);
+    if (piped && m == 0) return PT_BAD_DEGREES;
+    if ((uint64_t)dp * tpd * pp > tp->n_gpus) return PT_BAD_DEGREES;
+    if (pp > T->n_layers) return PT_BAD_DEGREES;
+    uint64_t mm = piped ? m : 1;
+    if (pt->global_batch == 0 || pt->global_batch % ((uint64_t)dp * mm) != 0) return PT_BAD_BATCH;
+    if (piped && have_plan) {
+        if (plan_len != pp || plan[0] != 0) return PT_BAD_PLAN;
+        for (uint32_t s = 1; s < pp; s++)
+            if (plan[s] <= plan[s - 1] || plan[s] >= T->n_layers) return PT_BAD_PLAN;
+    }
+    return PT_OK;
+}
+
+static const int *ring_order_of(const uint32_t *ro, uint32_t n_gpus, int *buf) {
+    for (uint32_t i = 0; i < n_gpus; i++) buf[i] = ro ? (int)ro[i] : (int)i;
+    return buf;
+}
+
+/* ------------------------------------------------------------------ */
+/* Extrapolation: DP / DDP (R6)                           */
+/* ------------------------------------------------------------------ */
+typedef struct { uint32_t x; int prod; } WEnt;
+static int cmp_went(const void *a, const void *b) {
+    const WEnt *p = (const WEnt *)a, *q = (const WEnt *)b;
+    if (p->prod != q->prod) return (p->prod > q->prod) - (p->prod < q->prod);
+    return (p->x > q->x) - (p->x < q->x);
+}
+
+static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) {
+    int dp = pt->dp;
+    uint32_t N = T->n_ops;
+    double r_b = (double)(pt->global_batch / dp) / (double)T->b0;
+    int *task = (int *)malloc(sizeof(int) * (size_t)dp * N);
+    if (!task) return -1;
+    /* every rank duplicates every operator */
+    for (int r = 0; r < dp; r++)
+        for (uint32_t o = 0; o < N; o++)
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, 1, pt->tp_mode));
+    if (dp > 1) {
+        /* weight gradients in production order (reading Q4: produced by the backward pass) */
+        WEnt *w = (WEnt *)malloc(sizeof(WEnt) * (T->n_ts ? T->n_ts : 1));
+        int nw = 0;
+        for (uint32_t x = 0; x < T->n_ts; x++)
+            if (T->ts[x].category == CAT_WGRAD && T->prod[x] >= 0 && T->ops[T->prod[x]].phase != PH_OPT) {
+                w[nw].x = x; w[nw].prod = T->prod[x]; nw++;
+            }
+        qsort(w, (size_t)nw, sizeof(WEnt), cmp_went);
+        int last_nonopt = -1;
+        for (uint32_t o = 0; o < N; o++) if (T->ops[o].phase != PH_OPT) last_nonopt = (int)o;
+        int first_opt = -1;
+        for (uint32_t o = 0; o < N; o++) if (T->ops[o].phase == PH_OPT) { first_opt = (int)o; break; }
+        int *trig = (int *)malloc(sizeof(int) * (size_t)dp), *prev = (int *)malloc(sizeof(int) * (size_t)dp),
+            *done = (int *)malloc(sizeof(int) * (size_t)dp);
+        int have_prev = 0;
+        int i = 0;
+        while (i < nw) {
+            /* bucket (reading Q5): bucket_bytes == 0 -> one tensor per AllReduce (paper-literal);
+             * else greedy: close the bucket once its u64 byte sum reaches bucket_bytes */
+            int j = i;
+            uint64_t sum = 0;
+            double S = 0.0;
+            for (;;) {
+                sum += T->ts[w[j].x].bytes_b0;
+                S = S + tensor_bytes(T, w[j].x, r_b, 1, pt->tp_mode);
+                j++;
+                if (pt->bucket_bytes == 0 || sum >= pt->bucket_bytes || j == nw) break;
+            }
+            /* DDP: AllReduce parallel with backward, triggered by the op producing the bucket's
+             * last gradient; DP (DataParallel): after the backward pass (reading Q6) */
+            int trig_op = (pt->strategy == ST_DDP) ? w[j - 1].prod : last_nonopt;
+            for (int r = 0; r < dp; r++) trig[r] = task[(size_t)r * N + trig_op];
+            if (build_collective(G, ro, dp, CK_AR, pt->coll_algo, S, trig, have_prev ? prev : NULL, done)) return -1;
+            memcpy(prev, done, sizeof(int) * (size_t)dp);
+            have_prev = 1;
+            i = j;
+        }
+        /* optimizer waits for this GPU's gradient collectives (reading Q7) */
+        if (have_prev && first_opt >= 0)
+            for (int r = 0; r < dp; r++) g_dep(G, task[(size_t)r * N + first_opt], prev[r]);
+        free(w); free(trig); free(prev); free(done);
+    }
+    free(task);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Extrapolation: TP (R7)                              */
+/* ------------------------------------------------------------------ */
+static int expand_tp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) {
+    int tp = pt->tp;
+    uint32_t N = T->n_ops;
+    double r_b = (double)pt->global_batch / (double)T->b0;
+    int *task = (int *)malloc(sizeof(int) * (size_t)tp * N);
+    if (!task) return -1;
+    for (int r = 0; r < tp; r++)
+        for (uint32_t o = 0; o < N; o++)
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, tp, pt->tp_mode));
+    if (tp > 1) {
+        int *done_of = (int *)malloc(sizeof(int) * (size_t)(T->n_ts ? T->n_ts : 1) * (size_t)tp);
+        char *has = (char *)calloc(T->n_ts ? T->n_ts : 1, 1);
+        int *trig = (int *)malloc(sizeof(int) * (size_t)tp), *prev = (int *)malloc(sizeof(int) * (size_t)tp);
+        int have_prev = 0;
+        for (uint32_t o = 0; o < N; o++) {
+            const OOp *op = &T->ops[o];
+            for (uint32_t k = 0; k < op->n_out; k++) {
+                uint32_t x = T->io[op->io_off + op->n_in + k];
+                int kind = -1;
+                if (pt->tp_mode == TPM_PAPER) {
+                    /* "collects the partial outputs from all devices" */
+                    if ((op->tp_role & ROLE_GATHER) && op->phase == PH_FWD) kind = CK_AG;
+                    if ((op->tp_role & ROLE_GATHER) && op->phase == PH_BWD && T->ts[x].category == CAT_AGRAD) kind = CK_AR;
+                } else {
+                    if ((op->tp_role & 3) == ROLE_ROW && op->phase == PH_FWD) kind = CK_AR;
+                    if ((op->tp_role & 3) == ROLE_COL && op->phase == PH_BWD && T->ts[x].category == CAT_AGRAD) kind = CK_AR;
+                }
+                if (kind < 0) continue;
+                /* payload = the full tensor (not divided by tp), reading Q8 */
+                double S = (double)T->ts[x].bytes_b0;
+                if (T->ts[x].batch_scaled) S = S * r_b;
+                for (int r = 0; r < tp; r++) trig[r] = task[(size_t)r * N + o];
+                if (build_collective(G, ro, tp, kind, pt->coll_algo, S, trig, have_prev ? prev : NULL,
+                                     done_of + (size_t)x * tp)) return -1;
+                memcpy(prev, done_of + (size_t)x * tp, sizeof(int) * (size_t)tp);
+                have_prev = 1;
+                has[x] = 1;
+            }
+        }
+        /* a later operator that reads a communicated tensor waits for it on its GPU */
+        for (uint32_t o = 0; o < N; o++) {
+            const OOp *op = &T->ops[o];
+            for (uint32_t k = 0; k < op->n_in; k++) {
+                uint32_t x = T->io[op->io_off + k];
+                if (has[x])
+                    for (int r = 0; r < tp; r++) g_dep(G, task[(size_t)r * N + o], done_of[(size_t)x * tp + r]);
+            }
+        }
+        free(done_of); free(has); free(trig); free(prev);
+    }
+    free(task);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Extrapolation: PP / GPipe (R8; Fig. 4)                    */
+/* ------------------------------------------------------------------ */
+static int expand_pp(const Trace *T, const OPoint *pt, const int *ro, const uint32_t *first_layer, Graph *G) {
+    int S = pt->pp, m = (int)pt->microbatches;
+    uint32_t N = T->n_ops, L = T->n_layers;
+    double r_b = (double)(pt->global_batch / (uint32_t)m) / (double)T->b0;
+    int *stage_of_layer = (int *)malloc(sizeof(int) * L);
+    for (uint32_t l = 0, s = 0; l < L; l++) {
+        while ((int)s + 1 < S && first_layer[s + 1] <= l) s++;
+        stage_of_layer[l] = (int)s;
+    }
+    /* task id of instance (o, j); OPT ops use j = 0 */
+    int *inst = (int *)malloc(sizeof(int) * (size_t)N * (size_t)m);
+    int *prog_op = (int *)malloc(sizeof(int) * ((size_t)N * (size_t)m + 1));
+    int *prog_mb = (int *)malloc(sizeof(int) * ((size_t)N * (size_t)m + 1));
+    /* readers: for each tensor, which stages read it (bitmask over <=64 stages) */
+    uint64_t *readers = (uint64_t *)calloc(T->n_ts ? T->n_ts : 1, sizeof(uint64_t));
+    if (!stage_of_layer || !inst || !prog_op || !prog_mb || !readers) return -1;
+    for (uint32_t o = 0; o < N; o++) {
+        const OOp *op = &T->ops[o];
+        for (uint32_t k = 0; k < op->n_in; k++) readers[T->io[op->io_off + k]] |= 1ull << stage_of_layer[op->layer];
+    }
+    /* cross-stage transfers: (tensor, producer instance, destination) -> flow id */
+    int *xidx = (int *)malloc(sizeof(int) * (T->n_ts ? T->n_ts : 1));
+    int ncross = 0;
+    for (uint32_t x = 0; x < T->n_ts; x++) {
+        xidx[x] = -1;
+        if (T->prod[x] >= 0) {
+            int ps = stage_of_layer[T->ops[T->prod[x]].layer];
+            if (readers[x] & ~(1ull << ps)) xidx[x] = ncross++;
+        }
+    }
+    int *p2p = (int *)malloc(sizeof(int) * ((size_t)ncross * (size_t)m * (size_t)S + 1));
+    for (size_t q = 0; q < (size_t)ncross * (size_t)m * (size_t)S; q++) p2p[q] = -1;
+
+    for (int s = 0; s < S; s++) {
+        /* GPipe program on stage s: FWD of micro-batches 0..m-1, BWD of m-1..0, then OPT once */
+        long np = 0;
+        for (int j = 0; j < m; j++)
+            for (uint32_t o = 0; o < N; o++)
+                if (T->ops[o].phase == PH_FWD && stage_of_layer[T->ops[o].layer] == s) { prog_op[np] = (int)o; prog_mb[np++] = j; }
+        for (int j = m - 1; j >= 0; j--)
+            for (uint32_t o = 0; o < N; o++)
+                if (T->ops[o].phase == PH_BWD && stage_of_layer[T->ops[o].layer] == s) { prog_op[np] = (int)o; prog_mb[np++] = j; }
+        for (uint32_t o = 0; o < N; o++)
+            if (T->ops[o].phase == PH_OPT && stage_of_layer[T->ops[o].layer] == s) { prog_op[np] = (int)o; prog_mb[np++] = 0; }
+        int prev_send = -1;
+        for (long q = 0; q < np; q++) {
+            int o = prog_op[q], j = prog_mb[q];
+            int t = add_task(G, ro[s], q, op_time(T, (uint32_t)o, r_b, 1, pt->tp_mode));
+            inst[(size_t)o * m + j] = t;
+            /* "send its output data to the next GPU. Simultaneously ... the next micro-batch"
+             * (P:190): push every produced tensor to each other stage that reads it, FIFO per
+             * sending GPU (reading Q14/Q15) */
+            const OOp *op = &T->ops[o];
+            for (uint32_t k = 0; k < op->n_out; k++) {
+                uint32_t x = T->io[op->io_off + op->n_in + k];
+                if (xidx[x] < 0) continue;
+                for (int d = 0; d < S; d++) {
+                    if (d == s || !(readers[x] & (1ull << d))) continue;
+                    double b = tensor_bytes(T, x, r_b, 1, pt->tp_mode);
+                    int f = add_flow(G, ro[s], ro[d], b, p2p_flow_code(x, j, ro[d]), NF_P2P);
+                    g_dep(G, f, t);
+                    if (prev_send >= 0) g_dep(G, f, prev_send);
+                    prev_send = f;
+                    p2p[((size_t)xidx[x] * m + j) * S + d] = f;
+                }
+            }
+        }
+    }
+    /* consumers wait for the delivery of every remote input ("execution cannot start
+     * until the data is available") */
+    for (uint32_t o = 0; o < N; o++) {
+        const OOp *op = &T->ops[o];
+        int s = stage_of_layer[op->layer];
+        int nj = (op->phase == PH_OPT) ? 1 : m;
+        for (int j = 0; j < nj; j++) {
+            int t = inst[(size_t)o * m + j];
+            for (uint32_t k = 0; k < op->n_in; k++) {
+                uint32_t x = T->io[op->io_off + k];
+                int po = T->prod[x];
+                if (po < 0 || stage_of_layer[T->ops[po].layer] == s) continue;
+                int jp = (T->ops[po].phase == PH_OPT || op->phase == PH_OPT) ? 0 : j;
+                int f = p2p[((size_t)xidx[x] * m + jp) * S + s];
+                if (f < 0) return -1;
+                g_dep(G, t, f);
+            }
+        }
+    }
+    free(stage_of_layer); free(inst); free(prog_op); free(prog_mb); free(readers); free(xidx); free(p2p);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Water-filling (R14; "bandwidth sharing between streams",        */
+/* P:210 "allocate bandwidth for the links on the route", reading Q18:  */
+/* max-min fair progressive filling).                                   */
+/* ------------------------------------------------------------------ */
+typedef struct {
+    int n_links;
+    double *bw;      /* per-point link bandwidth */
+    int *n_e, *k_e;
+    double *res, *share;
+} WF;
+
+/* flows[0..nf): route given by (roff, rlen) into rlinks; writes rate[]; returns rounds */
+static long waterfill(WF *w, int nf, const int *flows, const long *roff, const int *rlen, const int *rlinks,
+                      double *rate, char *unfrozen) {
+    for (int e = 0; e < w->n_links; e++) { w->n_e[e] = 0; w->k_e[e] = 0; w->res[e] = w->bw[e]; }
+    for (int a = 0; a < nf; a++) {
+        int f = flows[a];
+        for (int h = 0; h < rlen[f]; h++) w->n_e[rlinks[roff[f] + h]]++;
+        unfrozen[a] = 1;
+    }
+    int left = nf;
+    long rounds = 0;
+    while (left > 0) {
+        double s = INFINITY;
+        for (int e = 0; e < w->n_links; e++)
+            if (w->n_e[e] > 0) {
+                w->share[e] = w->res[e] / (double)w->n_e[e];
+                if (w->share[e] < s) s = w->share[e];
+            }
+        /* F_r: unfrozen flows crossing a link whose share equals the minimum */
+        for (int a = 0; a < nf; a++) {
+            if (!unfrozen[a]) continue;
+            int f = flows[a], inb = 0;
+            for (int h = 0; h < rlen[f]; h++) {
+                int e = rlinks[roff[f] + h];
+                if (w->n_e[e] > 0 && w->share[e] == s) inb = 1;
+            }
+            if (inb) {
+                rate[a] = s;
+                unfrozen[a] = 2; /* mark: frozen this round */
+                for (int h = 0; h < rlen[f]; h++) w->k_e[rlinks[roff[f] + h]]++;
+            }
+        }
+        for (int e = 0; e < w->n_links; e++)
+            if (w->k_e[e] > 0) {
+                double r = w->res[e] - s * (double)w->k_e[e];
+                w->res[e] = r > 0.0 ? r : 0.0;
+                w->n_e[e] -= w->k_e[e];
+                w->k_e[e] = 0;
+            }
+        for (int a = 0; a < nf; a++)
+            if (unfrozen[a] == 2) { unfrozen[a] = 0; left--; }
+        rounds++;
+    }
+    return rounds;
+}
+
+/* ------------------------------------------------------------------ */
+/* Order hash helpers (R19)                                             */
+/* ------------------------------------------------------------------ */
+static uint64_t mix64(uint64_t z) {
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    return z ^ (z >> 31);
+}
+static uint64_t fnv_u64(uint64_t h, uint64_t v) {
+    for (int b = 0; b < 8; b++) { h ^= (v >> (8 * b)) & 0xff; h *= 0x100000001b3ull; }
+    return h;
+}
+static uint64_t dbits(double d) { uint64_t u; memcpy(&u, &d, 8); return u; }
+
+/* ------------------------------------------------------------------ */
+/* The event-driven timeline (R13-R17)                                  */
+/* ------------------------------------------------------------------ */
+enum { S_WAIT = 0, S_QUEUED = 1, S_RUN = 2, S_LATENT = 3, S_ACTIVE = 4, S_DONE = 5 };
+
+static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale, OResult *res, double *t_done) {
+    long NN = G->count;
+    int n_nodes_topo = (int)tp->n_nodes;
+    /* dependency CSR (forward) and dependents CSR (reverse) */
+    long NE = G->dep_from.n;
+    long *doff = (long *)calloc((size_t)NN + 1, sizeof(long)), *roff = (long *)calloc((size_t)NN + 1, sizeof(long));
+    int *dlist = (int *)malloc(sizeof(int) * (size_t)(NE ? NE : 1)), *rlist = (int *)malloc(sizeof(int) * (size_t)(NE ? NE : 1));
+    int *pending = (int *)calloc((size_t)(NN ? NN : 1), sizeof(int));
+    if (!doff || !roff || !dlist || !rlist || !pending) return -1;
+    for (long e = 0; e < NE; e++) { doff[G->dep_from.v[e] + 1]++; roff[G->dep_to.v[e] + 1]++; }
+    for (long i = 0; i < NN; i++) { doff[i + 1] += doff[i]; roff[i + 1] += roff[i]; }
+    {
+        long *fd = (long *)calloc((size_t)NN + 1, sizeof(long)), *fr = (long *)calloc((size_t)NN + 1, sizeof(long));
+        for (long e = 0; e < NE; e++) {
+            int a = G->dep_from.v[e], b = G->dep_to.v[e];
+            dlist[doff[a] + fd[a]++] = b;
+            rlist[roff[b] + fr[b]++] = a;
+        }
+        free(fd); free(fr);
+    }
+    for (long i = 0; i < NN; i++) pending[i] = (int)(doff[i + 1] - doff[i]);
+
+    /* per-GPU in-order queues */
+    int *qoff = (int *)calloc((size_t)n_nodes_topo + 1, sizeof(int));
+    for (long i = 0; i < NN; i++) if (G->n[i].type == N_TASK) qoff[G->n[i].gpu + 1]++;
+    for (int g = 0; g < n_nodes_topo; g++) qoff[g + 1] += qoff[g];
+    int *qlist = (int *)malloc(sizeof(int) * (size_t)(qoff[n_nodes_topo] ? qoff[n_nodes_topo] : 1));
+    {
+        int *fq = (int *)calloc((size_t)n_nodes_topo, sizeof(int));
+        for (long i = 0; i < NN; i++) if (G->n[i].type == N_TASK) { int g = G->n[i].gpu; qlist[qoff[g] + fq[g]++] = (int)i; }
+        free(fq);
+    }
+    int *head = (int *)calloc((size_t)n_nodes_topo, sizeof(int)), *running = (int *)malloc(sizeof(int) * (size_t)n_nodes_topo);
+    for (int g = 0; g < n_nodes_topo; g++) running[g] = -1;
+
+    /* compute_busy_max: per GPU left fold of t' in program order (R18) */
+    double cbmax = 0.0;
+    long n_tasks = 0, n_flows = 0, n_p2p = 0;
+    for (int g = 0; g < n_nodes_topo; g++) {
+        double b = 0.0;
+        for (int q = qoff[g]; q < qoff[g + 1]; q++) b = b + G->n[qlist[q]].dur;
+        if (b > cbmax) cbmax = b;
+    }
+
+    /* routes: per flow, BFS route (cached per ordered GPU pair) */
+    long *froff = (long *)calloc((size_t)(NN ? NN : 1), sizeof(long));
+    int *frlen = (int *)calloc((size_t)(NN ? NN : 1), sizeof(int));
+    IVec rpool = {0};
+    long *pair_off = (long *)malloc(sizeof(long) * (size_t)n_nodes_topo * (size_t)n_nodes_topo);
+    int *pair_len = (int *)malloc(sizeof(int) * (size_t)n_nodes_topo * (size_t)n_nodes_topo);
+    for (long q = 0; q < (long)n_nodes_topo * n_nodes_topo; q++) pair_len[q] = -9;
+    int *tmp = (int *)malloc(sizeof(int) * (size_t)(n_nodes_topo + 1));
+    double *lat = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+    int status = PT_OK;
+    for (long i = 0; i < NN; i++) {
+        if (G->n[i].type != N_FLOW) continue;
+        n_flows++;
+        if (G->n[i].flags & NF_P2P) n_p2p++;
+        int s = G->n[i].src, d = G->n[i].dst;
+        long key = (long)s * n_nodes_topo + d;
+        if (pair_len[key] == -9) {
+            int h = bfs_route(tp, s, d, tmp, n_nodes_topo);
+            pair_off[key] = rpool.n;
+            pair_len[key] = h;
+            for (int k = 0; k < h; k++) iv_push(&rpool, tmp[k]);
+        }
+        if (pair_len[key] < 0) { status = PT_NO_ROUTE; break; }
+        froff[i] = pair_off[key];
+        frlen[i] = pair_len[key];
+        /* route latency: left fold of per-link latencies (R12/R13) */
+        double L = 0.0;
+        for (int k = 0; k < frlen[i]; k++) L = L + tp->links[rpool.v[froff[i] + k]].lat * lat_scale;
+        lat[i] = L;
+    }
+    for (long i = 0; i < NN; i++) if (G->n[i].type == N_TASK) n_tasks++;
+
+    memset(res, 0, sizeof *res);
+    if (status != PT_OK) {
+        res->status = status;
+        goto out;
+    }
+    {
+        WF w;
+        w.n_links = (int)tp->n_links;
+        w.bw = (double *)malloc(sizeof(double) * (size_t)(w.n_links ? w.n_links : 1));
+        w.n_e = (int *)malloc(sizeof(int) * (size_t)(w.n_links ? w.n_links : 1));
+        w.k_e = (int *)malloc(sizeof(int) * (size_t)(w.n_links ? w.n_links : 1));
+        w.res = (double *)malloc(sizeof(double) * (size_t)(w.n_links ? w.n_links : 1));
+        w.share = (double *)malloc(sizeof(double) * (size_t)(w.n_links ? w.n_links : 1));
+        for (int e = 0; e < w.n_links; e++) w.bw[e] = tp->links[e].bw * bw_scale;
+
+        int *state = (int *)calloc((size_t)(NN ? NN : 1), sizeof(int));
+        double *t_end = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        double *t_act = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        double *rem = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        double *rate = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        double *t_upd = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        double *t_drain = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        char *has_dependents = (char *)calloc((size_t)(NN ? NN : 1), 1);
+        for (long i = 0; i < NN; i++) has_dependents[i] = roff[i + 1] > roff[i];
+        IVec ready = {0}, latent = {0}, active = {0};
+        int *wf_flows = (int *)malloc(sizeof(int) * (size_t)(NN ? NN : 1));
+        double *wf_rate = (double *)malloc(sizeof(double) * (size_t)(NN ? NN : 1));
+        char *wf_unf = (char *)malloc((size_t)(NN ? NN : 1));
+        for (long i = 0; i < NN; i++)
+            if (pending[i] == 0 && G->n[i].type != N_TASK) { iv_push(&ready, (int)i); state[i] = S_QUEUED; }
+
+        long n_done = 0;
+        double t = 0.0;
+        uint64_t H = 0xcbf29ce484222325ull;
+        uint64_t n_inst = 0, n_wf = 0, n_rounds = 0;
+        uint32_t max_act = 0;
+        int busy_on = 0;
+        double busy_start = 0.0, comm_busy = 0.0;
+        long inflight = 0;
+
+#define COMPLETE(i)                                                          \
+    do {                                                                     \
+        state[i] = S_DONE; n_done++;                                         \
+        if (t_done) t_done[i] = t;                                           \
+        for (long _r = roff[i]; _r < roff[(i) + 1]; _r++) {                  \
+            int _d = rlist[_r];                                              \
+            if (--pending[_d] == 0 && G->n[_d].type != N_TASK) {             \
+                iv_push(&ready, _d); state[_d] = S_QUEUED;                   \
+            }                                                                \
+        }                                                                    \
+    } while (0)
+#define EVENT(kind, code) do { acc += mix64(((uint64_t)(kind) << 60) | (code)); nev++; } while (0)
+
+        for (;;) {
+            uint64_t acc = 0;
+            long nev = 0;
+            int again;
+            int dirty = 0;
+            do {
+                int changed;
+                do {
+                    changed = 0;
+                    /* (a) compute completions */
+                    for (int g = 0; g < n_nodes_topo; g++) {
+                        int k = running[g];
+                        if (k >= 0 && t_end[k] == t) {
+                            COMPLETE(k);
+                            if (has_dependents[k]) EVENT(EV_TASK_END, G->n[k].code);
+                            running[g] = -1;
+                            changed = 1;
+                        }
+                    }
+                    /* (b) deliveries: push to the destination, notify the receiver */
+                    for (long a = 0; a < active.n;) {
+                        int f = active.v[a];
+                        if (t_drain[f] == t) {
+                            active.v[a] = active.v[--active.n];
+                            COMPLETE(f);
+                            EVENT(EV_DELIVER, G->n[f].code);
+                            inflight--;
+                            dirty = 1; changed = 1;
+                        } else {
+                            a++;
+                        }
+                    }
+                    /* (c) activations after the route latency (reading Q19: latency first) */
+                    for (long a = 0; a < latent.n;) {
+                        int f = latent.v[a];
+                        if (t_act[f] == t) {
+                            latent.v[a] = latent.v[--latent.n];
+                            EVENT(EV_ACTIVATE, G->n[f].code);
+                            if (G->n[f].bytes == 0.0 || frlen[f] == 0) {
+                                COMPLETE(f);
+                                EVENT(EV_DELIVER, G->n[f].code);
+                                inflight--;
+                            } else {
+                                state[f] = S_ACTIVE;
+                                rem[f] = G->n[f].bytes; t_upd[f] = t; rate[f] = 0.0; t_drain[f] = INFINITY;
+                                iv_push(&active, f);
+                                dirty = 1;
+                            }
+                            changed = 1;
+                        } else {
+                            a++;
+                        }
+                    }
+                    /* (d) dependency resolution: barriers fire, flows are released */
+                    while (ready.n > 0) {
+                        int k = ready.v[--ready.n];
+                        if (G->n[k].type == N_BARRIER) {
+                            COMPLETE(k);
+                            if (G->n[k].flags & NF_COLL_START) EVENT(EV_COLL_START, G->n[k].code);
+                        } else {
+                            state[k] = S_LATENT;
+                            t_act[k] = t + lat[k];
+                            EVENT(EV_RELEASE, G->n[k].code);
+                            iv_push(&latent, k);
+                            inflight++;
+                        }
+                        changed = 1;
+                    }
+                    /* (e) an idle GPU starts its head operator once its data is present */
+                    for (int g = 0; g < n_nodes_topo; g++) {
+                        if (running[g] >= 0 || head[g] >= qoff[g + 1] - qoff[g]) continue;
+                        int k = qlist[qoff[g] + head[g]];
+                        if (pending[k] != 0) continue;
+                        running[g] = k; head[g]++;
+                        state[k] = S_RUN;
+                        t_end[k] = t + G->n[k].dur;
+                        if (doff[k + 1] > doff[k]) EVENT(EV_TASK_START, G->n[k].code);
+                        changed = 1;
+                    }
+                } while (changed);
+                /* (f) re-allocate bandwidth of every in-transit flow */
+                again = 0;
+                if (dirty) {
+                    dirty = 0;
+                    int nf = (int)active.n;
+                    for (int a = 0; a < nf; a++) {
+                        int f = active.v[a];
+                        wf_flows[a] = f;
+                        if (t_upd[f] < t) {
+                            double r = rem[f] - rate[f] * (t - t_upd[f]);
+                            rem[f] = r > 0.0 ? r : 0.0;
+                            t_upd[f] = t;
+                        }
+                    }
+                    n_rounds += (uint64_t)waterfill(&w, nf, wf_flows, froff, frlen, rpool.v, wf_rate, wf_unf);
+                    n_wf++;
+                    if ((uint32_t)nf > max_act) max_act = (uint32_t)nf;
+                    for (int a = 0; a < nf; a++) {
+                        int f = wf_flows[a];
+                        rate[f] = wf_rate[a];
+                        t_drain[f] = (rem[f] == 0.0) ? t : t + rem[f] / rate[f];
+                        if (t_drain[f] == t) again = 1;
+                    }
+                }
+            } while (again);
+
+            if (nev > 0) { n_inst++; H = fnv_u64(H, dbits(t)); H = fnv_u64(H, acc); }
+            if (inflight > 0 && !busy_on) { busy_on = 1; busy_start = t; }
+            else if (inflight == 0 && busy_on) { busy_on = 0; comm_busy = comm_busy + (t - busy_start); }
+            if (n_done == NN) break;
+            double tn = INFINITY;
+            for (int g = 0; g < n_nodes_topo; g++) if (running[g] >= 0 && t_end[running[g]] < tn) tn = t_end[running[g]];
+            for (long a = 0; a < latent.n; a++) if (t_act[latent.v[a]] < tn) tn = t_act[latent.v[a]];
+            for (long a = 0; a < active.n; a++) if (t_drain[active.v[a]] < tn) tn = t_drain[active.v[a]];
+            if (!(tn < INFINITY)) { status = PT_DEADLOCK; break; }
+            t = tn;
+        }
+#undef COMPLETE
+#undef EVENT
+        if (status == PT_OK) {
+            res->iter_time_s = t;
+            res->compute_busy_max_s = cbmax;
+            res->comm_busy_s = comm_busy;
+            res->exposed_comm_s = t - cbmax;
+            res->coll_payload_bytes = G->coll_payload;
+            res->n_compute = (uint64_t)n_tasks;
+            res->n_flows = (uint64_t)n_flows;
+            res->n_collectives = (uint64_t)G->n_coll;
+            res->n_p2p = (uint64_t)n_p2p;
+            res->n_instants = n_inst;
+            res->n_wf_calls = n_wf;
+            res->n_wf_rounds = n_rounds;
+            res->order_hash = H;
+            res->max_active_flows = max_act;
+        }
+        res->status = status;
+        free(w.bw); free(w.n_e); free(w.k_e); free(w.res); free(w.share);
+        free(state); free(t_end); free(t_act); free(rem); free(rate); free(t_upd); free(t_drain); free(has_dependents);
+        iv_free(&ready); iv_free(&latent); iv_free(&active);
+        free(wf_flows); free(wf_rate); free(wf_unf);
+    }
+out:
+    free(doff); free(roff); free(dlist); free(rlist); free(pending);
+    free(qoff); free(qlist); free(head); free(running);
+    free(froff); free(frlen); iv_free(&rpool); free(pair_off); free(pair_len); free(tmp); free(lat);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Public entry points (called through ctypes by tests / bench only)   */
+/* ------------------------------------------------------------------ */
+static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_order, const uint32_t *plan,
+                       uint32_t plan_len, int have_plan, const OPoint *pt, Graph *G, int *status) {
+    *status = point_check(T, tp, pt, plan, plan_len, have_plan);
+    if (*status != PT_OK) return 0;
+    int *ro = (int *)malloc(sizeof(int) * tp->n_gpus);
+    if (!ro) return -1;
+    ring_order_of(ring_order, tp->n_gpus, ro);
+    int rc = 0;
+    switch (pt->strategy) {
+    case ST_DP: case ST_DDP: rc = expand_dp(T, pt, ro, G); break;
+    case ST_TP: rc = expand_tp(T, pt, ro, G); break;
+    case ST_PP: {
+        uint32_t *fl = (uint32_t *)malloc(sizeof(uint32_t) * pt->pp);
+        if (have_plan) memcpy(fl, plan, sizeof(uint32_t) * pt->pp);
+        else if (auto_partition(T, pt->pp, fl)) { free(fl); free(ro); return -1; }
+        rc = expand_pp(T, pt, ro, fl, G);
+        free(fl);
+        break;
+    }
+    default:
+        *status = PT_BAD_CONFIG; /* HYBRID: not built in this oracle revision */
+        break;
+    }
+    free(ro);
+    return rc;
+}
+
+int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
+                     uint32_t n_io, uint32_t trace_batch, uint32_t n_nodes, uint32_t n_gpus, const OLink *links,
+                     uint32_t n_links, const uint32_t *ring_order, const uint32_t *plan, uint32_t plan_len,
+                     int have_plan, const OPoint *pt, OResult *out) {
+    Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
+    Topo tp; memset(&tp, 0, sizeof tp);
+    int rc = trace_check(&T);
+    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc == O_OK && ring_order) {
+        for (uint32_t i = 0; i < n_gpus; i++) {
+            if (ring_order[i] >= n_gpus) rc = O_EINVAL;
+            for (uint32_t j = 0; j < i; j++) if (ring_order[j] == ring_order[i]) rc = O_EINVAL;
+        }
+    }
+    if (rc != O_OK) { free(T.prod); topo_free(&tp); return rc; }
+    Graph G; memset(&G, 0, sizeof G);
+    int status = PT_OK;
+    memset(out, 0, sizeof *out);
+    if (build_graph(&T, &tp, ring_order, plan, plan_len, have_plan, pt, &G, &status)) rc = O_ENOMEM;
+    else if (status != PT_OK) out->status = status;
+    else if (simulate(&G, &tp, pt->bw_scale, pt->lat_scale, out, NULL)) rc = O_ENOMEM;
+    g_free(&G); free(T.prod); topo_free(&tp);
+    return rc;
+}
+
+/* Export the explicit task graph of one point (for the exact-rational re-simulation in
+ * tests/).  Two calls: with arrays NULL to get the sizes, then with arrays to fill. */
+int oracle_export_graph(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
+                        uint32_t n_io, uint32_t trace_batch, uint32_t n_nodes, uint32_t n_gpus, const OLink *links,
+                        uint32_t n_links, const uint32_t *ring_order, const uint32_t *plan, uint32_t plan_len,
+                        int have_plan, const OPoint *pt, int64_t *n_graph_nodes, int64_t *n_graph_deps,
+                        int32_t *type, int32_t *gpu, double *dur, int32_t *src, int32_t *dst, double *bytes,
+                        uint64_t *code, int32_t *flags, int64_t *dep_off, int32_t *dep_ids, int32_t *status) {
+    Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
+    Topo tp; memset(&tp, 0, sizeof tp);
+    int rc = trace_check(&T);
+    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc != O_OK) { free(T.prod); topo_free(&tp); return rc; }
+    Graph G; memset(&G, 0, sizeof G);
+    int st = PT_OK;
+    if (build_graph(&T, &tp, ring_order, plan, plan_len, have_plan, pt, &G, &st)) rc = O_ENOMEM;
+    *status = st;
+    *n_graph_nodes = G.count;
+    *n_graph_deps = G.dep_from.n;
+    if (rc == O_OK && type) {
+        for (long i = 0; i < G.count; i++) {
+            type[i] = G.n[i].type; gpu[i] = G.n[i].gpu; dur[i] = G.n[i].dur;
+            src[i] = G.n[i].src; dst[i] = G.n[i].dst; bytes[i] = G.n[i].bytes;
+            code[i] = G.n[i].code; flags[i] = G.n[i].flags;
+        }
+        for (long i = 0; i <= G.count; i++) dep_off[i] = 0;
+        for (long e = 0; e < G.dep_from.n; e++) dep_off[G.dep_from.v[e] + 1]++;
+        for (long i = 0; i < G.count; i++) dep_off[i + 1] += dep_off[i];
+        int64_t *fill = (int64_t *)calloc((size_t)(G.count > 0 ? G.count : 0) + 1, sizeof(int64_t));
+        for (long e = 0; e < G.dep_from.n; e++) {
+            int a = G.dep_from.v[e];
+            dep_ids[dep_off[a] + fill[a]++] = G.dep_to.v[e];
+        }
+        free(fill);
+    }
+    g_free(&G); free(T.prod); topo_free(&tp);
+    return rc;
+}
+
+/* Simulate an explicit task graph given as arrays (same layout as the export). */
+int oracle_sim_graph(int64_t n, const int32_t *type, const int32_t *gpu, const double *dur, const int32_t *src,
+                     const int32_t *dst, const double *bytes, const uint64_t *code, const int32_t *flags,
+                     const int64_t *dep_off, const int32_t *dep_ids, int32_t n_coll, double coll_payload,
+                     uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links, double bw_scale,
+                     double lat_scale, OResult *out, double *t_done) {
+    Topo tp; memset(&tp, 0, sizeof tp);
+    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc != O_OK) { topo_free(&tp); return rc; }
+    Graph G; memset(&G, 0, sizeof G);
+    for (int64_t i = 0; i < n; i++) {
+        GNode nd; memset(&nd, 0, sizeof nd);
+        nd.type = type[i]; nd.gpu = gpu[i]; nd.dur = dur[i]; nd.src = src[i]; nd.dst = dst[i];
+        nd.bytes = bytes[i]; nd.code = code[i]; nd.flags = flags[i];
+        if (nd.type == N_TASK && (nd.gpu < 0 || (uint32_t)nd.gpu >= n_nodes)) { rc = O_EINVAL; break; }
+        if (nd.type == N_FLOW && (nd.src < 0 || nd.dst < 0 || (uint32_t)nd.src >= n_nodes || (uint32_t)nd.dst >= n_nodes)) { rc = O_EINVAL; break; }
+        if (g_add(&G, nd) < 0) { rc = O_ENOMEM; break; }
+        for (int64_t q = dep_off[i]; q < dep_off[i + 1]; q++) {
+            if (dep_ids[q] < 0 || dep_ids[q] >= n) { rc = O_EINVAL; break; }
+            g_dep(&G, (int)i, dep_ids[q]);
+        }
+        if (rc) break;
+    }
+    G.n_coll = n_coll;
+    G.coll_payload = coll_payload;
+    if (rc == O_OK && simulate(&G, &tp, bw_scale, lat_scale, out, t_done)) rc = O_ENOMEM;
+    g_free(&G); topo_free(&tp);
+    return rc;
+}
+
+/* Standalone pieces for the pin tests */
+int oracle_route(uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links, uint32_t src, uint32_t dst,
+                 int32_t *out_links, int32_t cap) {
+    Topo tp; memset(&tp, 0, sizeof tp);
+    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc != O_OK) { topo_free(&tp); return -100 + rc; }
+    int *tmp = (int *)malloc(sizeof(int) * (size_t)(n_nodes + 1));
+    int h = bfs_route(&tp, (int)src, (int)dst, tmp, (int)n_nodes);
+    for (int k = 0; k < h && k < cap; k++) out_links[k] = tmp[k];
+    free(tmp); topo_free(&tp);
+    return h;
+}
+
+int64_t oracle_waterfill(int32_t n_links, const double *bw, int32_t n_flows, const int64_t *route_off,
+                         const int32_t *route_len, const int32_t *route_links, double *rate_out) {
+    WF w;
+    w.n_links = n_links;
+    w.bw = (double *)malloc(sizeof(double) * (size_t)(n_links ? n_links : 1));
+    w.n_e = (int *)malloc(sizeof(int) * (size_t)(n_links ? n_links : 1));
+    w.k_e = (int *)malloc(sizeof(int) * (size_t)(n_links ? n_links : 1));
+    w.res = (double *)malloc(sizeof(double) * (size_t)(n_links ? n_links : 1));
+    w.share = (double *)malloc(sizeof(double) * (size_t)(n_links ? n_links : 1));
+    memcpy(w.bw, bw, sizeof(double) * (size_t)n_links);
+    int *flows = (int *)malloc(sizeof(int) * (size_t)(n_flows ? n_flows : 1));
+    long *roff = (long *)malloc(sizeof(long) * (size_t)(n_flows ? n_flows : 1));
+    int *rlen = (int *)malloc(sizeof(int) * (size_t)(n_flows ? n_flows : 1));
+    char *unf = (char *)malloc((size_t)(n_flows ? n_flows : 1));
+    long tot = 0;
+    for (int f = 0; f < n_flows; f++) { flows[f] = f; roff[f] = (long)route_off[f]; rlen[f] = route_len[f]; tot = roff[f] + rlen[f] > tot ? roff[f] + rlen[f] : tot; }
+    int *rl = (int *)malloc(sizeof(int) * (size_t)(tot ? tot : 1));
+    for (long q = 0; q < tot; q++) rl[q] = route_links[q];
+    long rounds = waterfill(&w, n_flows, flows, roff, rlen, rl, rate_out, unf);
+    free(w.bw); free(w.n_e); free(w.k_e); free(w.res); free(w.share);
+    free(flows); free(roff); free(rlen); free(unf); free(rl);
+    return rounds;
+}
+
+int oracle_partition(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
+                     uint32_t n_io, uint32_t trace_batch, uint32_t n_stages, uint32_t *first_layer) {
+    Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
+    int rc = trace_check(&T);
+    if (rc == O_OK) rc = auto_partition(&T, (int)n_stages, first_layer) ? O_EINVAL : O_OK;
+    free(T.prod);
+    return rc;
+}
+
+int oracle_check_trace(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
+                       uint32_t n_io, uint32_t trace_batch, uint32_t *n_layers) {
+    Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
+    int rc = trace_check(&T);
+    if (n_layers) *n_layers = T.n_layers;
+    free(T.prod);
+    return rc;
+}
