@@ -1,0 +1,227 @@
+/*
+ * triosim.h -- C ABI of libtriosim.so, the B200-native batched design-point
+ * simulator of TrioSim (Li et al., ISCA'25; PAPER.md = "P:N" line refs).
+ *
+ * A design point = (parallelism strategy, degrees, topology + bandwidth /
+ * latency scale, batch size, ...).  For every point the library runs the three
+ * steps of the paper's method on the GPU (DESIGN.md "Semantics" R1-R19):
+ *   1. operator-time model on the single-GPU trace,
+ *   2. trace extrapolation of DP / DDP / TP / PP into compute tasks and
+ *      collective / point-to-point flows,
+ *   3. an event-driven timeline whose in-transit flows share link bandwidth by
+ *      max-min fair progressive filling, re-allocated whenever a flow starts or
+ *      completes (Fig. 5),
+ * and returns the predicted iteration time plus breakdowns.
+ *
+ * Conventions: all structs are little-endian with natural alignment (sizes are
+ * asserted below).  Times are seconds, bandwidths bytes/s, sizes bytes, IEEE
+ * binary64.  Entry points return a triosim_status (0 = OK, < 0 = error); the
+ * message of the last error is available from triosim_last_error().  A context
+ * is bound to one CUDA device and is not thread-safe (use one per thread).
+ * Every input array is deep-copied during the call: the caller may free it as
+ * soon as the call returns.  There is no CPU fallback: if the CUDA device is
+ * missing or not sm_100, triosim_create fails with TRIOSIM_EUNSUPPORTED.
+ */
+#ifndef TRIOSIM_H
+#define TRIOSIM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t triosim_status;
+#define TRIOSIM_OK 0
+#define TRIOSIM_EINVAL (-1)       /* malformed input table / argument */
+#define TRIOSIM_ENOMEM (-2)       /* host or device allocation failed */
+#define TRIOSIM_ECUDA (-3)        /* CUDA runtime error (sticky errors reported on the next call) */
+#define TRIOSIM_ENOTFOUND (-4)    /* unknown trace / sweep handle */
+#define TRIOSIM_ERANGE (-5)       /* point range outside the sweep */
+#define TRIOSIM_EUNSUPPORTED (-6) /* no sm_100 device */
+
+/* per-point status in triosim_result.status (R3) */
+#define TRIOSIM_PT_OK 0
+#define TRIOSIM_PT_BAD_BATCH 1   /* global_batch not divisible by dp * microbatches (Q3, Q12) */
+#define TRIOSIM_PT_BAD_DEGREES 2 /* zero / inconsistent degrees, dp*tp*pp > GPUs, pp > layers or > 64 */
+#define TRIOSIM_PT_NO_ROUTE 3    /* a needed (src, dst) GPU pair has no path */
+#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 32 lanes, > 128 links, > 8 hops) */
+#define TRIOSIM_PT_DEADLOCK 5    /* the task graph cannot make progress */
+#define TRIOSIM_PT_BAD_PLAN 6    /* explicit stage plan invalid for this point */
+#define TRIOSIM_PT_BAD_CONFIG 7  /* unknown enum, topology index out of range, bw_scale <= 0, lat_scale < 0 */
+
+/* operator phases, tensor categories, TP roles */
+#define TRIOSIM_PHASE_FWD 0
+#define TRIOSIM_PHASE_BWD 1
+#define TRIOSIM_PHASE_OPT 2
+#define TRIOSIM_CAT_INPUT 0
+#define TRIOSIM_CAT_WEIGHT 1
+#define TRIOSIM_CAT_WGRAD 2
+#define TRIOSIM_CAT_ACT 3
+#define TRIOSIM_CAT_AGRAD 4
+#define TRIOSIM_CAT_OTHER 5
+#define TRIOSIM_ROLE_NONE 0   /* bits 0-1: Megatron role */
+#define TRIOSIM_ROLE_COL 1
+#define TRIOSIM_ROLE_ROW 2
+#define TRIOSIM_ROLE_LOCAL 3
+#define TRIOSIM_ROLE_GATHER 4 /* bit 2: paper-mode split layer (conv / linear / embedding) */
+#define TRIOSIM_OPF_BATCH_SCALED 1u
+
+/* One operator of the single-GPU trace, in program order ("operator name, measured
+ * execution time, and input/output as a list of tensor IDs").  Phases must be FWD* BWD* OPT*;
+ * layer ids are numbered by first FWD appearance (0, 1, 2, ...).  io[io_off .. io_off+n_in)
+ * are the inputs, the next n_out entries the outputs. */
+typedef struct {
+    uint32_t kind;    /* operator name id (informational) */
+    uint32_t layer;
+    uint8_t phase;
+    uint8_t tp_role;
+    uint16_t flags;   /* TRIOSIM_OPF_* */
+    uint32_t io_off;
+    uint16_t n_in, n_out;
+    uint32_t pad;
+    double time_s;    /* measured time on the trace GPU at trace_batch */
+    double flops;     /* informational */
+} triosim_op;         /* 40 B */
+
+/* One tensor: bytes at the trace batch, category, batch dependence. */
+typedef struct {
+    uint64_t bytes_b0;
+    uint8_t category;
+    uint8_t batch_scaled;
+    uint16_t pad;
+    uint32_t param_id;
+} triosim_tensor;     /* 16 B */
+
+typedef struct {
+    uint32_t n_ops, n_tensors, n_io, trace_batch;
+    const triosim_op *ops;          /* host pointers */
+    const triosim_tensor *tensors;
+    const uint32_t *io;
+} triosim_trace_desc;
+
+/* Directed link (P:142 topology input, P:226 bandwidth is a user input). */
+typedef struct {
+    uint32_t src, dst;  /* node ids; GPUs are nodes [0, n_gpus), switches after */
+    double bw_Bps;      /* > 0 */
+    double lat_s;       /* >= 0 */
+} triosim_link;         /* 24 B */
+
+typedef struct {
+    uint32_t n_nodes, n_gpus, n_links, pad;
+    const triosim_link *links;      /* at most one link per ordered pair */
+    const uint32_t *ring_order;     /* permutation of [0, n_gpus) or NULL (= identity) */
+} triosim_topology;
+
+/* Explicit PP stage plans: plan k has first_layer[off[k] .. off[k+1]) (first must be 0,
+ * strictly increasing); a point selects one with stage_plan = k, or -1 = automatic. */
+typedef struct {
+    uint32_t n_plans;
+    const uint32_t *off;            /* n_plans + 1 entries */
+    const uint32_t *first_layer;
+} triosim_stage_plans;
+
+#define TRIOSIM_DP 0      /* DataParallel: gradient AllReduce after the backward pass */
+#define TRIOSIM_DDP 1     /* DistributedDataParallel: AllReduce overlapped with backward */
+#define TRIOSIM_TP 2      /* tensor parallel */
+#define TRIOSIM_PP 3      /* GPipe pipeline parallel */
+#define TRIOSIM_HYBRID 4  /* reserved (DP x TP x PP): reported as PT_BAD_CONFIG in this revision */
+#define TRIOSIM_TP_PAPER 0
+#define TRIOSIM_TP_MEGATRON 1
+#define TRIOSIM_ALGO_RING 0
+#define TRIOSIM_ALGO_TREE 1
+
+typedef struct {
+    uint32_t topo;
+    uint8_t strategy, tp_mode, coll_algo, pad0;
+    uint16_t dp, tp, pp, pad1;
+    uint32_t microbatches, global_batch;
+    int32_t stage_plan;      /* -1 = automatic balanced partition */
+    uint32_t pad2;
+    uint64_t bucket_bytes;   /* DP/DDP gradient bucket; 0 = one AllReduce per tensor */
+    double bw_scale;         /* multiplies every link bandwidth (> 0) */
+    double lat_scale;        /* multiplies every link latency (>= 0) */
+} triosim_point;             /* 56 B */
+
+typedef struct {
+    double iter_time_s;          /* predicted iteration time T */
+    double compute_busy_max_s;   /* max over GPUs of summed operator time */
+    double comm_busy_s;          /* time with >= 1 flow in flight */
+    double exposed_comm_s;       /* T - compute_busy_max_s */
+    double coll_payload_bytes;   /* summed collective payloads ("amount of data ... AllReduce") */
+    uint64_t n_compute, n_flows, n_collectives, n_p2p;
+    uint64_t n_instants, n_wf_calls, n_wf_rounds, order_hash; /* DESIGN.md R19 */
+    int32_t status;              /* TRIOSIM_PT_* */
+    uint32_t max_active_flows;
+} triosim_result;                /* 112 B */
+
+#ifdef __cplusplus
+static_assert(sizeof(triosim_op) == 40, "op");
+static_assert(sizeof(triosim_tensor) == 16, "tensor");
+static_assert(sizeof(triosim_link) == 24, "link");
+static_assert(sizeof(triosim_point) == 56, "point");
+static_assert(sizeof(triosim_result) == 112, "result");
+#endif
+
+typedef struct triosim_ctx triosim_ctx;
+
+/* Create a context on CUDA device `cuda_device` (must be sm_100).  *out owns every device and
+ * host copy made later; free with triosim_destroy.  Errors: EUNSUPPORTED, ECUDA, ENOMEM. */
+triosim_status triosim_create(int cuda_device, triosim_ctx **out);
+void triosim_destroy(triosim_ctx *ctx);
+
+/* Message for the last error on ctx (owned by ctx, valid until the next call). */
+const char *triosim_last_error(const triosim_ctx *ctx);
+
+/* Trace ingest (S1).  Validates the tables (EINVAL: ids out of range, a tensor
+ * produced twice or read before it is produced, phases not FWD* BWD* OPT*, layers not numbered
+ * by first FWD appearance, negative / non-finite time, trace_batch == 0), copies them to the
+ * device and runs the ingest kernel.  Synchronous.  *trace_id receives the handle. */
+triosim_status triosim_load_trace(triosim_ctx *ctx, const triosim_trace_desc *t, int32_t *trace_id);
+
+/* Build a sweep of n_pts design points over trace_id (P:142 inputs).  Validates topologies
+ * (EINVAL: bad endpoints, bw <= 0, lat < 0, duplicate ordered pair, bad ring_order), computes
+ * routes (S5) and stage partitions on the host, groups points into structural classes and
+ * stages everything in device memory.  Invalid design points do NOT fail the call: they get a
+ * per-point status.  plans may be NULL.  Synchronous.  *sweep_id receives the handle. */
+triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const triosim_topology *topos,
+                                   uint32_t n_topos, const triosim_stage_plans *plans, const triosim_point *pts,
+                                   uint64_t n_pts, int32_t *sweep_id);
+
+/* Simulate points [first, first+count) of sweep_id: operator rescale (K1), task-graph
+ * expansion (K2) and the timeline kernel (K3) on `cuda_stream` (cudaStream_t; NULL = the
+ * legacy default stream).  Asynchronous and stream-ordered; returns after enqueue.
+ * Errors: ERANGE, ENOTFOUND, ECUDA. */
+triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
+                                      void *cuda_stream);
+
+/* Copy result records [first, first+count) to out.  out_is_device == 0: host memory, the call
+ * synchronises the stream of the last simulate_batch.  out_is_device != 0: a device pointer on
+ * the context's GPU; the copy is enqueued on `cuda_stream` (stream-ordered, asynchronous). */
+triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
+                               triosim_result *out, int out_is_device, void *cuda_stream);
+
+/* Free a trace or sweep handle (a trace must outlive its sweeps). */
+triosim_status triosim_release(triosim_ctx *ctx, int32_t handle);
+
+/* Kernel launch counters since the context was created (K1, K2, K3 launches), for the bench. */
+triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3);
+
+/* fp64 operations of the method (folds, latencies, progress, shares,
+ * residual updates, drain times) performed by the last simulate_batch of sweep_id.  Synchronises
+ * that call's stream. */
+triosim_status triosim_work_counters(triosim_ctx *ctx, int32_t sweep_id, uint64_t *fp64_ops);
+
+/* CUDA-event timing of simulate_batch calls (events recorded on the call's stream): enable
+ * resets the log; triosim_timings returns how many calls were logged (<= 512, <= max) and their
+ * durations in ms: whole call (K1b+K2+K3) and the K3 timeline phase (fork to join). */
+triosim_status triosim_timing(triosim_ctx *ctx, int enable);
+int32_t triosim_timings(triosim_ctx *ctx, float *ms_total, float *ms_k3, int32_t max);
+
+/* Device pointer of the sweep's result records (for stream-ordered gathers), or NULL. */
+const void *triosim_results_device_ptr(const triosim_ctx *ctx, int32_t sweep_id);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TRIOSIM_H */

@@ -99,19 +99,18 @@ def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None):
 
 
 def run_sweep(sw: W.Sweep, idx=None):
+    """Oracle results for points idx of a sweep; topology index and plan index are resolved
+    here in DESIGN.md R3 order (topology first, the plan inside the point checks)."""
     idx = range(len(sw.points)) if idx is None else idx
     res = np.zeros(len(idx), W.RESULT_DTYPE)
     for q, i in enumerate(idx):
         pt = sw.points[i]
-        plan = None
-        if pt["stage_plan"] >= 0 and pt["stage_plan"] < len(sw.plans):
-            plan = sw.plans[pt["stage_plan"]]
-        elif pt["stage_plan"] >= 0:
-            res[q]["status"] = W.PT_BAD_PLAN
-            continue
         if pt["topo"] >= len(sw.topos):
             res[q]["status"] = W.PT_BAD_CONFIG
             continue
+        plan = None
+        if pt["stage_plan"] >= 0:
+            plan = sw.plans[pt["stage_plan"]] if pt["stage_plan"] < len(sw.plans) else []
         res[q] = run_point(sw.trace, sw.topos[pt["topo"]], pt, plan)
     return res
 

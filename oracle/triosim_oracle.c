@@ -509,7 +509,7 @@ static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const u
     int piped = (pt->strategy == ST_PP || pt->strategy == ST_HYBRID);
     if (piped && m == 0) return PT_BAD_DEGREES;
     if ((uint64_t)dp * tpd * pp > tp->n_gpus) return PT_BAD_DEGREES;
-    if (pp > T->n_layers) return PT_BAD_DEGREES;
+    if (pp > T->n_layers || pp > 64) return PT_BAD_DEGREES;
     uint64_t mm = piped ? m : 1;
     if (pt->global_batch == 0 || pt->global_batch % ((uint64_t)dp * mm) != 0) return PT_BAD_BATCH;
     if (piped && have_plan) {

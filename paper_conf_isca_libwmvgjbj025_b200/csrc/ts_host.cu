@@ -1,0 +1,788 @@
+// ts_host.cu -- host side of libtriosim: the C ABI of include/triosim.h.
+//
+// load_trace   host validation + H2D + K1a ingest kernel
+// build_sweep  topology validation, BFS routes (S5), PP auto-partition,
+//              per-point status (R3), structural classes, device pools, work lists
+// simulate     K1b rescale + K2 expansion (all classes) + K3 timeline (requested points),
+//              stream-ordered on the caller's stream
+// results      D2H (synchronising) or stream-ordered D2D
+#include <cuda_runtime.h>
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <string>
+#include <tuple>
+#include <vector>
+#include "ts_internal.h"
+
+using namespace ts;
+
+namespace {
+
+template <class T>
+struct DevBuf {
+    T *p = nullptr;
+    size_t n = 0;
+    ~DevBuf() { if (p) cudaFree(p); }
+    cudaError_t alloc(size_t count) {
+        if (p) { cudaFree(p); p = nullptr; }
+        n = count;
+        if (count == 0) count = 1;
+        return cudaMalloc((void **)&p, count * sizeof(T));
+    }
+    cudaError_t upload(const std::vector<T> &v) {
+        cudaError_t e = alloc(v.size());
+        if (e != cudaSuccess || v.empty()) return e;
+        return cudaMemcpy(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+    }
+};
+
+struct Trace {
+    std::vector<triosim_op> ops;
+    std::vector<triosim_tensor> ts;
+    std::vector<uint32_t> io;
+    uint32_t b0 = 0, n_layers = 0;
+    std::vector<int32_t> prod;
+    // trace-level facts the host needs (route needs, cost estimates, partitions)
+    uint32_t n_wgrad = 0;
+    uint64_t wgrad_bytes = 0;
+    uint32_t n_out_total = 0, n_in_total = 0;
+    std::map<int, std::vector<uint32_t>> auto_plans;   // pp -> first layers
+    DevBuf<triosim_op> d_ops;
+    DevBuf<triosim_tensor> d_ts;
+    DevBuf<uint32_t> d_io;
+    DevBuf<double> d_time;
+    DevBuf<uint32_t> d_info, d_layer, d_wgrad;
+    DevBuf<int32_t> d_prod, d_scal;
+    TraceDev dev;
+    int n_sweeps = 0;
+};
+
+struct Sweep {
+    int trace_handle = -1;
+    uint64_t n_pts = 0;
+    std::vector<int32_t> status;            // host-side status per point (-1 = simulate)
+    std::vector<int> width;                 // W per point
+    std::vector<double> cost;
+    std::vector<ClassDesc> classes;
+    std::vector<uint32_t> coll_list, pipe_list;
+    DevBuf<ClassDesc> d_cls;
+    DevBuf<uint32_t> d_coll_list, d_pipe_list;
+    DevBuf<double> d_dur;
+    DevBuf<OpHook> d_hooks;
+    DevBuf<CollEnt> d_colls;
+    DevBuf<int32_t> d_scr_i32;
+    DevBuf<unsigned long long> d_scr_u64;
+    DevBuf<uint32_t> d_plans;
+    DevBuf<StageInfo> d_stages;
+    DevBuf<StageEnt> d_ents;
+    DevBuf<SendEnt> d_sends;
+    DevBuf<RecvEnt> d_recvs;
+    DevBuf<TopoDev> d_topo;
+    DevBuf<double> d_bw, d_lat;
+    DevBuf<uint32_t> d_rt_off, d_ro;
+    DevBuf<uint8_t> d_rt_len;
+    DevBuf<uint16_t> d_rt_links;
+    DevBuf<PointDesc> d_pts;
+    DevBuf<triosim_result> d_res;
+    std::vector<uint32_t> work[6];           // per W index (2,4,8,16,32)
+    DevBuf<uint32_t> d_work[6];
+    DevBuf<uint32_t> d_work_tmp[6];
+    DevBuf<unsigned int> d_counter;
+    DevBuf<unsigned long long> d_alg;
+    cudaStream_t last_stream = nullptr;
+};
+
+int w_index(int W) { return W == 2 ? 0 : W == 4 ? 1 : W == 8 ? 2 : W == 16 ? 3 : 4; }
+const int W_OF[5] = {2, 4, 8, 16, 32};
+
+}  // namespace
+
+struct triosim_ctx {
+    int device = 0;
+    int n_sms = 148;
+    std::string err;
+    std::map<int, std::unique_ptr<Trace>> traces;
+    std::map<int, std::unique_ptr<Sweep>> sweeps;
+    int next_handle = 1;
+    cudaStream_t side[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev_fork = nullptr, ev_join[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint64_t n_k1 = 0, n_k2 = 0, n_k3 = 0;
+    int occ[5] = {0, 0, 0, 0, 0};
+    // optional CUDA-event timing of each simulate_batch (recorded on the caller's stream)
+    static constexpr int NT = 512;
+    bool timing = false;
+    int n_timed = 0;
+    cudaEvent_t t_begin[NT] = {}, t_mid[NT] = {}, t_end[NT] = {};
+};
+
+static triosim_status fail(triosim_ctx *c, triosim_status st, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    return st;
+}
+#define CK(call)                                                                                    \
+    do {                                                                                            \
+        cudaError_t _e = (call);                                                                    \
+        if (_e != cudaSuccess)                                                                      \
+            return fail(ctx, _e == cudaErrorMemoryAllocation ? TRIOSIM_ENOMEM : TRIOSIM_ECUDA,      \
+                        "%s: %s (%s:%d)", #call, cudaGetErrorString(_e), __FILE__, __LINE__);       \
+    } while (0)
+
+extern "C" {
+
+triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
+    if (!out) return TRIOSIM_EINVAL;
+    *out = nullptr;
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || cuda_device < 0 || cuda_device >= n) return TRIOSIM_EUNSUPPORTED;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, cuda_device) != cudaSuccess) return TRIOSIM_ECUDA;
+    if (prop.major != 10 || prop.minor != 0) return TRIOSIM_EUNSUPPORTED;  // built for sm_100a only
+    if (cudaSetDevice(cuda_device) != cudaSuccess) return TRIOSIM_ECUDA;
+    auto *ctx = new (std::nothrow) triosim_ctx();
+    if (!ctx) return TRIOSIM_ENOMEM;
+    ctx->device = cuda_device;
+    ctx->n_sms = prop.multiProcessorCount;
+    for (int i = 0; i < 5; i++) {
+        if (cudaStreamCreateWithFlags(&ctx->side[i], cudaStreamNonBlocking) != cudaSuccess ||
+            cudaEventCreateWithFlags(&ctx->ev_join[i], cudaEventDisableTiming) != cudaSuccess) {
+            triosim_destroy(ctx);
+            return TRIOSIM_ECUDA;
+        }
+        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i]);
+    }
+    if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
+        triosim_destroy(ctx);
+        return TRIOSIM_ECUDA;
+    }
+    *out = ctx;
+    return TRIOSIM_OK;
+}
+
+void triosim_destroy(triosim_ctx *ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->device);
+    cudaDeviceSynchronize();
+    ctx->sweeps.clear();
+    ctx->traces.clear();
+    for (int i = 0; i < 5; i++) {
+        if (ctx->side[i]) cudaStreamDestroy(ctx->side[i]);
+        if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
+    }
+    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
+    for (int i = 0; i < triosim_ctx::NT; i++) {
+        if (ctx->t_begin[i]) cudaEventDestroy(ctx->t_begin[i]);
+        if (ctx->t_mid[i]) cudaEventDestroy(ctx->t_mid[i]);
+        if (ctx->t_end[i]) cudaEventDestroy(ctx->t_end[i]);
+    }
+    delete ctx;
+}
+
+const char *triosim_last_error(const triosim_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    if (k1) *k1 = ctx->n_k1;
+    if (k2) *k2 = ctx->n_k2;
+    if (k3) *k3 = ctx->n_k3;
+    return TRIOSIM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+// load_trace
+// ------------------------------------------------------------------------------------------
+triosim_status triosim_load_trace(triosim_ctx *ctx, const triosim_trace_desc *t, int32_t *trace_id) {
+    if (!ctx || !t || !trace_id) return fail(ctx, TRIOSIM_EINVAL, "null argument");
+    CK(cudaSetDevice(ctx->device));
+    if (t->n_ops == 0 || t->trace_batch == 0 || !t->ops || (t->n_tensors && !t->tensors) || (t->n_io && !t->io))
+        return fail(ctx, TRIOSIM_EINVAL, "empty trace or trace_batch == 0");
+    auto tr = std::make_unique<Trace>();
+    tr->ops.assign(t->ops, t->ops + t->n_ops);
+    tr->ts.assign(t->tensors, t->tensors + t->n_tensors);
+    tr->io.assign(t->io, t->io + t->n_io);
+    tr->b0 = t->trace_batch;
+    tr->prod.assign(t->n_tensors, -1);
+    for (uint32_t x = 0; x < t->n_tensors; x++)
+        if (tr->ts[x].category > TRIOSIM_CAT_OTHER) return fail(ctx, TRIOSIM_EINVAL, "tensor %u: bad category", x);
+    int last_phase = 0;
+    uint32_t next_layer = 0;
+    for (uint32_t o = 0; o < t->n_ops; o++) {
+        const triosim_op &op = tr->ops[o];
+        if (op.phase > 2 || op.phase < last_phase) return fail(ctx, TRIOSIM_EINVAL, "op %u: phases not FWD* BWD* OPT*", o);
+        last_phase = op.phase;
+        if (!(op.time_s >= 0.0) || std::isinf(op.time_s)) return fail(ctx, TRIOSIM_EINVAL, "op %u: bad time", o);
+        if ((uint64_t)op.io_off + op.n_in + op.n_out > t->n_io) return fail(ctx, TRIOSIM_EINVAL, "op %u: io out of range", o);
+        if (op.tp_role > 7) return fail(ctx, TRIOSIM_EINVAL, "op %u: bad tp_role", o);
+        if (op.phase == 0) {
+            if (op.layer == next_layer) next_layer++;
+            else if (op.layer > next_layer) return fail(ctx, TRIOSIM_EINVAL, "op %u: layers not numbered by first FWD use", o);
+        } else if (op.layer >= next_layer) {
+            return fail(ctx, TRIOSIM_EINVAL, "op %u: layer without FWD op", o);
+        }
+        for (uint32_t k = 0; k < op.n_in; k++)
+            if (tr->io[op.io_off + k] >= t->n_tensors) return fail(ctx, TRIOSIM_EINVAL, "op %u: input id out of range", o);
+        for (uint32_t k = 0; k < op.n_out; k++) {
+            uint32_t x = tr->io[op.io_off + op.n_in + k];
+            if (x >= t->n_tensors) return fail(ctx, TRIOSIM_EINVAL, "op %u: output id out of range", o);
+            if (tr->prod[x] != -1) return fail(ctx, TRIOSIM_EINVAL, "tensor %u produced twice", x);
+            tr->prod[x] = (int32_t)o;
+        }
+        tr->n_out_total += op.n_out;
+        tr->n_in_total += op.n_in;
+    }
+    for (uint32_t o = 0; o < t->n_ops; o++) {
+        const triosim_op &op = tr->ops[o];
+        for (uint32_t k = 0; k < op.n_in; k++)
+            if (tr->prod[tr->io[op.io_off + k]] >= (int32_t)o) return fail(ctx, TRIOSIM_EINVAL, "op %u reads a tensor before it is produced", o);
+    }
+    tr->n_layers = next_layer;
+    if (tr->n_layers == 0) return fail(ctx, TRIOSIM_EINVAL, "no FWD op");
+    for (uint32_t x = 0; x < t->n_tensors; x++)
+        if (tr->ts[x].category == TRIOSIM_CAT_WGRAD && tr->prod[x] >= 0 && tr->ops[tr->prod[x]].phase != 2) {
+            tr->n_wgrad++;
+            tr->wgrad_bytes += tr->ts[x].bytes_b0;
+        }
+    // stage to the device and run the ingest kernel
+    CK(tr->d_ops.upload(tr->ops));
+    CK(tr->d_ts.upload(tr->ts));
+    CK(tr->d_io.upload(tr->io));
+    CK(tr->d_time.alloc(t->n_ops));
+    CK(tr->d_info.alloc(t->n_ops));
+    CK(tr->d_layer.alloc(t->n_ops));
+    CK(tr->d_wgrad.alloc(std::max<uint32_t>(tr->n_wgrad, 1)));
+    CK(tr->d_prod.alloc(std::max<uint32_t>(t->n_tensors, 1)));
+    CK(tr->d_scal.alloc(4));
+    CK(cudaMemset(tr->d_prod.p, 0xff, sizeof(int32_t) * std::max<uint32_t>(t->n_tensors, 1)));
+    int32_t scal0[4] = {0, INT32_MAX, -1, 0};
+    CK(cudaMemcpy(tr->d_scal.p, scal0, sizeof scal0, cudaMemcpyHostToDevice));
+    TraceDev &D = tr->dev;
+    D.ops = tr->d_ops.p; D.ts = tr->d_ts.p; D.io = tr->d_io.p;
+    D.time = tr->d_time.p; D.info = tr->d_info.p; D.layer = tr->d_layer.p; D.prod = tr->d_prod.p;
+    D.wgrad = tr->d_wgrad.p; D.scal = tr->d_scal.p;
+    D.n_ops = t->n_ops; D.n_ts = t->n_tensors; D.n_io = t->n_io; D.b0 = t->trace_batch; D.n_layers = tr->n_layers;
+    D.pad = 0;
+    CK(launch_k1_ingest(D, 0));
+    ctx->n_k1++;
+    CK(cudaDeviceSynchronize());
+    int h = ctx->next_handle++;
+    ctx->traces[h] = std::move(tr);
+    *trace_id = h;
+    return TRIOSIM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+// host helpers: routing (BFS, ascending neighbours, first discovery) and the PP partition
+// ------------------------------------------------------------------------------------------
+static std::vector<uint32_t> auto_partition(const Trace &T, int S) {
+    const int L = (int)T.n_layers;
+    std::vector<double> lc(L, 0.0);
+    for (const auto &op : T.ops) lc[op.layer] = lc[op.layer] + op.time_s;
+    std::vector<double> cost((size_t)L * L, 0.0);
+    for (int a = 0; a < L; a++) {
+        double s = 0.0;
+        for (int b = a; b < L; b++) { s = s + lc[b]; cost[(size_t)a * L + b] = s; }
+    }
+    std::vector<double> best((size_t)(S + 1) * (L + 1), INFINITY);
+    auto B = [&](int s, int i) -> double & { return best[(size_t)s * (L + 1) + i]; };
+    for (int i = 0; i < L; i++) B(1, i) = cost[(size_t)i * L + L - 1];
+    for (int s = 2; s <= S; s++)
+        for (int i = 0; i + s <= L; i++) {
+            double b = INFINITY;
+            for (int j = i + 1; L - j >= s - 1; j++) {
+                double a = cost[(size_t)i * L + j - 1], r = B(s - 1, j);
+                double mx = a > r ? a : r;
+                if (mx < b) b = mx;
+            }
+            B(s, i) = b;
+        }
+    const double V = B(S, 0);
+    std::vector<uint32_t> fl(S, 0);
+    int i = 0;
+    for (int s = S; s >= 2; s--) {
+        int jj = -1;
+        for (int j = i + 1; L - j >= s - 1; j++)
+            if (cost[(size_t)i * L + j - 1] <= V && B(s - 1, j) <= V) { jj = j; break; }
+        fl[S - s + 1] = (uint32_t)jj;
+        i = jj;
+    }
+    return fl;
+}
+
+struct HostTopo {
+    uint32_t n_nodes, n_gpus, n_links, max_hops;
+    std::vector<uint32_t> ro;
+    std::vector<uint32_t> rt_off;   // n_gpus^2
+    std::vector<uint8_t> rt_len;
+    std::vector<uint16_t> links;    // route pool (local)
+};
+
+static triosim_status prep_topology(triosim_ctx *ctx, const triosim_topology &tp, uint32_t idx, HostTopo &H) {
+    if (tp.n_gpus == 0 || tp.n_gpus > tp.n_nodes || (tp.n_links && !tp.links))
+        return fail(ctx, TRIOSIM_EINVAL, "topology %u: bad sizes", idx);
+    H.n_nodes = tp.n_nodes; H.n_gpus = tp.n_gpus; H.n_links = tp.n_links; H.max_hops = 0;
+    std::vector<std::vector<std::pair<uint32_t, uint32_t>>> adj(tp.n_nodes);
+    std::vector<std::vector<uint32_t>> seen(tp.n_nodes);
+    for (uint32_t e = 0; e < tp.n_links; e++) {
+        const triosim_link &l = tp.links[e];
+        if (l.src >= tp.n_nodes || l.dst >= tp.n_nodes || l.src == l.dst)
+            return fail(ctx, TRIOSIM_EINVAL, "topology %u link %u: bad endpoints", idx, e);
+        if (!(l.bw_Bps > 0.0) || std::isinf(l.bw_Bps) || !(l.lat_s >= 0.0) || std::isinf(l.lat_s))
+            return fail(ctx, TRIOSIM_EINVAL, "topology %u link %u: bw must be > 0, lat >= 0", idx, e);
+        for (uint32_t d : seen[l.src])
+            if (d == l.dst) return fail(ctx, TRIOSIM_EINVAL, "topology %u: duplicate link %u->%u", idx, l.src, l.dst);
+        seen[l.src].push_back(l.dst);
+        adj[l.src].push_back({l.dst, e});
+    }
+    for (auto &v : adj) std::sort(v.begin(), v.end());
+    H.ro.resize(tp.n_gpus);
+    std::vector<char> used(tp.n_gpus, 0);
+    for (uint32_t i = 0; i < tp.n_gpus; i++) {
+        uint32_t g = tp.ring_order ? tp.ring_order[i] : i;
+        if (g >= tp.n_gpus || used[g]) return fail(ctx, TRIOSIM_EINVAL, "topology %u: ring_order not a permutation", idx);
+        used[g] = 1;
+        H.ro[i] = g;
+    }
+    const uint32_t G = tp.n_gpus;
+    H.rt_off.assign((size_t)G * G, 0);
+    H.rt_len.assign((size_t)G * G, NO_ROUTE);
+    std::vector<int32_t> par(tp.n_nodes);
+    std::vector<uint32_t> q(tp.n_nodes);
+    for (uint32_t s = 0; s < G; s++) {
+        std::fill(par.begin(), par.end(), -2);
+        par[s] = -1;
+        uint32_t qh = 0, qt = 0;
+        q[qt++] = s;
+        while (qh < qt) {
+            uint32_t u = q[qh++];
+            for (auto &pe : adj[u])
+                if (par[pe.first] == -2) { par[pe.first] = (int32_t)pe.second; q[qt++] = pe.first; }
+        }
+        for (uint32_t d = 0; d < G; d++) {
+            size_t k = (size_t)s * G + d;
+            if (d == s) { H.rt_len[k] = 0; H.rt_off[k] = 0; continue; }
+            if (par[d] == -2) continue;
+            std::vector<uint16_t> path;
+            for (uint32_t v = d; v != s; v = tp.links[par[v]].src) path.push_back((uint16_t)par[v]);
+            std::reverse(path.begin(), path.end());
+            if (path.size() > 250) continue;
+            H.rt_off[k] = (uint32_t)H.links.size();
+            H.rt_len[k] = (uint8_t)path.size();
+            H.max_hops = std::max<uint32_t>(H.max_hops, (uint32_t)path.size());
+            H.links.insert(H.links.end(), path.begin(), path.end());
+        }
+    }
+    return TRIOSIM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+// build_sweep
+// ------------------------------------------------------------------------------------------
+triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const triosim_topology *topos, uint32_t n_topos,
+                                   const triosim_stage_plans *plans, const triosim_point *pts, uint64_t n_pts,
+                                   int32_t *sweep_id) {
+    if (!ctx || !sweep_id || (n_topos && !topos) || (n_pts && !pts)) return fail(ctx, TRIOSIM_EINVAL, "null argument");
+    CK(cudaSetDevice(ctx->device));
+    auto it = ctx->traces.find(trace_id);
+    if (it == ctx->traces.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown trace %d", trace_id);
+    Trace &T = *it->second;
+    if (n_pts > (1ull << 31)) return fail(ctx, TRIOSIM_EINVAL, "too many points");
+    if (plans && plans->n_plans && (!plans->off || !plans->first_layer)) return fail(ctx, TRIOSIM_EINVAL, "bad plans");
+    if (plans && plans->n_plans && plans->off[0] != 0) return fail(ctx, TRIOSIM_EINVAL, "bad plans");
+    if (plans)
+        for (uint32_t k = 0; k < plans->n_plans; k++)
+            if (plans->off[k + 1] < plans->off[k]) return fail(ctx, TRIOSIM_EINVAL, "bad plan offsets");
+
+    std::vector<HostTopo> HT(n_topos);
+    for (uint32_t i = 0; i < n_topos; i++) {
+        triosim_status st = prep_topology(ctx, topos[i], i, HT[i]);
+        if (st != TRIOSIM_OK) return st;
+    }
+    auto S = std::make_unique<Sweep>();
+    S->trace_handle = trace_id;
+    S->n_pts = n_pts;
+    S->status.assign(n_pts, -1);
+    S->width.assign(n_pts, 0);
+    S->cost.assign(n_pts, 0.0);
+    std::vector<PointDesc> pdesc(n_pts);
+    std::map<std::tuple<int, int, int, int, int, uint64_t, int, int>, uint32_t> cls_of;
+    std::vector<uint32_t> plan_pool;
+    const uint32_t N = (uint32_t)T.ops.size(), NT = (uint32_t)T.ts.size();
+
+    // trace-level counts used for cost estimates
+    uint32_t n_tp_coll[2] = {0, 0};
+    for (const auto &op : T.ops) {
+        for (uint32_t k = 0; k < op.n_out; k++) {
+            uint8_t cat = T.ts[T.io[op.io_off + op.n_in + k]].category;
+            if ((op.tp_role & 4) && (op.phase == 0 || (op.phase == 1 && cat == TRIOSIM_CAT_AGRAD))) n_tp_coll[0]++;
+            if (((op.tp_role & 3) == 2 && op.phase == 0) || ((op.tp_role & 3) == 1 && op.phase == 1 && cat == TRIOSIM_CAT_AGRAD))
+                n_tp_coll[1]++;
+        }
+    }
+
+    for (uint64_t i = 0; i < n_pts; i++) {
+        const triosim_point &pt = pts[i];
+        auto setst = [&](int st) { S->status[i] = st; };
+        // R3, in order
+        if (pt.topo >= n_topos) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 1) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        if (!(pt.bw_scale > 0.0) || std::isinf(pt.bw_scale) || !(pt.lat_scale >= 0.0) || std::isinf(pt.lat_scale)) {
+            setst(TRIOSIM_PT_BAD_CONFIG);
+            continue;
+        }
+        const HostTopo &tp = HT[pt.topo];
+        const uint32_t dp = pt.dp, tpd = pt.tp, pp = pt.pp, mb = pt.microbatches;
+        bool bad = dp == 0 || tpd == 0 || pp == 0;
+        if (!bad) {
+            if ((pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP) && (tpd != 1 || pp != 1)) bad = true;
+            if (pt.strategy == TRIOSIM_TP && (dp != 1 || pp != 1)) bad = true;
+            if (pt.strategy == TRIOSIM_PP && (dp != 1 || tpd != 1)) bad = true;
+        }
+        const bool piped = pt.strategy == TRIOSIM_PP || pt.strategy == TRIOSIM_HYBRID;
+        if (!bad && piped && mb == 0) bad = true;
+        if (!bad && (uint64_t)dp * tpd * pp > tp.n_gpus) bad = true;
+        if (!bad && (pp > T.n_layers || pp > 64)) bad = true;
+        if (bad) { setst(TRIOSIM_PT_BAD_DEGREES); continue; }
+        const uint64_t mm = piped ? mb : 1;
+        if (pt.global_batch == 0 || pt.global_batch % ((uint64_t)dp * mm) != 0) { setst(TRIOSIM_PT_BAD_BATCH); continue; }
+        std::vector<uint32_t> plan;
+        int plan_key = -1;
+        if (piped && pt.stage_plan >= 0) {
+            if (!plans || (uint32_t)pt.stage_plan >= plans->n_plans) { setst(TRIOSIM_PT_BAD_PLAN); continue; }
+            uint32_t a0 = plans->off[pt.stage_plan], a1 = plans->off[pt.stage_plan + 1];
+            plan.assign(plans->first_layer + a0, plans->first_layer + a1);
+            bool ok = plan.size() == pp && plan[0] == 0;
+            for (size_t s = 1; ok && s < plan.size(); s++) ok = plan[s] > plan[s - 1] && plan[s] < T.n_layers;
+            if (!ok) { setst(TRIOSIM_PT_BAD_PLAN); continue; }
+            plan_key = pt.stage_plan;
+        }
+        if (pt.strategy == TRIOSIM_HYBRID) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        // GPU kernel limits
+        const uint32_t lanes = pt.strategy == TRIOSIM_TP ? tpd : pt.strategy == TRIOSIM_PP ? pp : dp;
+        int W = 2;
+        while (W < (int)lanes) W <<= 1;
+        while (W <= 32 && (int)tp.n_links > std::max(8, 4 * W)) W <<= 1;
+        if (W > 32) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
+        // structural class
+        const int mode = pt.strategy == TRIOSIM_PP ? MODE_PIPE : MODE_COLL;
+        uint32_t b_loc = pt.strategy == TRIOSIM_TP ? pt.global_batch
+                       : pt.strategy == TRIOSIM_PP ? pt.global_batch / mb : pt.global_batch / dp;
+        int key_mode = pt.strategy == TRIOSIM_TP ? pt.tp_mode : 0;
+        int key_algo = mode == MODE_COLL ? pt.coll_algo : 0;
+        uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP) ? pt.bucket_bytes : 0;
+        int key_m = mode == MODE_PIPE ? (int)mb : 0;
+        auto key = std::make_tuple((int)pt.strategy, (int)lanes, (int)b_loc, key_mode, key_algo, key_bucket, key_m,
+                                   mode == MODE_PIPE ? plan_key : -2);
+        auto ci = cls_of.find(key);
+        uint32_t c;
+        if (ci == cls_of.end()) {
+            ClassDesc cd;
+            std::memset(&cd, 0, sizeof cd);
+            cd.mode = mode;
+            cd.strategy = pt.strategy;
+            cd.tp_mode = key_mode;
+            cd.algo = key_algo;
+            cd.p = lanes;
+            cd.m = mode == MODE_PIPE ? mb : 1;
+            cd.tpdeg = pt.strategy == TRIOSIM_TP ? tpd : 1;
+            cd.b_loc = b_loc;
+            cd.bucket_bytes = key_bucket;
+            cd.r_b = (double)b_loc / (double)T.b0;
+            if (mode == MODE_PIPE) {
+                if (plan_key < 0) {
+                    auto ap = T.auto_plans.find((int)pp);
+                    if (ap == T.auto_plans.end()) ap = T.auto_plans.emplace((int)pp, auto_partition(T, (int)pp)).first;
+                    plan = ap->second;
+                }
+                cd.plan_off = (uint32_t)plan_pool.size();
+                plan_pool.insert(plan_pool.end(), plan.begin(), plan.end());
+            }
+            c = (uint32_t)S->classes.size();
+            S->classes.push_back(cd);
+            cls_of[key] = c;
+        } else {
+            c = ci->second;
+        }
+        PointDesc &pd = pdesc[i];
+        pd.bw_scale = pt.bw_scale;
+        pd.lat_scale = pt.lat_scale;
+        pd.cls = c;
+        pd.topo = pt.topo;
+        pd.idx = (uint32_t)i;
+        pd.pad = 0;
+        S->width[i] = W;
+        double cost;
+        if (mode == MODE_COLL) {
+            double ncol = pt.strategy == TRIOSIM_TP ? n_tp_coll[pt.tp_mode == TRIOSIM_TP_PAPER ? 0 : 1]
+                        : (key_bucket == 0 ? T.n_wgrad : std::ceil((double)T.wgrad_bytes / (double)key_bucket));
+            cost = (double)N * 2 + ncol * 2.0 * lanes * 8.0;
+        } else {
+            cost = (double)mb * N * 2.0 / lanes + (double)mb * 2.0 * 8.0 * lanes;
+        }
+        S->cost[i] = cost;
+    }
+
+    // per-class pools
+    uint32_t dur_n = 0, hook_n = 0, coll_n = 0, scr_i = 0, scr_u = 0, stage_n = 0, ent_n = 0, send_n = 0, recv_n = 0;
+    for (uint32_t c = 0; c < S->classes.size(); c++) {
+        ClassDesc &cd = S->classes[c];
+        cd.dur_off = dur_n; dur_n += N;
+        if (cd.mode == MODE_COLL) {
+            S->coll_list.push_back(c);
+            cd.hook_off = hook_n; hook_n += N;
+            cd.coll_cap = (cd.strategy == TRIOSIM_TP) ? T.n_out_total : T.n_wgrad;
+            cd.coll_off = coll_n; coll_n += cd.coll_cap;
+            if (cd.strategy == TRIOSIM_TP) { cd.scratch_off = scr_i; scr_i += NT; }
+        } else {
+            S->pipe_list.push_back(c);
+            cd.stage_off = stage_n; stage_n += cd.p;
+            cd.ent_off = ent_n; cd.ent_cap = N; ent_n += N;
+            cd.send_cap = T.n_out_total * (cd.p > 1 ? cd.p - 1 : 1);
+            cd.send_off = send_n; send_n += cd.send_cap;
+            cd.recv_cap = T.n_in_total;
+            cd.recv_off = recv_n; recv_n += cd.recv_cap;
+            cd.scratch_off = scr_u; scr_u += NT;
+        }
+    }
+    // topologies to the device
+    std::vector<TopoDev> td(n_topos);
+    std::vector<double> bw, lat;
+    std::vector<uint32_t> rt_off, ro;
+    std::vector<uint8_t> rt_len;
+    std::vector<uint16_t> rt_links;
+    for (uint32_t i = 0; i < n_topos; i++) {
+        TopoDev &d = td[i];
+        d.n_nodes = HT[i].n_nodes; d.n_gpus = HT[i].n_gpus; d.n_links = HT[i].n_links;
+        d.link_off = (uint32_t)bw.size();
+        for (uint32_t e = 0; e < topos[i].n_links; e++) { bw.push_back(topos[i].links[e].bw_Bps); lat.push_back(topos[i].links[e].lat_s); }
+        d.rt_off = (uint32_t)rt_off.size();
+        uint32_t base = (uint32_t)rt_links.size();
+        for (size_t k = 0; k < HT[i].rt_off.size(); k++) { rt_off.push_back(HT[i].rt_off[k] + base); rt_len.push_back(HT[i].rt_len[k]); }
+        rt_links.insert(rt_links.end(), HT[i].links.begin(), HT[i].links.end());
+        d.ro_off = (uint32_t)ro.size();
+        ro.insert(ro.end(), HT[i].ro.begin(), HT[i].ro.end());
+        d.max_hops = HT[i].max_hops;
+        d.pad = 0;
+    }
+    CK(S->d_topo.upload(td));
+    CK(S->d_bw.upload(bw));
+    CK(S->d_lat.upload(lat));
+    CK(S->d_rt_off.upload(rt_off));
+    CK(S->d_rt_len.upload(rt_len));
+    CK(S->d_rt_links.upload(rt_links));
+    CK(S->d_ro.upload(ro));
+    CK(S->d_cls.upload(S->classes));
+    CK(S->d_coll_list.upload(S->coll_list));
+    CK(S->d_pipe_list.upload(S->pipe_list));
+    CK(S->d_dur.alloc(dur_n));
+    CK(S->d_hooks.alloc(hook_n));
+    CK(S->d_colls.alloc(coll_n));
+    CK(S->d_scr_i32.alloc(scr_i));
+    CK(S->d_scr_u64.alloc(scr_u));
+    CK(S->d_plans.upload(plan_pool));
+    CK(S->d_stages.alloc(stage_n));
+    CK(S->d_ents.alloc(ent_n));
+    CK(S->d_sends.alloc(send_n));
+    CK(S->d_recvs.alloc(recv_n));
+    CK(S->d_pts.upload(pdesc));
+    // result records: host-decided statuses now, simulated points overwritten by K3
+    std::vector<triosim_result> res0(n_pts);
+    std::memset(res0.data(), 0, sizeof(triosim_result) * n_pts);
+    for (uint64_t i = 0; i < n_pts; i++) res0[i].status = S->status[i] < 0 ? TRIOSIM_PT_OK : S->status[i];
+    CK(S->d_res.upload(res0));
+    // work lists per width, most expensive first (LPT)
+    std::vector<uint64_t> order;
+    for (uint64_t i = 0; i < n_pts; i++) if (S->status[i] < 0) order.push_back(i);
+    std::stable_sort(order.begin(), order.end(), [&](uint64_t a, uint64_t b) {
+        if (S->cost[a] != S->cost[b]) return S->cost[a] > S->cost[b];
+        return pdesc[a].cls < pdesc[b].cls;
+    });
+    for (uint64_t i : order) S->work[w_index(S->width[i])].push_back((uint32_t)i);
+    for (int w = 0; w < 5; w++) {
+        CK(S->d_work[w].upload(S->work[w]));
+        CK(S->d_work_tmp[w].alloc(S->work[w].size()));
+    }
+    CK(S->d_counter.alloc(5));
+    CK(S->d_alg.alloc(1));
+    CK(cudaMemset(S->d_alg.p, 0, sizeof(unsigned long long)));
+    CK(cudaDeviceSynchronize());
+    int h = ctx->next_handle++;
+    T.n_sweeps++;
+    ctx->sweeps[h] = std::move(S);
+    *sweep_id = h;
+    return TRIOSIM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+// simulate_batch
+// ------------------------------------------------------------------------------------------
+triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
+                                      void *cuda_stream) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    CK(cudaSetDevice(ctx->device));
+    CK(cudaGetLastError());  // report sticky errors from earlier asynchronous work
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    if (first > S.n_pts || count > S.n_pts - first) return fail(ctx, TRIOSIM_ERANGE, "range [%llu,+%llu) outside sweep of %llu",
+                                                              (unsigned long long)first, (unsigned long long)count,
+                                                              (unsigned long long)S.n_pts);
+    Trace &T = *ctx->traces.at(S.trace_handle);
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    S.last_stream = st;
+    const uint32_t ncls = (uint32_t)S.classes.size();
+    const int slot = ctx->timing ? ctx->n_timed % triosim_ctx::NT : -1;
+    if (slot >= 0) CK(cudaEventRecord(ctx->t_begin[slot], st));
+    // K1b + K2 for every class of the sweep (cheap; part of every step)
+    CK(launch_k1_rescale(S.d_cls.p, ncls, T.dev, S.d_dur.p, st));
+    if (ncls) ctx->n_k1++;
+    CK(launch_k2_coll(S.d_cls.p, S.d_coll_list.p, (uint32_t)S.coll_list.size(), T.dev, S.d_dur.p, S.d_hooks.p,
+                      S.d_colls.p, S.d_scr_i32.p, st));
+    if (!S.coll_list.empty()) ctx->n_k2++;
+    CK(launch_k2_pipe(S.d_cls.p, S.d_pipe_list.p, (uint32_t)S.pipe_list.size(), T.dev, S.d_dur.p, S.d_plans.p,
+                      S.d_stages.p, S.d_ents.p, S.d_sends.p, S.d_recvs.p, S.d_scr_u64.p, st));
+    if (!S.pipe_list.empty()) ctx->n_k2++;
+    // K3 per segment width, forked onto side streams so the widths run concurrently
+    const bool full = first == 0 && count == S.n_pts;
+    CK(cudaMemsetAsync(S.d_counter.p, 0, 5 * sizeof(unsigned int), st));
+    CK(cudaMemsetAsync(S.d_alg.p, 0, sizeof(unsigned long long), st));
+    if (slot >= 0) CK(cudaEventRecord(ctx->t_mid[slot], st));
+    CK(cudaEventRecord(ctx->ev_fork, st));
+    int launched[5] = {0, 0, 0, 0, 0};
+    for (int w = 0; w < 5; w++) {
+        const uint32_t *wl = S.d_work[w].p;
+        uint32_t n = (uint32_t)S.work[w].size();
+        if (!full) {
+            std::vector<uint32_t> sub;
+            for (uint32_t i : S.work[w]) if (i >= first && i < first + count) sub.push_back(i);
+            n = (uint32_t)sub.size();
+            if (n) CK(cudaMemcpyAsync(S.d_work_tmp[w].p, sub.data(), n * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+            CK(cudaStreamSynchronize(st));  // sub is a host temporary
+            wl = S.d_work_tmp[w].p;
+        }
+        if (n == 0) continue;
+        const int W = W_OF[w];
+        K3Args a;
+        std::memset(&a, 0, sizeof a);
+        a.pts = S.d_pts.p; a.work = wl; a.n_work = n; a.counter = S.d_counter.p + w;
+        a.cls = S.d_cls.p; a.topo = S.d_topo.p;
+        a.link_bw = S.d_bw.p; a.link_lat = S.d_lat.p; a.rt_off = S.d_rt_off.p; a.rt_len = S.d_rt_len.p;
+        a.rt_links = S.d_rt_links.p; a.ro = S.d_ro.p;
+        a.hooks = S.d_hooks.p; a.colls = S.d_colls.p; a.dur = S.d_dur.p;
+        a.stages = S.d_stages.p; a.ents = S.d_ents.p; a.sends = S.d_sends.p; a.recvs = S.d_recvs.p;
+        a.out = S.d_res.p;
+        a.alg_ops = S.d_alg.p;
+        const int nseg = 32 / W;
+        const uint64_t warps = (n + nseg - 1) / nseg;
+        uint64_t blocks = (warps + K3_WARPS - 1) / K3_WARPS;
+        const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)ctx->occ[w];
+        if (blocks > cap) blocks = cap;
+        CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
+        CK(launch_k3(W, a, (int)blocks, ctx->side[w]));
+        ctx->n_k3++;
+        CK(cudaEventRecord(ctx->ev_join[w], ctx->side[w]));
+        launched[w] = 1;
+    }
+    for (int w = 0; w < 5; w++)
+        if (launched[w]) CK(cudaStreamWaitEvent(st, ctx->ev_join[w], 0));
+    if (slot >= 0) {
+        CK(cudaEventRecord(ctx->t_end[slot], st));
+        ctx->n_timed++;
+    }
+    return TRIOSIM_OK;
+}
+
+triosim_status triosim_timing(triosim_ctx *ctx, int enable) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    CK(cudaSetDevice(ctx->device));
+    if (enable && !ctx->t_begin[0])
+        for (int i = 0; i < triosim_ctx::NT; i++) {
+            CK(cudaEventCreate(&ctx->t_begin[i]));
+            CK(cudaEventCreate(&ctx->t_mid[i]));
+            CK(cudaEventCreate(&ctx->t_end[i]));
+        }
+    ctx->timing = enable != 0;
+    ctx->n_timed = 0;
+    return TRIOSIM_OK;
+}
+
+int32_t triosim_timings(triosim_ctx *ctx, float *ms_total, float *ms_k3, int32_t max) {
+    if (!ctx || !ctx->timing) return TRIOSIM_EINVAL;
+    int n = ctx->n_timed < triosim_ctx::NT ? ctx->n_timed : triosim_ctx::NT;
+    if (n > max) n = max;
+    for (int i = 0; i < n; i++) {
+        if (cudaEventSynchronize(ctx->t_end[i]) != cudaSuccess) return TRIOSIM_ECUDA;
+        if (ms_total && cudaEventElapsedTime(&ms_total[i], ctx->t_begin[i], ctx->t_end[i]) != cudaSuccess) return TRIOSIM_ECUDA;
+        if (ms_k3 && cudaEventElapsedTime(&ms_k3[i], ctx->t_mid[i], ctx->t_end[i]) != cudaSuccess) return TRIOSIM_ECUDA;
+    }
+    return n;
+}
+
+triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count, triosim_result *out,
+                               int out_is_device, void *cuda_stream) {
+    if (!ctx || (count && !out)) return fail(ctx, TRIOSIM_EINVAL, "null argument");
+    CK(cudaSetDevice(ctx->device));
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    if (first > S.n_pts || count > S.n_pts - first) return fail(ctx, TRIOSIM_ERANGE, "range outside sweep");
+    if (count == 0) return TRIOSIM_OK;
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    if (out_is_device) {
+        CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToDevice, st));
+    } else {
+        CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+    }
+    return TRIOSIM_OK;
+}
+
+triosim_status triosim_work_counters(triosim_ctx *ctx, int32_t sweep_id, uint64_t *fp64_ops) {
+    if (!ctx || !fp64_ops) return fail(ctx, TRIOSIM_EINVAL, "null argument");
+    CK(cudaSetDevice(ctx->device));
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    unsigned long long v = 0;
+    CK(cudaMemcpyAsync(&v, S.d_alg.p, sizeof v, cudaMemcpyDeviceToHost, S.last_stream));
+    CK(cudaStreamSynchronize(S.last_stream));
+    *fp64_ops = v;
+    return TRIOSIM_OK;
+}
+
+const void *triosim_results_device_ptr(const triosim_ctx *ctx, int32_t sweep_id) {
+    if (!ctx) return nullptr;
+    auto it = ctx->sweeps.find(sweep_id);
+    return it == ctx->sweeps.end() ? nullptr : (const void *)it->second->d_res.p;
+}
+
+triosim_status triosim_release(triosim_ctx *ctx, int32_t handle) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    cudaSetDevice(ctx->device);
+    auto s = ctx->sweeps.find(handle);
+    if (s != ctx->sweeps.end()) {
+        cudaDeviceSynchronize();
+        auto t = ctx->traces.find(s->second->trace_handle);
+        if (t != ctx->traces.end()) t->second->n_sweeps--;
+        ctx->sweeps.erase(s);
+        return TRIOSIM_OK;
+    }
+    auto t = ctx->traces.find(handle);
+    if (t != ctx->traces.end()) {
+        if (t->second->n_sweeps > 0) return fail(ctx, TRIOSIM_EINVAL, "trace %d still used by a sweep", handle);
+        cudaDeviceSynchronize();
+        ctx->traces.erase(t);
+        return TRIOSIM_OK;
+    }
+    return fail(ctx, TRIOSIM_ENOTFOUND, "unknown handle %d", handle);
+}
+
+}  // extern "C"

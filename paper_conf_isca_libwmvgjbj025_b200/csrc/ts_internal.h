@@ -1,0 +1,139 @@
+// ts_internal.h -- device-side data layout of libtriosim.
+// Shared only by ts_host.cu and ts_kernels.cu (product path).  Nothing here is shared
+// with oracle/.
+#pragma once
+#include <cstdint>
+#include "triosim.h"
+
+namespace ts {
+
+enum { MODE_COLL = 0, MODE_PIPE = 1 };
+enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
+enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
+constexpr int MAX_HOPS = 8;
+constexpr uint8_t NO_ROUTE = 0xFF;
+constexpr int K3_THREADS = 256;
+constexpr int K3_WARPS = K3_THREADS / 32;
+
+// per-op packed info written by the ingest kernel
+constexpr uint32_t INFO_PHASE_MASK = 3u;
+constexpr uint32_t INFO_ROLE_SHIFT = 2;   // 3 bits of tp_role
+constexpr uint32_t INFO_SCALED = 1u << 5;
+
+struct TraceDev {
+    // raw staged records
+    const triosim_op *ops;
+    const triosim_tensor *ts;
+    const uint32_t *io;
+    // SoA produced by K1a (ingest)
+    double *time;       // n_ops
+    uint32_t *info;     // n_ops: phase | role << 2 | scaled << 5
+    uint32_t *layer;    // n_ops
+    int32_t *prod;      // n_ts: producing op or -1
+    uint32_t *wgrad;    // weight gradients in production order (non-OPT producers)
+    int32_t *scal;      // [0] n_wgrad, [1] first OPT op (INT_MAX = none), [2] last non-OPT op (-1 = none)
+    uint32_t n_ops, n_ts, n_io, b0, n_layers, pad;
+};
+
+// COLL mode (DP / DDP / TP): one entry per operator of a class
+struct OpHook {
+    double dur;       // t' (K1b)
+    int32_t wait;     // collective index that must be done on this GPU before the op starts, or -1
+    uint32_t nsig;    // number of collectives triggered by this op's completion
+};
+struct CollEnt {
+    double S;         // payload bytes
+    uint32_t kind;    // CK_*
+    uint32_t pad;
+};
+
+// PIPE mode (GPipe): per stage of a class
+struct StageInfo {
+    uint32_t nF, nB, nO;      // ops of the stage per phase
+    uint32_t SF, SB, SO;      // P2P sends per micro-batch (F, B) and once (O)
+    uint32_t ent_off;         // StageEnt list: [F nF][B nB][O nO]
+    uint32_t send_off;        // SendEnt list: [F SF][B SB][O SO]
+    uint32_t recv_off;        // RecvEnt pool base of this stage
+    uint32_t pad;
+    uint64_t dst_mask;        // stages this stage sends to (route check)
+};
+struct StageEnt {
+    uint32_t op;
+    uint16_t nsend, nrecv;
+    uint32_t recv_off;
+    uint32_t pad;
+};
+struct SendEnt {
+    double bytes;
+    uint32_t x;
+    uint16_t dst;    // destination stage
+    uint16_t pidx;   // producer index inside its phase list
+};
+struct RecvEnt {
+    uint16_t src;    // producing stage
+    uint8_t phase;   // producer phase
+    uint8_t pad;
+    uint32_t e;      // index in the producer stage's send list of that phase
+};
+
+struct ClassDesc {
+    // set by the host
+    uint32_t mode, strategy, tp_mode, algo;
+    uint32_t p, m, tpdeg, b_loc;
+    uint64_t bucket_bytes;
+    double r_b;
+    uint32_t dur_off, hook_off, coll_off, coll_cap;
+    uint32_t plan_off, stage_off, ent_off, ent_cap;
+    uint32_t send_off, send_cap, recv_off, recv_cap;
+    uint32_t scratch_off, pad0;
+    // written by K2
+    uint32_t n_coll, need_ring, need_tree, n_prog_max;
+    double coll_payload;
+    uint64_t n_compute, n_flows;
+};
+
+struct TopoDev {
+    uint32_t n_nodes, n_gpus, n_links, link_off;
+    uint32_t rt_off, ro_off, max_hops, pad;
+};
+
+struct PointDesc {
+    double bw_scale, lat_scale;
+    uint32_t cls, topo, idx, pad;
+};
+
+struct K3Args {
+    const PointDesc *pts;
+    const uint32_t *work;
+    uint32_t n_work, pad;
+    unsigned int *counter;
+    const ClassDesc *cls;
+    const TopoDev *topo;
+    const double *link_bw, *link_lat;
+    const uint32_t *rt_off;
+    const uint8_t *rt_len;
+    const uint16_t *rt_links;
+    const uint32_t *ro;
+    const OpHook *hooks;
+    const CollEnt *colls;
+    const double *dur;
+    const StageInfo *stages;
+    const StageEnt *ents;
+    const SendEnt *sends;
+    const RecvEnt *recvs;
+    triosim_result *out;
+    unsigned long long *alg_ops;   // method fp64 operations performed
+};
+
+// launchers (ts_kernels.cu)
+cudaError_t launch_k1_ingest(const TraceDev &T, cudaStream_t s);
+cudaError_t launch_k1_rescale(const ClassDesc *cls, uint32_t n_cls, const TraceDev &T, double *dur, cudaStream_t s);
+cudaError_t launch_k2_coll(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T, const double *dur,
+                           OpHook *hooks, CollEnt *colls, int32_t *scratch_i32, cudaStream_t s);
+cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T, const double *dur,
+                           const uint32_t *plan_pool, StageInfo *stages, StageEnt *ents, SendEnt *sends,
+                           RecvEnt *recvs, unsigned long long *scratch_u64, cudaStream_t s);
+cudaError_t launch_k3(int W, const K3Args &a, int grid, cudaStream_t s);
+int k3_max_blocks_per_sm(int W);
+
+}  // namespace ts

@@ -1,0 +1,193 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Small seeded cases are compared in full; the BASELINE.json configs are run at full size in
+the launch configuration bench.py times and compared on seeded samples the oracle computes
+one by one, plus properties that must hold for every point.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_isca_libwmvgjbj025_b200 import workloads as W
+from tests.parity import compare
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_isca_libwmvgjbj025_b200 import triosim
+    c = triosim.Context(0)
+    yield c
+    c.close()
+
+
+def sample(n, k, seed):
+    rng = np.random.Generator(np.random.PCG64(seed))
+    return sorted(rng.choice(n, size=min(k, n), replace=False).tolist())
+
+
+def check(got, sw, idx, allow_too_large=False):
+    ref = oracle.run_sweep(sw, idx)
+    bad, ulp = compare(got[idx], ref, idx, allow_too_large)
+    assert not bad, "\n".join(bad[:20])
+    return ulp
+
+
+def test_c1_mlp_dp2_exact(ctx):
+    sw = W.sweep_c1()
+    got = ctx.run_sweep(sw)
+    ref = oracle.run_sweep(sw)
+    bad, ulp = compare(got, ref)
+    assert not bad, bad
+    assert ulp == 0
+    assert (got["status"] == 0).all() and got["n_collectives"][0] == 8
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_random_small_all_strategies(ctx, seed):
+    """Random traces x random topologies x every strategy / collective, several hundred points
+    so each launch spans many warps, segments and a ragged tail."""
+    rng = np.random.Generator(np.random.PCG64(500 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=4)
+    topos = [W.random_topology(rng, n_gpus=g, n_switch=int(rng.integers(0, 3)), p_edge=0.25)
+             for g in (2, 3, 4, 5, 8, 12)]
+    topos += [W.ring(16, 40e9, 1e-6), W.star(8, 80e9, 2e-6), W.mesh(2, 4, 60e9, 1e-6), W.cube_mesh8(50e9, 1e-6),
+              W.double_ring(8, 30e9, 3e-6), W.perturb(W.ring_graph(8, 90e9, 1e-6), seed)]
+    pts = []
+    for _ in range(400):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        st = int(rng.integers(0, 4))
+        bw, lat = float(rng.uniform(0.2, 3.0)), float(rng.uniform(0.0, 2.0))
+        algo = int(rng.integers(0, 2))
+        if st in (W.ST_DP, W.ST_DDP):
+            dp = int(rng.integers(1, G + 1))
+            pts.append(W.make_point(ti, st, dp=dp, B=dp * int(rng.integers(1, 9)), algo=algo, bw=bw, lat=lat,
+                                    bucket=int(rng.choice([0, 1 << 10, 1 << 14, 1 << 30]))))
+        elif st == W.ST_TP:
+            tpd = int(rng.integers(1, G + 1))
+            pts.append(W.make_point(ti, st, tp=tpd, B=int(rng.integers(1, 9)), algo=algo, bw=bw, lat=lat,
+                                    tp_mode=int(rng.integers(0, 2))))
+        else:
+            pp = int(rng.integers(1, min(G, tr.n_layers) + 1))
+            m = int(rng.integers(1, 6))
+            pts.append(W.make_point(ti, st, pp=pp, m=m, B=m * int(rng.integers(1, 4)), bw=bw, lat=lat))
+    sw = W.Sweep("rand", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    check(got, sw, list(range(len(pts))))
+    assert (got["status"] == 0).sum() > 300
+
+
+def test_statuses_and_edge_cases(ctx):
+    tr = W.mlp_trace()
+    topos = [W.ring(4, 10e9, 1e-6), W.ring(32, 10e9, 1e-6), W.ring(40, 10e9, 1e-6), W.star(32, 10e9, 1e-6)]
+    links = np.zeros(1, W.LINK_DTYPE)
+    links[0] = (0, 1, 1e9, 0.0)
+    topos.insert(3, W.Topology("oneway", 2, 2, links, np.arange(2, dtype=np.uint32)))
+    P = W.make_point
+    pts = W.points_array([
+        P(0, W.ST_DP, dp=3, B=64),                       # bad batch
+        P(0, W.ST_DP, dp=5, B=5),                        # too many GPUs
+        P(0, W.ST_PP, pp=2, m=3, B=4),                   # bad batch (micro-batches)
+        P(0, W.ST_PP, pp=2, m=1, B=4, plan=0),           # explicit plan ok
+        P(0, W.ST_PP, pp=2, m=1, B=4, plan=1),           # bad plan
+        P(0, W.ST_PP, pp=2, m=1, B=4, plan=7),           # plan index out of range
+        P(9, W.ST_DP, dp=1, B=1),                        # topology out of range
+        P(0, 7, dp=1, B=1),                              # unknown strategy
+        P(0, W.ST_HYBRID, dp=2, tp=2, pp=1, m=1, B=4),   # hybrid: reserved
+        P(0, W.ST_DP, dp=1, B=64, bw=-1.0),              # bad scale
+        P(3, W.ST_DDP, dp=2, B=128),                     # no route back
+        P(1, W.ST_DDP, dp=32, B=32 * 64, bucket=1 << 20),  # 32 lanes: W = 32
+        P(4, W.ST_DDP, dp=32, B=32 * 64, algo=W.ALG_TREE),  # tree over a 32-GPU switch
+        P(0, W.ST_DP, dp=1, B=64),                       # single GPU: no communication
+        P(0, W.ST_TP, tp=1, B=64),
+        P(0, W.ST_PP, pp=1, m=2, B=128),
+    ])
+    sw = W.Sweep("edge", tr, topos, pts, plans=[[0, 2], [0, 0]])
+    got = ctx.run_sweep(sw)
+    check(got, sw, list(range(len(pts))))
+    assert list(got["status"][:11]) == [1, 2, 1, 0, 6, 6, 7, 7, 7, 7, 3]
+    # beyond the warp kernel's limits -- more than 32 lanes, a route longer than 8 hops (tree
+    # edges across a 32-GPU ring) -- is reported, never silently wrong
+    big = W.Sweep("big", tr, topos, W.points_array([P(2, W.ST_DDP, dp=40, B=40 * 64),
+                                                    P(1, W.ST_DDP, dp=32, B=32 * 64, algo=W.ALG_TREE)]))
+    assert list(ctx.run_sweep(big)["status"]) == [W.PT_TOO_LARGE, W.PT_TOO_LARGE]
+    # empty sweep
+    empty = W.Sweep("empty", tr, topos, np.zeros(0, W.POINT_DTYPE))
+    assert len(ctx.run_sweep(empty)) == 0
+
+
+def test_partial_ranges_and_device_results(ctx):
+    import torch
+    rng = np.random.Generator(np.random.PCG64(3))
+    tr = W.random_trace(rng, n_layers=4)
+    topos = [W.ring(8, 20e9, 1e-6), W.mesh(2, 2, 20e9, 1e-6)]
+    pts = W.points_array([W.make_point(i % 2, W.ST_DDP, dp=2 + (i % 3), B=12, bucket=(i % 4) * 500, bw=1 + i / 50)
+                          for i in range(300)])
+    sw = W.Sweep("ranges", tr, topos, pts)
+    tid = ctx.triosim_load_trace(tr)
+    sid = ctx.triosim_build_sweep(tid, topos, pts)
+    ctx.triosim_simulate_batch(sid, 0, 300)
+    full = ctx.triosim_results(sid, 0, 300)
+    for first, count in ((0, 1), (17, 83), (299, 1), (100, 0)):
+        ctx.triosim_simulate_batch(sid, first, count)
+        part = ctx.triosim_results(sid, first, count)
+        assert part.tobytes() == full[first:first + count].tobytes()
+    buf = torch.zeros(300 * W.RESULT_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.current_stream()
+    ctx.triosim_simulate_batch(sid, 0, 300, stream=s.cuda_stream)
+    ctx.triosim_results(sid, 0, 300, device_ptr=buf.data_ptr(), stream=s.cuda_stream)
+    torch.cuda.synchronize()
+    assert buf.cpu().numpy().tobytes() == full.tobytes()
+    with pytest.raises(Exception):
+        ctx.triosim_simulate_batch(sid, 250, 100)
+    ctx.triosim_release(sid)
+    ctx.triosim_release(tid)
+    check(full, sw, sample(300, 60, 1))
+
+
+def _properties_dp(got, sw):
+    ok = got["status"] == 0
+    assert ok.all()
+    tr = sw.trace
+    wsum = float(tr.tensors["bytes_b0"][tr.tensors["category"] == W.CAT_WGRAD].sum())
+    p = sw.points["dp"].astype(np.int64)
+    assert (got["coll_payload_bytes"] == wsum).all()
+    assert (got["n_compute"] == p * len(tr.ops)).all()
+    assert (got["n_flows"] == got["n_collectives"] * 2 * (p - 1) * p).all()
+    assert (got["iter_time_s"] >= got["compute_busy_max_s"]).all()
+    assert (got["exposed_comm_s"] == got["iter_time_s"] - got["compute_busy_max_s"]).all()
+
+
+def test_c2_resnet50_dp_full_sweep(ctx):
+    """configs[1] at full size (10,000 points, the bench workload): every point checked for
+    the invariants, a stratified seeded sample against the oracle."""
+    sw = W.sweep_c2()
+    got = ctx.run_sweep(sw)
+    _properties_dp(got, sw)
+    # stratify: a few points of each (p, batch, bucket) class
+    keys = {}
+    for i, pt in enumerate(sw.points):
+        keys.setdefault((int(pt["dp"]), int(pt["global_batch"]), int(pt["bucket_bytes"])), []).append(i)
+    idx = sorted(set(i for v in keys.values() for i in v[:10]) | set(sample(len(sw.points), 600, 2)))
+    check(got, sw, idx)
+
+
+def test_c3_bert_large_tp_sampled(ctx):
+    sw = W.sweep_c3()
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all()
+    check(got, sw, sample(len(sw.points), 1000, 3))
+
+
+def test_c4_gpt2xl_pp_sampled(ctx):
+    sw = W.sweep_c4()
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all()
+    assert (got["n_collectives"] == 0).all() and (got["n_p2p"] > 0).all()
+    # cheap points plus a few of the largest (S=16, m=64)
+    big = [i for i, pt in enumerate(sw.points) if pt["pp"] == 16 and pt["microbatches"] == 64][:3]
+    check(got, sw, sorted(set(sample(len(sw.points), 300, 4) + big)))
