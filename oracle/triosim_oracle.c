@@ -809,10 +809,6 @@ static uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     return z ^ (z >> 31);
 }
-static uint64_t fnv_u64(uint64_t h, uint64_t v) {
-    for (int b = 0; b < 8; b++) { h ^= (v >> (8 * b)) & 0xff; h *= 0x100000001b3ull; }
-    return h;
-}
 static uint64_t dbits(double d) { uint64_t u; memcpy(&u, &d, 8); return u; }
 
 /* ------------------------------------------------------------------ */
@@ -1055,7 +1051,8 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                 }
             } while (again);
 
-            if (nev > 0) { n_inst++; H = fnv_u64(H, dbits(t)); H = fnv_u64(H, acc); }
+            /* R19: H <- mix64(mix64(H ^ bits(t)) ^ sum of the instant's event mixes) */
+            if (nev > 0) { n_inst++; H = mix64(mix64(H ^ dbits(t)) ^ acc); }
             if (inflight > 0 && !busy_on) { busy_on = 1; busy_start = t; }
             else if (inflight == 0 && busy_on) { busy_on = 0; comm_busy = comm_busy + (t - busy_start); }
             if (n_done == NN) break;

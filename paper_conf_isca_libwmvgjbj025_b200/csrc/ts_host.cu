@@ -89,9 +89,10 @@ struct Sweep {
     DevBuf<uint16_t> d_rt_links;
     DevBuf<PointDesc> d_pts;
     DevBuf<triosim_result> d_res;
-    std::vector<uint32_t> work[6];           // per W index (2,4,8,16,32)
-    DevBuf<uint32_t> d_work[6];
-    DevBuf<uint32_t> d_work_tmp[6];
+    std::vector<uint32_t> work[N_GROUPS];    // per (W index, mode)
+    DevBuf<uint32_t> d_work[N_GROUPS];
+    DevBuf<uint32_t> d_work_tmp[N_GROUPS];
+    std::vector<int> mode;                   // per point
     DevBuf<unsigned int> d_counter;
     DevBuf<unsigned long long> d_alg;
     cudaStream_t last_stream = nullptr;
@@ -109,10 +110,10 @@ struct triosim_ctx {
     std::map<int, std::unique_ptr<Trace>> traces;
     std::map<int, std::unique_ptr<Sweep>> sweeps;
     int next_handle = 1;
-    cudaStream_t side[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
-    cudaEvent_t ev_fork = nullptr, ev_join[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+    cudaStream_t side[N_GROUPS] = {};
+    cudaEvent_t ev_fork = nullptr, ev_join[N_GROUPS] = {};
     uint64_t n_k1 = 0, n_k2 = 0, n_k3 = 0;
-    int occ[5] = {0, 0, 0, 0, 0};
+    int occ[N_GROUPS] = {};
     // optional CUDA-event timing of each simulate_batch (recorded on the caller's stream)
     static constexpr int NT = 512;
     bool timing = false;
@@ -152,13 +153,13 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
     if (!ctx) return TRIOSIM_ENOMEM;
     ctx->device = cuda_device;
     ctx->n_sms = prop.multiProcessorCount;
-    for (int i = 0; i < 5; i++) {
+    for (int i = 0; i < N_GROUPS; i++) {
         if (cudaStreamCreateWithFlags(&ctx->side[i], cudaStreamNonBlocking) != cudaSuccess ||
             cudaEventCreateWithFlags(&ctx->ev_join[i], cudaEventDisableTiming) != cudaSuccess) {
             triosim_destroy(ctx);
             return TRIOSIM_ECUDA;
         }
-        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i]);
+        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i / 2], i % 2);
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
         triosim_destroy(ctx);
@@ -174,7 +175,7 @@ void triosim_destroy(triosim_ctx *ctx) {
     cudaDeviceSynchronize();
     ctx->sweeps.clear();
     ctx->traces.clear();
-    for (int i = 0; i < 5; i++) {
+    for (int i = 0; i < N_GROUPS; i++) {
         if (ctx->side[i]) cudaStreamDestroy(ctx->side[i]);
         if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
     }
@@ -412,6 +413,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     S->status.assign(n_pts, -1);
     S->width.assign(n_pts, 0);
     S->cost.assign(n_pts, 0.0);
+    S->mode.assign(n_pts, 0);
     std::vector<PointDesc> pdesc(n_pts);
     std::map<std::tuple<int, int, int, int, int, uint64_t, int, int>, uint32_t> cls_of;
     std::vector<uint32_t> plan_pool;
@@ -519,6 +521,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         pd.idx = (uint32_t)i;
         pd.pad = 0;
         S->width[i] = W;
+        S->mode[i] = mode;
         double cost;
         if (mode == MODE_COLL) {
             double ncol = pt.strategy == TRIOSIM_TP ? n_tp_coll[pt.tp_mode == TRIOSIM_TP_PAPER ? 0 : 1]
@@ -569,8 +572,28 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         rt_links.insert(rt_links.end(), HT[i].links.begin(), HT[i].links.end());
         d.ro_off = (uint32_t)ro.size();
         ro.insert(ro.end(), HT[i].ro.begin(), HT[i].ro.end());
-        d.max_hops = HT[i].max_hops;
-        d.pad = 0;
+        d.ring_disjoint_lo = d.ring_disjoint_hi = 0;
+        {
+            const HostTopo &Ht = HT[i];
+            const uint32_t G = Ht.n_gpus;
+            for (uint32_t pp = 2; pp <= std::min<uint32_t>(G, 32); pp++) {
+                std::vector<char> seen(Ht.n_links, 0);
+                bool ok = true;
+                for (uint32_t r = 0; r < pp && ok; r++) {
+                    const size_t k = (size_t)Ht.ro[r] * G + Ht.ro[(r + 1) % pp];
+                    if (Ht.rt_len[k] == NO_ROUTE) { ok = false; break; }
+                    for (uint32_t h = 0; h < Ht.rt_len[k]; h++) {
+                        const uint16_t e = Ht.links[Ht.rt_off[k] + h];
+                        if (seen[e]) { ok = false; break; }
+                        seen[e] = 1;
+                    }
+                }
+                if (ok) {
+                    if (pp < 32) d.ring_disjoint_lo |= 1u << pp;
+                    else d.ring_disjoint_hi |= 1u << (pp - 32);
+                }
+            }
+        }
     }
     CK(S->d_topo.upload(td));
     CK(S->d_bw.upload(bw));
@@ -605,12 +628,12 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         if (S->cost[a] != S->cost[b]) return S->cost[a] > S->cost[b];
         return pdesc[a].cls < pdesc[b].cls;
     });
-    for (uint64_t i : order) S->work[w_index(S->width[i])].push_back((uint32_t)i);
-    for (int w = 0; w < 5; w++) {
+    for (uint64_t i : order) S->work[2 * w_index(S->width[i]) + S->mode[i]].push_back((uint32_t)i);
+    for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
         CK(S->d_work_tmp[w].alloc(S->work[w].size()));
     }
-    CK(S->d_counter.alloc(5));
+    CK(S->d_counter.alloc(N_GROUPS));
     CK(S->d_alg.alloc(1));
     CK(cudaMemset(S->d_alg.p, 0, sizeof(unsigned long long)));
     CK(cudaDeviceSynchronize());
@@ -652,12 +675,12 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     if (!S.pipe_list.empty()) ctx->n_k2++;
     // K3 per segment width, forked onto side streams so the widths run concurrently
     const bool full = first == 0 && count == S.n_pts;
-    CK(cudaMemsetAsync(S.d_counter.p, 0, 5 * sizeof(unsigned int), st));
+    CK(cudaMemsetAsync(S.d_counter.p, 0, N_GROUPS * sizeof(unsigned int), st));
     CK(cudaMemsetAsync(S.d_alg.p, 0, sizeof(unsigned long long), st));
     if (slot >= 0) CK(cudaEventRecord(ctx->t_mid[slot], st));
     CK(cudaEventRecord(ctx->ev_fork, st));
-    int launched[5] = {0, 0, 0, 0, 0};
-    for (int w = 0; w < 5; w++) {
+    int launched[N_GROUPS] = {};
+    for (int w = 0; w < N_GROUPS; w++) {
         const uint32_t *wl = S.d_work[w].p;
         uint32_t n = (uint32_t)S.work[w].size();
         if (!full) {
@@ -669,7 +692,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
             wl = S.d_work_tmp[w].p;
         }
         if (n == 0) continue;
-        const int W = W_OF[w];
+        const int W = W_OF[w / 2], mode = w % 2;
         K3Args a;
         std::memset(&a, 0, sizeof a);
         a.pts = S.d_pts.p; a.work = wl; a.n_work = n; a.counter = S.d_counter.p + w;
@@ -686,12 +709,12 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)ctx->occ[w];
         if (blocks > cap) blocks = cap;
         CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
-        CK(launch_k3(W, a, (int)blocks, ctx->side[w]));
+        CK(launch_k3(W, mode, a, (int)blocks, ctx->side[w]));
         ctx->n_k3++;
         CK(cudaEventRecord(ctx->ev_join[w], ctx->side[w]));
         launched[w] = 1;
     }
-    for (int w = 0; w < 5; w++)
+    for (int w = 0; w < N_GROUPS; w++)
         if (launched[w]) CK(cudaStreamWaitEvent(st, ctx->ev_join[w], 0));
     if (slot >= 0) {
         CK(cudaEventRecord(ctx->t_end[slot], st));

@@ -94,7 +94,10 @@ struct ClassDesc {
 
 struct TopoDev {
     uint32_t n_nodes, n_gpus, n_links, link_off;
-    uint32_t rt_off, ro_off, max_hops, pad;
+    uint32_t rt_off, ro_off;
+    // bit p (p = 2..32 over the two words): the routes ring_order[i] -> ring_order[(i+1) % p] of
+    // the first p GPUs are pairwise link-disjoint, so ring flows never share a link (K3 fast path)
+    uint32_t ring_disjoint_lo, ring_disjoint_hi;
 };
 
 struct PointDesc {
@@ -133,7 +136,9 @@ cudaError_t launch_k2_coll(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T, const double *dur,
                            const uint32_t *plan_pool, StageInfo *stages, StageEnt *ents, SendEnt *sends,
                            RecvEnt *recvs, unsigned long long *scratch_u64, cudaStream_t s);
-cudaError_t launch_k3(int W, const K3Args &a, int grid, cudaStream_t s);
-int k3_max_blocks_per_sm(int W);
+cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
+int k3_max_blocks_per_sm(int W, int mode);
+constexpr int N_WIDTHS = 5;             // W = 2, 4, 8, 16, 32
+constexpr int N_GROUPS = 2 * N_WIDTHS;  // (width, mode) launch groups
 
 }  // namespace ts

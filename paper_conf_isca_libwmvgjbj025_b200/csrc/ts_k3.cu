@@ -1,0 +1,714 @@
+// ts_k3.cu -- K3, the timeline kernel.
+//
+// One design point per W-lane segment of a warp (W = 2..32, 32/W points per warp).  Lane i of a
+// segment is simulated GPU i: it owns that GPU's in-order compute stream and its single flow slot
+// (ring step i -> i+1, tree edge, or the GPU's FIFO P2P send).  Segment-wide decisions are
+// ballots / shuffles: collective start (all members ready), ring predecessor progress, the
+// bottleneck share of each water-filling round, the next event time.
+//
+// Instant processing (R17) is ONE ordered pass -- completions, deliveries, activations,
+// collective done / finish / start, releases, compute starts -- which is already a fixed point
+// because every phase only consumes state produced by earlier phases; the pass repeats only when
+// a zero-latency release or a zero-duration operator creates another event at the same instant.
+// Then the max-min progressive filling (R14) re-allocates every in-transit flow if the active set
+// changed, and the instant repeats if that made a flow drain now.
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "ts_internal.h"
+
+namespace ts {
+
+#define FULL 0xffffffffu
+
+enum { CS_IDLE = 0, CS_RUN = 1 };
+enum { FS_NONE = 0, FS_LAT = 1, FS_ACT = 2 };
+enum { EV_COLL_START = 1, EV_RELEASE = 2, EV_ACTIVATE = 3, EV_DELIVER = 4, EV_TASK_START = 5, EV_TASK_END = 6 };
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    return z ^ (z >> 31);
+}
+__device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
+
+template <int W>
+__device__ __forceinline__ double seg_min(double v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) {
+        double w = __shfl_xor_sync(FULL, v, o);
+        v = w < v ? w : v;
+    }
+    return v;
+}
+template <int W>
+__device__ __forceinline__ double seg_max(double v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) {
+        double w = __shfl_xor_sync(FULL, v, o);
+        v = w > v ? w : v;
+    }
+    return v;
+}
+template <int W>
+__device__ __forceinline__ unsigned long long seg_sum_u64(unsigned long long v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+template <int W>
+__device__ __forceinline__ uint32_t seg_sum_u32(uint32_t v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+
+struct Route {
+    uint32_t off;
+    int len;
+};
+
+struct TopoRef {
+    uint32_t n_gpus, link_off, rt_off, ro_off;
+};
+
+__device__ __forceinline__ Route get_route(const K3Args &a, const TopoRef &T, uint32_t s, uint32_t d) {
+    const uint32_t k = T.rt_off + s * T.n_gpus + d;
+    Route r;
+    r.len = a.rt_len[k];
+    r.off = a.rt_off[k];
+    return r;
+}
+
+// route latency: left fold of link latency x lat_scale (R12); caches the link ids (<= 8 hops,
+// 16 bit each) in four registers for the water-filling rounds
+__device__ __forceinline__ double load_route(const K3Args &a, const TopoRef &T, Route r, double lat_scale,
+                                             uint32_t (&hl)[4]) {
+    double L = 0.0;
+    hl[0] = hl[1] = hl[2] = hl[3] = 0;
+#pragma unroll
+    for (int h = 0; h < MAX_HOPS; h++)
+        if (h < r.len) {
+            const uint32_t e = a.rt_links[r.off + h];
+            hl[h >> 1] |= e << (16 * (h & 1));
+            L = L + a.link_lat[T.link_off + e] * lat_scale;
+        }
+    return L;
+}
+__device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[h >> 1] >> (16 * (h & 1))) & 0xffff; }
+
+template <int W, int MODE>
+__global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
+    constexpr int NSEG = 32 / W;
+    constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
+    constexpr bool COLL = MODE == MODE_COLL;
+    __shared__ double s_res[K3_WARPS][NSEG * LMAX];
+    __shared__ int s_n[K3_WARPS][NSEG * LMAX];
+    __shared__ int s_k[K3_WARPS][NSEG * LMAX];
+    __shared__ uint32_t s_cnt[K3_WARPS][COLL ? 1 : 32];
+
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int seg = lane / W, li = lane % W, sbase = seg * W;
+    const unsigned smask = (W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase;
+    double *lres = &s_res[wid][seg * LMAX];
+    int *ln = &s_n[wid][seg * LMAX];
+    int *lk = &s_k[wid][seg * LMAX];
+    uint32_t *cnt = &s_cnt[wid][COLL ? 0 : sbase];
+    for (int q = lane; q < NSEG * LMAX; q += 32) { s_n[wid][q] = 0; s_k[wid][q] = 0; }
+    __syncwarp();
+
+    // ---- per-segment (uniform) state ----
+    bool have = false, exhausted = false;
+    uint32_t pidx = 0;
+    double t = 0.0, bws = 1.0, lats = 1.0;
+    int p = 1;
+    uint32_t ncoll = 0, m = 1;
+    const ClassDesc *C = nullptr;
+    TopoRef TR = {0, 0, 0, 0};
+    uint64_t H = 0;
+    uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
+    bool bon = false;
+    double bstart = 0.0, cbusy = 0.0;
+    uint32_t cur = 0;
+    bool running = false, tree_cur = false, tree_algo = false, ring_fast = false;
+    int K = 0;
+    double cS = 0.0, chunk = 0.0;
+    // ---- per-lane state ----
+    bool used = false;
+    uint32_t gpu = 0, pos = 0, run_start = 0, run_end = 0, nprog = 0;
+    int cst = CS_IDLE;
+    int hwait = -1;           // COLL: cached wait of the head operator
+    double t_end = 0.0, busy = 0.0;
+    uint32_t ntask = 0, nflow = 0;
+    uint32_t trig = 0, donec = 0;
+    int D = 0;
+    bool ldone = false, uprel = false, upd = false, dnrel = false, dnd = false, fup = false;
+    Route rring = {0, 0};
+    uint32_t hring[4] = {0, 0, 0, 0};
+    double Lring = 0.0, rbw = 0.0;   // ring flow: route latency, min-hop bandwidth
+    int fst = FS_NONE;
+    double t_act = 0.0, rem = 0.0, rate = 0.0, t_upd = 0.0, t_drain = 0.0, fbytes = 0.0;
+    int flen = 0;
+    uint32_t hl[4] = {0, 0, 0, 0};
+    uint64_t fcode = 0;
+    StageInfo SI;
+    SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
+    SI.ent_off = SI.send_off = SI.recv_off = 0;
+    uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
+    uint64_t acc = 0, alg = 0;
+    uint32_t nev = 0;
+
+#define EV(kind, code)                                                  \
+    do {                                                                \
+        acc += mix64(((uint64_t)(kind) << 60) | (uint64_t)(code));      \
+        nev++;                                                          \
+    } while (0)
+
+    for (;;) {
+        // ------------------------------ refill ------------------------------
+        const bool need = !have && !exhausted;
+        uint32_t it = 0;
+        if (need && li == 0) it = atomicAdd(a.counter, 1u);
+        it = __shfl_sync(FULL, it, sbase);
+        bool fresh = false, rbad = false, rlong = false;
+        if (need) {
+            if (it >= a.n_work) {
+                exhausted = true;
+            } else {
+                fresh = have = true;
+                const PointDesc pd = a.pts[a.work[it]];
+                pidx = pd.idx;
+                bws = pd.bw_scale;
+                lats = pd.lat_scale;
+                C = &a.cls[pd.cls];
+                p = (int)C->p;
+                {
+                    const TopoDev td = a.topo[pd.topo];
+                    TR.n_gpus = td.n_gpus; TR.link_off = td.link_off; TR.rt_off = td.rt_off; TR.ro_off = td.ro_off;
+                    ring_fast = COLL && (p < 32 ? (td.ring_disjoint_lo >> p) & 1u : (td.ring_disjoint_hi >> (p - 32)) & 1u);
+                }
+                ncoll = C->n_coll;
+                m = C->m;
+                tree_algo = C->algo == TRIOSIM_ALGO_TREE;
+                t = 0.0;
+                H = 0xcbf29ce484222325ull;
+                ninst = nwf = nrounds = maxact = 0;
+                bon = false;
+                bstart = cbusy = 0.0;
+                cur = 0;
+                running = false;
+                used = li < p;
+                pos = run_start = run_end = 0;
+                cst = CS_IDLE;
+                t_end = busy = 0.0;
+                ntask = nflow = 0;
+                trig = donec = 0;
+                D = 0;
+                ldone = uprel = upd = dnrel = dnd = false;
+                fst = FS_NONE;
+                sq = dcnt = 0;
+                acc = alg = 0;
+                nev = 0;
+                if (used) {
+                    gpu = a.ro[TR.ro_off + li];
+                    if constexpr (COLL) {
+                        nprog = C->n_prog_max;
+                        hwait = nprog > 0 ? a.hooks[C->hook_off].wait : -1;
+                        rring = get_route(a, TR, gpu, a.ro[TR.ro_off + (li + 1) % p]);
+                        if (C->need_ring) {
+                            if (rring.len == NO_ROUTE) rbad = true;
+                            else if (rring.len > MAX_HOPS) rlong = true;
+                        }
+                        if (rring.len != NO_ROUTE && rring.len <= MAX_HOPS) {
+                            Lring = load_route(a, TR, rring, lats, hring);
+                            alg += 2 * rring.len;
+                            // link-disjoint ring (host-checked): a ring flow is alone on each of its
+                            // links, so its max-min share is its smallest bw * bw_scale (R14 with
+                            // n_e = 1: res_e / 1.0 == res_e exactly)
+                            rbw = dinf();
+#pragma unroll
+                            for (int h = 0; h < MAX_HOPS; h++)
+                                if (h < rring.len) {
+                                    const double b = a.link_bw[TR.link_off + hop(hring, h)] * bws;
+                                    rbw = b < rbw ? b : rbw;
+                                }
+                            alg += 2 * rring.len;
+                        }
+                        if (C->need_tree && li >= 1) {
+                            const uint32_t par = a.ro[TR.ro_off + (li - 1) / 2];
+                            const int l1 = get_route(a, TR, gpu, par).len, l2 = get_route(a, TR, par, gpu).len;
+                            if (l1 == NO_ROUTE || l2 == NO_ROUTE) rbad = true;
+                            else if (l1 > MAX_HOPS || l2 > MAX_HOPS) rlong = true;
+                        }
+                    } else {
+                        SI = a.stages[C->stage_off + li];
+                        nprog = m * (SI.nF + SI.nB) + SI.nO;
+                        nsend_tot = m * (SI.SF + SI.SB) + SI.SO;
+                        unsigned long long dm = SI.dst_mask;
+                        while (dm) {
+                            const int d = __ffsll((long long)dm) - 1;
+                            dm &= dm - 1;
+                            const int l = get_route(a, TR, gpu, a.ro[TR.ro_off + d]).len;
+                            if (l == NO_ROUTE) rbad = true;
+                            else if (l > MAX_HOPS) rlong = true;
+                        }
+                    }
+                }
+            }
+        }
+        if (__all_sync(FULL, !have)) break;
+        {
+            // a needed (src, dst) pair without a path (R3) / beyond this kernel's hop limit
+            const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
+            const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
+            if (fresh && (bad || lng)) {
+                if (li == 0) {
+                    triosim_result r = {};
+                    r.status = bad ? TRIOSIM_PT_NO_ROUTE : TRIOSIM_PT_TOO_LARGE;
+                    a.out[pidx] = r;
+                }
+                have = used = false;
+            }
+        }
+
+        // ------------------------------ one instant at time t ------------------------------
+        bool dirty = false;
+        for (;;) {
+            for (;;) {
+                bool more = false;
+                // (a) compute completions
+                if (used && cst == CS_RUN && t_end == t) {
+                    cst = CS_IDLE;
+                    pos = run_end;
+                    if constexpr (COLL) {
+                        const uint32_t ns = a.hooks[C->hook_off + pos - 1].nsig;
+                        if (ns) {
+                            trig += ns;
+                            EV(EV_TASK_END, ((uint64_t)gpu << 40) | (pos - 1));
+                        }
+                        hwait = pos < nprog ? a.hooks[C->hook_off + pos].wait : -1;
+                    } else {
+                        const uint32_t q = pos - 1;
+                        uint32_t P, idx;
+                        if (q < m * SI.nF) { P = 0; idx = q % SI.nF; }
+                        else if (q < m * (SI.nF + SI.nB)) { P = 1; idx = (q - m * SI.nF) % SI.nB; }
+                        else { P = 2; idx = q - m * (SI.nF + SI.nB); }
+                        const uint32_t eo = SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx;
+                        if (a.ents[eo].nsend) EV(EV_TASK_END, ((uint64_t)gpu << 40) | q);
+                    }
+                }
+                // (b) deliveries and (c) activations after the route latency (Q19)
+                bool delivered = false;
+                if (used && fst == FS_ACT && t_drain == t) {
+                    fst = FS_NONE;
+                    EV(EV_DELIVER, fcode);
+                    delivered = dirty = true;
+                } else if (used && fst == FS_LAT && t_act == t) {
+                    EV(EV_ACTIVATE, fcode);
+                    if (fbytes == 0.0 || flen == 0) {
+                        fst = FS_NONE;
+                        EV(EV_DELIVER, fcode);
+                        delivered = true;
+                    } else {
+                        fst = FS_ACT;
+                        rem = fbytes;
+                        t_upd = t;
+                        rate = 0.0;
+                        t_drain = dinf();
+                        dirty = true;
+                    }
+                }
+                if (delivered) {
+                    nflow++;
+                    if constexpr (COLL) {
+                        if (tree_cur) {
+                            if (fup) upd = true; else dnd = true;
+                        } else {
+                            D++;
+                        }
+                    } else {
+                        dcnt++;
+                    }
+                }
+                if constexpr (COLL) {
+                    // (d) collective progress: done on this GPU, finish, start (R10)
+                    const int pred = (li + p - 1) % p;
+                    const int Dp = __shfl_sync(FULL, D, sbase + pred);
+                    const unsigned upm = (__ballot_sync(FULL, upd) & smask) >> sbase;
+                    const unsigned dnm = (__ballot_sync(FULL, dnd) & smask) >> sbase;
+                    const int c1 = 2 * li + 1, c2 = 2 * li + 2;
+                    if (used && running && !ldone) {
+                        bool dn;
+                        if (!tree_cur) {
+                            dn = D == K && Dp == K;
+                        } else {
+                            const bool ku = (c1 >= p || ((upm >> c1) & 1u)) && (c2 >= p || ((upm >> c2) & 1u));
+                            const bool kd = (c1 >= p || ((dnm >> c1) & 1u)) && (c2 >= p || ((dnm >> c2) & 1u));
+                            dn = (li == 0 || (upd && dnd)) && ku && kd;
+                        }
+                        if (dn) {
+                            ldone = true;
+                            donec = cur + 1;
+                        }
+                    }
+                    const bool allfin = (__ballot_sync(FULL, !used || ldone) & smask) == smask;
+                    if (have && running && allfin) {
+                        running = false;
+                        cur++;
+                    }
+                    const bool allrdy = (__ballot_sync(FULL, !used || trig > cur) & smask) == smask;
+                    bool started = false;
+                    if (have && !running && cur < ncoll && allrdy) {
+                        // every member ready: the collective starts (barrier, Q22)
+                        const CollEnt ce = a.colls[C->coll_off + cur];
+                        running = started = true;
+                        tree_cur = tree_algo && ce.kind == CK_AR;
+                        cS = ce.S;
+                        chunk = ce.S / (double)p;
+                        K = (ce.kind == CK_AR) ? 2 * (p - 1) : (p - 1);
+                        D = 0;
+                        ldone = uprel = upd = dnrel = dnd = false;
+                        if (li == 0) { EV(EV_COLL_START, cur); alg += 1; }
+                    }
+                    if (used && running && fst == FS_NONE) {
+                        bool rel = false;
+                        if (!tree_cur) {
+                            if (D < K && (D == 0 || Dp >= D)) {
+                                // ring step (i, k = D): m_i -> m_{i+1}, S/p bytes (Q21)
+                                rel = true;
+                                flen = rring.len;
+                                hl[0] = hring[0]; hl[1] = hring[1]; hl[2] = hring[2]; hl[3] = hring[3];
+                                fbytes = chunk;
+                                t_act = t + Lring;
+                                alg += 1;
+                                fcode = ((uint64_t)cur << 32) | ((uint64_t)D << 16) | (uint64_t)li;
+                            }
+                        } else if (li >= 1) {
+                            const unsigned um = started ? 0u : upm, dm = started ? 0u : dnm;
+                            const bool ku = (c1 >= p || ((um >> c1) & 1u)) && (c2 >= p || ((um >> c2) & 1u));
+                            const int par_i = (li - 1) / 2;
+                            const uint32_t par = a.ro[TR.ro_off + par_i];
+                            if (!uprel && ku) {
+                                // tree reduce edge i -> parent(i) (Q25)
+                                const Route r = get_route(a, TR, gpu, par);
+                                flen = r.len;
+                                t_act = t + load_route(a, TR, r, lats, hl);
+                                fcode = ((uint64_t)cur << 32) | (uint64_t)li;
+                                fup = uprel = rel = true;
+                            } else if (uprel && upd && !dnrel &&
+                                       (par_i == 0 ? ((p <= 1 || ((um >> 1) & 1u)) && (p <= 2 || ((um >> 2) & 1u)))
+                                                   : ((dm >> par_i) & 1u))) {
+                                // tree broadcast edge parent(i) -> i
+                                const Route r = get_route(a, TR, par, gpu);
+                                flen = r.len;
+                                t_act = t + load_route(a, TR, r, lats, hl);
+                                fcode = ((uint64_t)cur << 32) | (1ull << 16) | (uint64_t)li;
+                                fup = false;
+                                dnrel = rel = true;
+                            }
+                            if (rel) {
+                                fbytes = cS;
+                                alg += 2 * flen + 1;
+                            }
+                        }
+                        if (rel) {
+                            fst = FS_LAT;
+                            EV(EV_RELEASE, fcode);
+                            if (t_act == t) more = true;
+                        }
+                    }
+                } else {
+                    cnt[li] = dcnt;
+                    __syncwarp();
+                    if (used && fst == FS_NONE && sq < nsend_tot) {
+                        // next P2P send of this stage's FIFO stream (R11, Q14)
+                        uint32_t P, j, e;
+                        if (sq < m * SI.SF) { P = 0; j = sq / SI.SF; e = sq % SI.SF; }
+                        else if (sq < m * (SI.SF + SI.SB)) { const uint32_t r = sq - m * SI.SF; P = 1; j = m - 1 - r / SI.SB; e = r % SI.SB; }
+                        else { P = 2; j = 0; e = sq - m * (SI.SF + SI.SB); }
+                        const SendEnt se = a.sends[SI.send_off + (P == 0 ? 0 : P == 1 ? SI.SF : SI.SF + SI.SB) + e];
+                        const uint32_t prodpos = P == 0 ? j * SI.nF + se.pidx
+                                               : P == 1 ? m * SI.nF + (m - 1 - j) * SI.nB + se.pidx
+                                                        : m * (SI.nF + SI.nB) + se.pidx;
+                        const uint32_t donepos = (cst == CS_RUN) ? run_start : pos;
+                        if (donepos > prodpos) {
+                            const uint32_t dg = a.ro[TR.ro_off + se.dst];
+                            const Route r = get_route(a, TR, gpu, dg);
+                            flen = r.len;
+                            fst = FS_LAT;
+                            fbytes = se.bytes;
+                            t_act = t + load_route(a, TR, r, lats, hl);
+                            alg += 2 * flen + 1;
+                            fcode = (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg;
+                            EV(EV_RELEASE, fcode);
+                            sq++;
+                            if (t_act == t) more = true;
+                        }
+                    }
+                }
+                // (e) an idle GPU starts its head operator once its inputs are present
+                if (used && cst == CS_IDLE && pos < nprog) {
+                    if constexpr (COLL) {
+                        if (hwait < 0 || (int)donec > hwait) {
+                            const OpHook *HK = a.hooks + C->hook_off;
+                            const OpHook h = HK[pos];
+                            if (h.wait >= 0) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
+                            run_start = pos;
+                            double te = t + h.dur;
+                            busy = busy + h.dur;
+                            uint32_t q = pos + 1, sig = h.nsig;
+                            while (sig == 0 && q < nprog) {
+                                const OpHook h2 = HK[q];
+                                if (h2.wait >= 0) break;
+                                te = te + h2.dur;
+                                busy = busy + h2.dur;
+                                sig = h2.nsig;
+                                q++;
+                            }
+                            ntask += q - pos;
+                            alg += 2 * (q - pos);
+                            run_end = q;
+                            t_end = te;
+                            cst = CS_RUN;
+                            if (te == t) more = true;
+                        }
+                    } else {
+                        uint32_t q = pos, P, j, idx;
+                        if (q < m * SI.nF) { P = 0; j = q / SI.nF; idx = q % SI.nF; }
+                        else if (q < m * (SI.nF + SI.nB)) { const uint32_t r = q - m * SI.nF; P = 1; j = m - 1 - r / SI.nB; idx = r % SI.nB; }
+                        else { P = 2; j = 0; idx = q - m * (SI.nF + SI.nB); }
+                        const StageEnt en = a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx];
+                        bool ok = true;
+                        for (uint32_t r = 0; r < en.nrecv && ok; r++) {
+                            const RecvEnt re = a.recvs[en.recv_off + r];
+                            const StageInfo &ps = a.stages[C->stage_off + re.src];
+                            const uint32_t jp = (re.phase == 2 || P == 2) ? 0 : j;
+                            const uint32_t seqi = re.phase == 0 ? jp * ps.SF + re.e
+                                                : re.phase == 1 ? m * ps.SF + (m - 1 - jp) * ps.SB + re.e
+                                                                : m * (ps.SF + ps.SB) + re.e;
+                            if (!(cnt[re.src] > seqi)) ok = false;
+                        }
+                        if (ok) {
+                            if (en.nrecv) EV(EV_TASK_START, ((uint64_t)gpu << 40) | q);
+                            run_start = pos;
+                            const double *du = a.dur + C->dur_off;
+                            const double d0 = du[en.op];
+                            double te = t + d0;
+                            busy = busy + d0;
+                            uint32_t ns = en.nsend;
+                            q++;
+                            while (ns == 0 && q < nprog) {
+                                if (q < m * SI.nF) { P = 0; idx = q % SI.nF; }
+                                else if (q < m * (SI.nF + SI.nB)) { P = 1; idx = (q - m * SI.nF) % SI.nB; }
+                                else { P = 2; idx = q - m * (SI.nF + SI.nB); }
+                                const StageEnt e2 = a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx];
+                                if (e2.nrecv) break;
+                                const double dd = du[e2.op];
+                                te = te + dd;
+                                busy = busy + dd;
+                                ns = e2.nsend;
+                                q++;
+                            }
+                            ntask += q - pos;
+                            alg += 2 * (q - pos);
+                            run_end = q;
+                            t_end = te;
+                            cst = CS_RUN;
+                            if (te == t) more = true;
+                        }
+                    }
+                }
+                if constexpr (!COLL) __syncwarp();
+                if (!__any_sync(FULL, more)) break;
+            }
+
+            // (f) bandwidth re-allocation of every in-transit flow: max-min fair
+            //     progressive filling (R14, Q18)
+            const bool segdirty = (__ballot_sync(FULL, dirty) & smask) != 0;
+            if (!__any_sync(FULL, segdirty)) break;
+            dirty = false;
+            const bool act = segdirty && used && fst == FS_ACT;
+            // ring_fast is segment-uniform and only set while a ring collective runs (tree_cur off)
+            const bool fast = ring_fast && !tree_cur;
+            const bool gen = act && !fast;
+            if (act && t_upd < t) {
+                const double r = rem - rate * (t - t_upd);
+                rem = r > 0.0 ? r : 0.0;
+                t_upd = t;
+                alg += 4;
+            }
+            if (gen) {
+                alg += flen;
+#pragma unroll
+                for (int h = 0; h < MAX_HOPS; h++) if (h < flen) ln[hop(hl, h)] = 0;
+            }
+            __syncwarp();
+            if (gen) {
+#pragma unroll
+                for (int h = 0; h < MAX_HOPS; h++)
+                    if (h < flen) {
+                        const int e = hop(hl, h);
+                        atomicAdd(&ln[e], 1);
+                        lres[e] = a.link_bw[TR.link_off + e] * bws;
+                    }
+            }
+            __syncwarp();
+            if (act && fast) rate = rbw;
+            bool unf = act;
+            uint32_t rounds = 0;
+            while (__any_sync(FULL, unf)) {
+                const bool segact = (__ballot_sync(FULL, unf) & smask) != 0;
+                double my = dinf();
+                if (unf) {
+                    if (fast) {
+                        my = rate;
+                    } else {
+#pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if (h < flen) {
+                                const int e = hop(hl, h);
+                                const double sh = lres[e] / (double)ln[e];
+                                my = sh < my ? sh : my;
+                            }
+                        alg += 2 * flen;
+                    }
+                }
+                const double s = seg_min<W>(my);
+                const bool inF = unf && my == s;
+                unsigned own = 0;
+                if (inF && !fast) {
+                    rate = s;
+#pragma unroll
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if (h < flen && atomicAdd(&lk[hop(hl, h)], 1) == 0) own |= 1u << h;
+                }
+                __syncwarp();
+                if (inF && !fast) {
+#pragma unroll
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if ((own >> h) & 1u) {
+                            const int e = hop(hl, h);
+                            const int kk = lk[e];
+                            const double r = lres[e] - s * (double)kk;
+                            lres[e] = r > 0.0 ? r : 0.0;
+                            ln[e] -= kk;
+                            lk[e] = 0;
+                            alg += 3;
+                        }
+                }
+                __syncwarp();
+                if (segact) rounds++;
+                unf = unf && !inF;
+            }
+            const uint32_t nact = __popc(__ballot_sync(FULL, act) & smask);
+            if (segdirty) {
+                nwf++;
+                nrounds += rounds;
+                if (nact > maxact) maxact = nact;
+            }
+            bool again = false;
+            if (act) {
+                t_drain = (rem == 0.0) ? t : t + rem / rate;
+                alg += 2;
+                again = t_drain == t;
+            }
+            if (!__any_sync(FULL, again)) break;
+        }
+
+        // ------------------------------ end of instant ------------------------------
+        if (__ballot_sync(FULL, nev > 0) & smask) {
+            const unsigned long long acc_s = seg_sum_u64<W>(acc);
+            if (have) {
+                H = mix64(mix64(H ^ (uint64_t)__double_as_longlong(t)) ^ acc_s);   // R19
+                ninst++;
+            }
+        } else {
+            seg_sum_u64<W>(0ull);  // keep every lane on the same shuffles
+        }
+        acc = 0;
+        nev = 0;
+        const bool infl = (__ballot_sync(FULL, used && fst != FS_NONE) & smask) != 0;
+        if (have) {
+            if (infl && !bon) { bon = true; bstart = t; }
+            else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
+        }
+        bool lane_done = !used || (cst == CS_IDLE && pos >= nprog && fst == FS_NONE);
+        if constexpr (!COLL) lane_done = lane_done && (!used || sq >= nsend_tot);
+        const bool alldone = (__ballot_sync(FULL, lane_done) & smask) == smask;
+        const bool fin = have && alldone && (!COLL || (cur >= ncoll && !running));
+        double cand = dinf();
+        if (used) {
+            if (cst == CS_RUN) cand = t_end;
+            if (fst == FS_LAT && t_act < cand) cand = t_act;
+            if (fst == FS_ACT && t_drain < cand) cand = t_drain;
+        }
+        const double tn = seg_min<W>(cand);
+        const bool stuck = have && !fin && !(tn < dinf());
+        if (__any_sync(FULL, fin || stuck)) {
+            const double bmax = seg_max<W>(used ? busy : 0.0);
+            const uint32_t ntk = seg_sum_u32<W>(ntask);
+            const uint32_t nfl = seg_sum_u32<W>(nflow);
+            const unsigned long long alg_s = seg_sum_u64<W>(alg);
+            if ((fin || stuck) && li == 0) {
+                triosim_result r;
+                r.iter_time_s = fin ? t : 0.0;
+                r.compute_busy_max_s = fin ? bmax : 0.0;
+                r.comm_busy_s = fin ? cbusy : 0.0;
+                r.exposed_comm_s = fin ? t - bmax : 0.0;
+                r.coll_payload_bytes = fin ? C->coll_payload : 0.0;
+                r.n_compute = fin ? (uint64_t)ntk : 0;
+                r.n_flows = fin ? (uint64_t)nfl : 0;
+                r.n_collectives = fin ? ncoll : 0;
+                r.n_p2p = (fin && !COLL) ? (uint64_t)nfl : 0;
+                r.n_instants = fin ? ninst : 0;
+                r.n_wf_calls = fin ? nwf : 0;
+                r.n_wf_rounds = fin ? nrounds : 0;
+                r.order_hash = fin ? H : 0;
+                r.status = fin ? TRIOSIM_PT_OK : TRIOSIM_PT_DEADLOCK;
+                r.max_active_flows = fin ? maxact : 0;
+                a.out[pidx] = r;
+                if (a.alg_ops) atomicAdd(a.alg_ops, alg_s);
+            }
+            if (fin || stuck) have = used = false;
+        }
+        if (have) t = tn;
+    }
+#undef EV
+}
+
+template <int W, int MODE>
+static cudaError_t launch_wm(const K3Args &a, int grid, cudaStream_t s) {
+    k3_timeline<W, MODE><<<grid, K3_THREADS, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s) {
+#define CASE(w)                                                                                  \
+    case w:                                                                                      \
+        return mode == MODE_COLL ? launch_wm<w, MODE_COLL>(a, grid, s) : launch_wm<w, MODE_PIPE>(a, grid, s);
+    switch (W) {
+        CASE(2) CASE(4) CASE(8) CASE(16) CASE(32)
+    default:
+        return cudaErrorInvalidValue;
+    }
+#undef CASE
+}
+
+int k3_max_blocks_per_sm(int W, int mode) {
+    int nb = 0;
+#define CASE(w)                                                                                          \
+    case w:                                                                                              \
+        if (mode == MODE_COLL)                                                                           \
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<w, MODE_COLL>, K3_THREADS, 0); \
+        else                                                                                             \
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<w, MODE_PIPE>, K3_THREADS, 0); \
+        break;
+    switch (W) {
+        CASE(2) CASE(4) CASE(8) CASE(16) CASE(32)
+    default:
+        break;
+    }
+#undef CASE
+    return nb > 0 ? nb : 1;
+}
+
+}  // namespace ts
