@@ -925,7 +925,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
 
         long n_done = 0;
         double t = 0.0;
-        uint64_t H = 0xcbf29ce484222325ull;
+        uint64_t H = 0;
         uint64_t n_inst = 0, n_wf = 0, n_rounds = 0;
         uint32_t max_act = 0;
         int busy_on = 0;
@@ -943,10 +943,12 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
             }                                                                \
         }                                                                    \
     } while (0)
-#define EVENT(kind, code) do { acc += mix64(((uint64_t)(kind) << 60) | (code)); nev++; } while (0)
+/* R19: order hash = sum over events of mix64(mix64(bits(t)) ^ (kind << 60 | code)) */
+#define EVENT(kind, code) do { acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (code))); nev++; } while (0)
 
         for (;;) {
             uint64_t acc = 0;
+            const uint64_t tmix = mix64(dbits(t));
             long nev = 0;
             int again;
             int dirty = 0;
@@ -1051,8 +1053,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                 }
             } while (again);
 
-            /* R19: H <- mix64(mix64(H ^ bits(t)) ^ sum of the instant's event mixes) */
-            if (nev > 0) { n_inst++; H = mix64(mix64(H ^ dbits(t)) ^ acc); }
+            if (nev > 0) { n_inst++; H = H + acc; }
             if (inflight > 0 && !busy_on) { busy_on = 1; busy_start = t; }
             else if (inflight == 0 && busy_on) { busy_on = 0; comm_busy = comm_busy + (t - busy_start); }
             if (n_done == NN) break;

@@ -31,14 +31,26 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
 }
 __device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
 
+#ifndef TS_SEGMIN_REDUX
+#define TS_SEGMIN_REDUX 0
+#endif
 template <int W>
-__device__ __forceinline__ double seg_min(double v) {
+__device__ __forceinline__ double seg_min_shfl(double v) {
 #pragma unroll
     for (int o = W / 2; o > 0; o >>= 1) {
         double w = __shfl_xor_sync(FULL, v, o);
         v = w < v ? w : v;
     }
     return v;
+}
+// minimum of a NON-NEGATIVE double over the lanes of `mask` (this lane's segment): such doubles
+// order like their bit patterns, so two 32-bit warp reductions (REDUX) give the exact minimum
+__device__ __forceinline__ double seg_min_redux(double v, unsigned mask) {
+    const unsigned long long b = (unsigned long long)__double_as_longlong(v);
+    const unsigned hi = (unsigned)(b >> 32), lo = (unsigned)b;
+    const unsigned mhi = __reduce_min_sync(mask, hi);
+    const unsigned mlo = __reduce_min_sync(mask, hi == mhi ? lo : 0xffffffffu);
+    return __longlong_as_double((long long)(((unsigned long long)mhi << 32) | mlo));
 }
 template <int W>
 __device__ __forceinline__ double seg_max(double v) {
@@ -124,12 +136,11 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
     uint32_t ncoll = 0, m = 1;
     const ClassDesc *C = nullptr;
     TopoRef TR = {0, 0, 0, 0};
-    uint64_t H = 0;
     uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
     bool bon = false;
     double bstart = 0.0, cbusy = 0.0;
     uint32_t cur = 0;
-    bool running = false, tree_cur = false, tree_algo = false, ring_fast = false;
+    bool running = false, tree_cur = false, tree_algo = false, ring_fast = false, ring_uni = false;
     int K = 0;
     double cS = 0.0, chunk = 0.0;
     // ---- per-lane state ----
@@ -154,23 +165,25 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
     SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
     SI.ent_off = SI.send_off = SI.recv_off = 0;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
-    uint64_t acc = 0, alg = 0;
-    uint32_t nev = 0;
+    uint64_t acc = 0, alg = 0;   // acc: this lane's part of the order hash (R19)
+    uint64_t tmix = 0;           // mix64(bits(t)) of the current instant
+    bool nev = false;            // this lane recorded an event at the current instant
 
 #define EV(kind, code)                                                  \
     do {                                                                \
-        acc += mix64(((uint64_t)(kind) << 60) | (uint64_t)(code));      \
-        nev++;                                                          \
+        acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code))); \
+        nev = true;                                                     \
     } while (0)
 
     for (;;) {
         // ------------------------------ refill ------------------------------
         const bool need = !have && !exhausted;
-        uint32_t it = 0;
-        if (need && li == 0) it = atomicAdd(a.counter, 1u);
-        it = __shfl_sync(FULL, it, sbase);
         bool fresh = false, rbad = false, rlong = false;
-        if (need) {
+        if (__any_sync(FULL, need)) {
+          uint32_t it = 0;
+          if (need && li == 0) it = atomicAdd(a.counter, 1u);
+          it = __shfl_sync(FULL, it, sbase);
+          if (need) {
             if (it >= a.n_work) {
                 exhausted = true;
             } else {
@@ -190,7 +203,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 m = C->m;
                 tree_algo = C->algo == TRIOSIM_ALGO_TREE;
                 t = 0.0;
-                H = 0xcbf29ce484222325ull;
+                tmix = mix64(0ull);
                 ninst = nwf = nrounds = maxact = 0;
                 bon = false;
                 bstart = cbusy = 0.0;
@@ -207,7 +220,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 fst = FS_NONE;
                 sq = dcnt = 0;
                 acc = alg = 0;
-                nev = 0;
+                nev = false;
                 if (used) {
                     gpu = a.ro[TR.ro_off + li];
                     if constexpr (COLL) {
@@ -254,9 +267,17 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                     }
                 }
             }
+          }
+          if constexpr (COLL) {
+              // link-disjoint ring whose lanes all see the same min-hop bandwidth: every
+              // water-filling call is a single round at that rate (R14)
+              const double lo = seg_min_shfl<W>(used ? rbw : dinf());
+              const double hi = seg_max<W>(used ? rbw : 0.0);
+              if (fresh) ring_uni = ring_fast && lo == hi;
+          }
         }
         if (__all_sync(FULL, !have)) break;
-        {
+        if (__any_sync(FULL, fresh && (rbad || rlong))) {
             // a needed (src, dst) pair without a path (R3) / beyond this kernel's hop limit
             const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
             const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
@@ -333,8 +354,11 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                     // (d) collective progress: done on this GPU, finish, start (R10)
                     const int pred = (li + p - 1) % p;
                     const int Dp = __shfl_sync(FULL, D, sbase + pred);
-                    const unsigned upm = (__ballot_sync(FULL, upd) & smask) >> sbase;
-                    const unsigned dnm = (__ballot_sync(FULL, dnd) & smask) >> sbase;
+                    unsigned upm = 0, dnm = 0;
+                    if (__any_sync(FULL, tree_cur)) {
+                        upm = (__ballot_sync(FULL, upd) & smask) >> sbase;
+                        dnm = (__ballot_sync(FULL, dnd) & smask) >> sbase;
+                    }
                     const int c1 = 2 * li + 1, c2 = 2 * li + 2;
                     if (used && running && !ldone) {
                         bool dn;
@@ -536,25 +560,31 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 t_upd = t;
                 alg += 4;
             }
-            if (gen) {
-                alg += flen;
+            const bool anygen = __any_sync(FULL, gen);
+            if (anygen) {
+                if (gen) {
+                    alg += flen;
 #pragma unroll
-                for (int h = 0; h < MAX_HOPS; h++) if (h < flen) ln[hop(hl, h)] = 0;
-            }
-            __syncwarp();
-            if (gen) {
+                    for (int h = 0; h < MAX_HOPS; h++) if (h < flen) ln[hop(hl, h)] = 0;
+                }
+                __syncwarp();
+                if (gen) {
 #pragma unroll
-                for (int h = 0; h < MAX_HOPS; h++)
-                    if (h < flen) {
-                        const int e = hop(hl, h);
-                        atomicAdd(&ln[e], 1);
-                        lres[e] = a.link_bw[TR.link_off + e] * bws;
-                    }
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if (h < flen) {
+                            const int e = hop(hl, h);
+                            atomicAdd(&ln[e], 1);
+                            lres[e] = a.link_bw[TR.link_off + e] * bws;
+                        }
+                }
+                __syncwarp();
             }
-            __syncwarp();
             if (act && fast) rate = rbw;
-            bool unf = act;
-            uint32_t rounds = 0;
+            // uniform link-disjoint ring: one round at rate rbw, nothing to reduce
+            const bool uni = fast && ring_uni;
+            bool unf = act && !uni;
+            const bool segany = (__ballot_sync(FULL, act) & smask) != 0;
+            uint32_t rounds = (uni && segany) ? 1u : 0u;
             while (__any_sync(FULL, unf)) {
                 const bool segact = (__ballot_sync(FULL, unf) & smask) != 0;
                 double my = dinf();
@@ -572,7 +602,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                         alg += 2 * flen;
                     }
                 }
-                const double s = seg_min<W>(my);
+                const double s = TS_SEGMIN_REDUX ? seg_min_redux(my, smask) : seg_min_shfl<W>(my);
                 const bool inF = unf && my == s;
                 unsigned own = 0;
                 if (inF && !fast) {
@@ -581,7 +611,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                     for (int h = 0; h < MAX_HOPS; h++)
                         if (h < flen && atomicAdd(&lk[hop(hl, h)], 1) == 0) own |= 1u << h;
                 }
-                __syncwarp();
+                if (anygen) __syncwarp();
                 if (inF && !fast) {
 #pragma unroll
                     for (int h = 0; h < MAX_HOPS; h++)
@@ -595,11 +625,11 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                             alg += 3;
                         }
                 }
-                __syncwarp();
+                if (anygen) __syncwarp();
                 if (segact) rounds++;
                 unf = unf && !inF;
             }
-            const uint32_t nact = __popc(__ballot_sync(FULL, act) & smask);
+            const uint32_t nact = __popc(__ballot_sync(FULL, act) & smask);  // (all lanes vote)
             if (segdirty) {
                 nwf++;
                 nrounds += rounds;
@@ -615,17 +645,9 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
         }
 
         // ------------------------------ end of instant ------------------------------
-        if (__ballot_sync(FULL, nev > 0) & smask) {
-            const unsigned long long acc_s = seg_sum_u64<W>(acc);
-            if (have) {
-                H = mix64(mix64(H ^ (uint64_t)__double_as_longlong(t)) ^ acc_s);   // R19
-                ninst++;
-            }
-        } else {
-            seg_sum_u64<W>(0ull);  // keep every lane on the same shuffles
-        }
-        acc = 0;
-        nev = 0;
+        const bool any_ev = (__ballot_sync(FULL, nev) & smask) != 0;
+        if (have && any_ev) ninst++;
+        nev = false;
         const bool infl = (__ballot_sync(FULL, used && fst != FS_NONE) & smask) != 0;
         if (have) {
             if (infl && !bon) { bon = true; bstart = t; }
@@ -641,13 +663,14 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
             if (fst == FS_LAT && t_act < cand) cand = t_act;
             if (fst == FS_ACT && t_drain < cand) cand = t_drain;
         }
-        const double tn = seg_min<W>(cand);
+        const double tn = TS_SEGMIN_REDUX ? seg_min_redux(cand, smask) : seg_min_shfl<W>(cand);
         const bool stuck = have && !fin && !(tn < dinf());
         if (__any_sync(FULL, fin || stuck)) {
             const double bmax = seg_max<W>(used ? busy : 0.0);
             const uint32_t ntk = seg_sum_u32<W>(ntask);
             const uint32_t nfl = seg_sum_u32<W>(nflow);
             const unsigned long long alg_s = seg_sum_u64<W>(alg);
+            const unsigned long long H = seg_sum_u64<W>(acc);
             if ((fin || stuck) && li == 0) {
                 triosim_result r;
                 r.iter_time_s = fin ? t : 0.0;
@@ -670,7 +693,10 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
             }
             if (fin || stuck) have = used = false;
         }
-        if (have) t = tn;
+        if (have) {
+            t = tn;
+            tmix = mix64((uint64_t)__double_as_longlong(t));
+        }
     }
 #undef EV
 }

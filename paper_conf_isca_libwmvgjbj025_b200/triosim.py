@@ -15,7 +15,7 @@ import numpy as np
 from . import workloads as W
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libtriosim.so")
+LIB_PATH = os.environ.get("TRIOSIM_LIB", os.path.join(HERE, "libtriosim.so"))
 
 EXPORTS = ["triosim_create", "triosim_destroy", "triosim_last_error", "triosim_load_trace", "triosim_build_sweep",
            "triosim_simulate_batch", "triosim_results", "triosim_release", "triosim_launch_counts",
