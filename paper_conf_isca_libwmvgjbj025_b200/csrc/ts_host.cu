@@ -159,7 +159,7 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
             triosim_destroy(ctx);
             return TRIOSIM_ECUDA;
         }
-        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i / 2], i % 2);
+        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i / N_MODES], i % N_MODES);
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
         triosim_destroy(ctx);
@@ -521,7 +521,8 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         pd.idx = (uint32_t)i;
         pd.pad = 0;
         S->width[i] = W;
-        S->mode[i] = mode;
+        // K3 variant: tree-capable collectives only for classes that use the tree algorithm
+        S->mode[i] = (mode == MODE_COLL && pt.coll_algo == TRIOSIM_ALGO_TREE) ? MODE_TREE : mode;
         double cost;
         if (mode == MODE_COLL) {
             double ncol = pt.strategy == TRIOSIM_TP ? n_tp_coll[pt.tp_mode == TRIOSIM_TP_PAPER ? 0 : 1]
@@ -628,7 +629,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         if (S->cost[a] != S->cost[b]) return S->cost[a] > S->cost[b];
         return pdesc[a].cls < pdesc[b].cls;
     });
-    for (uint64_t i : order) S->work[2 * w_index(S->width[i]) + S->mode[i]].push_back((uint32_t)i);
+    for (uint64_t i : order) S->work[N_MODES * w_index(S->width[i]) + S->mode[i]].push_back((uint32_t)i);
     for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
         CK(S->d_work_tmp[w].alloc(S->work[w].size()));
@@ -692,7 +693,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
             wl = S.d_work_tmp[w].p;
         }
         if (n == 0) continue;
-        const int W = W_OF[w / 2], mode = w % 2;
+        const int W = W_OF[w / N_MODES], mode = w % N_MODES;
         K3Args a;
         std::memset(&a, 0, sizeof a);
         a.pts = S.d_pts.p; a.work = wl; a.n_work = n; a.counter = S.d_counter.p + w;

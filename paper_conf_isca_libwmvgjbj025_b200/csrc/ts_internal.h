@@ -7,7 +7,7 @@
 
 namespace ts {
 
-enum { MODE_COLL = 0, MODE_PIPE = 1 };
+enum { MODE_COLL = 0, MODE_PIPE = 1, MODE_TREE = 2 };  // K3 variants: ring-only collectives, GPipe, tree-capable collectives
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 constexpr int MAX_HOPS = 8;
@@ -139,6 +139,7 @@ cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
 int k3_max_blocks_per_sm(int W, int mode);
 constexpr int N_WIDTHS = 5;             // W = 2, 4, 8, 16, 32
-constexpr int N_GROUPS = 2 * N_WIDTHS;  // (width, mode) launch groups
+constexpr int N_MODES = 3;
+constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 
 }  // namespace ts

@@ -112,7 +112,8 @@ template <int W, int MODE>
 __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
     constexpr int NSEG = 32 / W;
     constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
-    constexpr bool COLL = MODE == MODE_COLL;
+    constexpr bool COLL = MODE != MODE_PIPE;   // DP / DDP / TP collectives
+    constexpr bool TREE = MODE == MODE_TREE;   // ... some of which may be tree AllReduces
     __shared__ double s_res[K3_WARPS][NSEG * LMAX];
     __shared__ int s_n[K3_WARPS][NSEG * LMAX];
     __shared__ int s_k[K3_WARPS][NSEG * LMAX];
@@ -133,6 +134,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
     uint32_t pidx = 0;
     double t = 0.0, bws = 1.0, lats = 1.0;
     int p = 1;
+    int pred = 0;   // ring predecessor lane of this lane (li - 1 mod p)
     uint32_t ncoll = 0, m = 1;
     const ClassDesc *C = nullptr;
     TopoRef TR = {0, 0, 0, 0};
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 }
                 ncoll = C->n_coll;
                 m = C->m;
-                tree_algo = C->algo == TRIOSIM_ALGO_TREE;
+                tree_algo = TREE && C->algo == TRIOSIM_ALGO_TREE;
                 t = 0.0;
                 tmix = mix64(0ull);
                 ninst = nwf = nrounds = maxact = 0;
@@ -210,6 +212,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 cur = 0;
                 running = false;
                 used = li < p;
+                pred = sbase + (li == 0 ? p - 1 : li - 1);
                 pos = run_start = run_end = 0;
                 cst = CS_IDLE;
                 t_end = busy = 0.0;
@@ -341,7 +344,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 if (delivered) {
                     nflow++;
                     if constexpr (COLL) {
-                        if (tree_cur) {
+                        if (TREE && tree_cur) {
                             if (fup) upd = true; else dnd = true;
                         } else {
                             D++;
@@ -352,17 +355,18 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                 }
                 if constexpr (COLL) {
                     // (d) collective progress: done on this GPU, finish, start (R10)
-                    const int pred = (li + p - 1) % p;
-                    const int Dp = __shfl_sync(FULL, D, sbase + pred);
+                    const int Dp = __shfl_sync(FULL, D, pred);
                     unsigned upm = 0, dnm = 0;
-                    if (__any_sync(FULL, tree_cur)) {
-                        upm = (__ballot_sync(FULL, upd) & smask) >> sbase;
-                        dnm = (__ballot_sync(FULL, dnd) & smask) >> sbase;
+                    if constexpr (TREE) {
+                        if (__any_sync(FULL, tree_cur)) {
+                            upm = (__ballot_sync(FULL, upd) & smask) >> sbase;
+                            dnm = (__ballot_sync(FULL, dnd) & smask) >> sbase;
+                        }
                     }
                     const int c1 = 2 * li + 1, c2 = 2 * li + 2;
                     if (used && running && !ldone) {
                         bool dn;
-                        if (!tree_cur) {
+                        if (!TREE || !tree_cur) {
                             dn = D == K && Dp == K;
                         } else {
                             const bool ku = (c1 >= p || ((upm >> c1) & 1u)) && (c2 >= p || ((upm >> c2) & 1u));
@@ -395,7 +399,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                     }
                     if (used && running && fst == FS_NONE) {
                         bool rel = false;
-                        if (!tree_cur) {
+                        if (!TREE || !tree_cur) {
                             if (D < K && (D == 0 || Dp >= D)) {
                                 // ring step (i, k = D): m_i -> m_{i+1}, S/p bytes (Q21)
                                 rel = true;
@@ -406,7 +410,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
                                 alg += 1;
                                 fcode = ((uint64_t)cur << 32) | ((uint64_t)D << 16) | (uint64_t)li;
                             }
-                        } else if (li >= 1) {
+                        } else if (TREE && li >= 1) {
                             const unsigned um = started ? 0u : upm, dm = started ? 0u : dnm;
                             const bool ku = (c1 >= p || ((um >> c1) & 1u)) && (c2 >= p || ((um >> c2) & 1u));
                             const int par_i = (li - 1) / 2;
@@ -707,33 +711,38 @@ static cudaError_t launch_wm(const K3Args &a, int grid, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s) {
-#define CASE(w)                                                                                  \
-    case w:                                                                                      \
-        return mode == MODE_COLL ? launch_wm<w, MODE_COLL>(a, grid, s) : launch_wm<w, MODE_PIPE>(a, grid, s);
-    switch (W) {
-        CASE(2) CASE(4) CASE(8) CASE(16) CASE(32)
-    default:
-        return cudaErrorInvalidValue;
+template <int W>
+static cudaError_t launch_w(int mode, const K3Args &a, int grid, cudaStream_t s) {
+    switch (mode) {
+    case MODE_COLL: return launch_wm<W, MODE_COLL>(a, grid, s);
+    case MODE_TREE: return launch_wm<W, MODE_TREE>(a, grid, s);
+    default: return launch_wm<W, MODE_PIPE>(a, grid, s);
     }
-#undef CASE
+}
+
+cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s) {
+    switch (W) {
+    case 2: return launch_w<2>(mode, a, grid, s);
+    case 4: return launch_w<4>(mode, a, grid, s);
+    case 8: return launch_w<8>(mode, a, grid, s);
+    case 16: return launch_w<16>(mode, a, grid, s);
+    case 32: return launch_w<32>(mode, a, grid, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+template <int W>
+static int occ_w(int mode) {
+    int nb = 0;
+    if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL>, K3_THREADS, 0);
+    else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE>, K3_THREADS, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE>, K3_THREADS, 0);
+    return nb;
 }
 
 int k3_max_blocks_per_sm(int W, int mode) {
-    int nb = 0;
-#define CASE(w)                                                                                          \
-    case w:                                                                                              \
-        if (mode == MODE_COLL)                                                                           \
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<w, MODE_COLL>, K3_THREADS, 0); \
-        else                                                                                             \
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<w, MODE_PIPE>, K3_THREADS, 0); \
-        break;
-    switch (W) {
-        CASE(2) CASE(4) CASE(8) CASE(16) CASE(32)
-    default:
-        break;
-    }
-#undef CASE
+    int nb = W == 2 ? occ_w<2>(mode) : W == 4 ? occ_w<4>(mode) : W == 8 ? occ_w<8>(mode)
+           : W == 16 ? occ_w<16>(mode) : occ_w<32>(mode);
     return nb > 0 ? nb : 1;
 }
 
