@@ -29,6 +29,8 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     return z ^ (z >> 31);
 }
+// per-event mix: one xorshift-multiply round (the per-instant time hash tmix is a full mix64)
+__device__ __forceinline__ uint64_t emix(uint64_t v) { return (v ^ (v >> 29)) * 0xbf58476d1ce4e5b9ull; }
 __device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
 
 #ifndef TS_SEGMIN_REDUX
@@ -108,8 +110,11 @@ __device__ __forceinline__ double load_route(const K3Args &a, const TopoRef &T, 
 }
 __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[h >> 1] >> (16 * (h & 1))) & 0xffff; }
 
+#ifndef TS_K3_MINB
+#define TS_K3_MINB 1
+#endif
 template <int W, int MODE>
-__global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
+__global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Args a) {
     constexpr int NSEG = 32 / W;
     constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
     constexpr bool COLL = MODE != MODE_PIPE;   // DP / DDP / TP collectives
@@ -173,7 +178,7 @@ __global__ void __launch_bounds__(K3_THREADS, 2) k3_timeline(const K3Args a) {
 
 #define EV(kind, code)                                                  \
     do {                                                                \
-        acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code))); \
+        acc += emix(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code))); \
         nev = true;                                                     \
     } while (0)
 
