@@ -283,21 +283,24 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
               const double hi = seg_max<W>(used ? rbw : 0.0);
               if (fresh) ring_uni = ring_fast && lo == hi;
           }
+          if (__any_sync(FULL, fresh && (rbad || rlong))) {
+              // a needed (src, dst) pair without a path (R3) / beyond this kernel's hop limit
+              const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
+              const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
+              if (fresh && (bad || lng)) {
+                  if (li == 0) {
+                      triosim_result r = {};
+                      r.status = bad ? TRIOSIM_PT_NO_ROUTE : TRIOSIM_PT_TOO_LARGE;
+                      a.out[pidx] = r;
+                  }
+                  have = used = false;
+              }
+          }
+
         }
-        if (__all_sync(FULL, !have)) break;
-        if (__any_sync(FULL, fresh && (rbad || rlong))) {
-            // a needed (src, dst) pair without a path (R3) / beyond this kernel's hop limit
-            const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
-            const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
-            if (fresh && (bad || lng)) {
-                if (li == 0) {
-                    triosim_result r = {};
-                    r.status = bad ? TRIOSIM_PT_NO_ROUTE : TRIOSIM_PT_TOO_LARGE;
-                    a.out[pidx] = r;
-                }
-                have = used = false;
-            }
-        }
+        // done when every segment has drained the work list (a segment whose point was just
+        // rejected refills on the next iteration)
+        if (__all_sync(FULL, !have && exhausted)) break;
 
         // ------------------------------ one instant at time t ------------------------------
         bool dirty = false;
@@ -556,8 +559,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 
             // (f) bandwidth re-allocation of every in-transit flow: max-min fair
             //     progressive filling (R14, Q18)
-            const bool segdirty = (__ballot_sync(FULL, dirty) & smask) != 0;
-            if (!__any_sync(FULL, segdirty)) break;
+            const unsigned dball = __ballot_sync(FULL, dirty);
+            if (!dball) break;
+            const bool segdirty = (dball & smask) != 0;
             dirty = false;
             const bool act = segdirty && used && fst == FS_ACT;
             // ring_fast is segment-uniform and only set while a ring collective runs (tree_cur off)
