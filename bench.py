@@ -205,6 +205,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--shard", action="store_true",
+                    help="strong scaling: deal one sweep to the ranks by cost instead of a full sweep per rank")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -212,7 +214,7 @@ def main():
 
     import torch
     import torch.distributed as dist
-    from paper_conf_isca_libwmvgjbj025_b200 import triosim
+    from paper_conf_isca_libwmvgjbj025_b200 import dist as D, triosim
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -222,14 +224,21 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     sw = CONFIGS[args.config]()
+    n_sweep = len(sw.points)
+    if args.shard and world > 1:
+        tr = sw.trace
+        wg = tr.tensors[tr.tensors["category"] == W.CAT_WGRAD]
+        costs = D.point_cost(sw.points, len(tr.ops), len(wg), int(wg["bytes_b0"].sum()))
+        maxc = max(D.shard_sizes(n_sweep, world, costs))
+        sw = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[D.shard_points(costs, world, rank)], sw.plans)
     n = len(sw.points)
+    maxc = maxc if (args.shard and world > 1) else n
     ctx = triosim.Context(local)
     tid = ctx.triosim_load_trace(sw.trace)
     sid = ctx.triosim_build_sweep(tid, sw.topos, sw.points, sw.plans or None)
     stream = torch.cuda.Stream()
     rec = W.RESULT_DTYPE.itemsize
-    res_local = torch.empty(n * rec, dtype=torch.uint8, device="cuda")
-    res_all = torch.empty(n * rec * world, dtype=torch.uint8, device="cuda") if world > 1 else None
+    res_local = torch.zeros(n * rec, dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
 
     def step():
@@ -237,7 +246,7 @@ def main():
         ctx.triosim_results(sid, 0, n, device_ptr=res_local.data_ptr(), stream=stream.cuda_stream)
         if world > 1:
             with torch.cuda.stream(stream):
-                dist.all_gather_into_tensor(res_all, res_local)
+                D.gather_records(res_local, world, maxc)   # one NCCL all-gather of the records
 
     for _ in range(args.warmup):
         step()
@@ -268,7 +277,8 @@ def main():
         t = torch.tensor([ms], device="cuda", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-    value = n * world / (ms / 1e3)
+    total_points = n_sweep if (args.shard and world > 1) else n * world
+    value = total_points / (ms / 1e3)
     gpu_launches = sum(k1) - sum(k0)
     res = ctx.triosim_results(sid, 0, n)
     n_ok = int((res["status"] == 0).sum())
@@ -296,6 +306,7 @@ def main():
     h2d = (sw.trace.ops.nbytes + sw.trace.tensors.nbytes + sw.trace.io.nbytes + sw.points.nbytes +
            sum(t.links.nbytes + t.ring_order.nbytes for t in sw.topos))
     e2e_ms = float(np.max(e2e_t)) * 1e3 if e2e_t else float("nan")
+    e2e_points = total_points
     if world > 1:
         t = torch.tensor([e2e_ms], device="cuda", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -316,12 +327,15 @@ def main():
         alg_b = algorithmic_bytes(sw)
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "scaling": "strong" if (args.shard and world > 1) else "weak",
             "config": {"workload": WORKLOAD[args.config], "points": n, "points_ok": n_ok,
                        "trace": sw.trace.name, "ops": int(len(sw.trace.ops)),
-                       "parallelism": f"points sharded: each of {world} rank(s) simulates a full sweep; "
-                                      "results all-gathered over NCCL",
+                       "parallelism": (f"one sweep dealt to {world} ranks by cost; records all-gathered over NCCL"
+                                       if (args.shard and world > 1) else
+                                       f"each of {world} rank(s) simulates a full sweep (weak scaling); "
+                                       "records all-gathered over NCCL"),
                        "l2": "flushed (256 MB write) before every timed step"},
             "roofline": {"bound": "alu", "kernel": "k3_timeline", "achieved": round(achieved / 1e12, 6),
                          "peak": round(peak_ops / 1e12, 3), "unit": "TFLOP/s (fp64, non-tensor)",
@@ -333,7 +347,7 @@ def main():
                              "peak": pk.get("hbm_gbs"), "unit": "GB/s",
                              "frac": round(alg_b / (k3 / 1e3) / 1e9 / float(pk.get("hbm_gbs", 6650.0)), 7),
                              "algorithmic_bytes_per_launch": int(alg_b), "peak_source": src},
-            "e2e": {"value": round(n * world / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+            "e2e": {"value": round(e2e_points / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(n * rec), "ms_per_step": round(e2e_ms, 3)},
             "gpu_launches": int(gpu_launches),
             "clocks": clk.summary(),

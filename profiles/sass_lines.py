@@ -15,10 +15,16 @@ import sys
 import tempfile
 
 
-def main(rep, so, fn, top=40):
+def main(rep, so, fn, top=40, section=None):
     sass = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
                           capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(sass)))
+    allrows = list(csv.reader(io.StringIO(sass)))
+    starts = [i for i, r in enumerate(allrows) if r and r[0] == "Kernel Name"] + [len(allrows)]
+    rows = None
+    for a, b in zip(starts, starts[1:]):
+        if section is None or section in allrows[a][1]:
+            rows = allrows[a:b]
+            break
     hdr = rows[1]
     ie, ss = hdr.index("Instructions Executed"), hdr.index("Warp Stall Sampling (All Samples)")
     counts = [(int(r[ie] or 0), int(r[ss] or 0)) for r in rows[2:] if len(r) > ie]
@@ -53,4 +59,5 @@ def main(rep, so, fn, top=40):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2], sys.argv[3], int(sys.argv[4]) if len(sys.argv) > 4 else 40)
+    main(sys.argv[1], sys.argv[2], sys.argv[3], int(sys.argv[4]) if len(sys.argv) > 4 else 40,
+         sys.argv[5] if len(sys.argv) > 5 else None)
