@@ -125,7 +125,7 @@ typedef struct {
 #define TRIOSIM_DDP 1     /* DistributedDataParallel: AllReduce overlapped with backward */
 #define TRIOSIM_TP 2      /* tensor parallel */
 #define TRIOSIM_PP 3      /* GPipe pipeline parallel */
-#define TRIOSIM_HYBRID 4  /* reserved (DP x TP x PP): reported as PT_BAD_CONFIG in this revision */
+#define TRIOSIM_HYBRID 4  /* DP x TP x PP (extension, R9) */
 #define TRIOSIM_TP_PAPER 0
 #define TRIOSIM_TP_MEGATRON 1
 #define TRIOSIM_ALGO_RING 0

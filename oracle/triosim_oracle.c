@@ -271,8 +271,8 @@ static int add_flow(Graph *G, int src, int dst, double bytes, uint64_t code, int
     n.type = N_FLOW; n.src = src; n.dst = dst; n.bytes = bytes; n.code = code; n.flags = flags;
     return g_add(G, n);
 }
-static uint64_t coll_flow_code(int c, int step, int member) {
-    return ((uint64_t)(uint32_t)c << 32) | ((uint64_t)(uint32_t)step << 16) | (uint64_t)(uint32_t)member;
+static uint64_t coll_flow_code(uint64_t c, int step, int member) {
+    return (c << 32) | ((uint64_t)(uint32_t)step << 16) | (uint64_t)(uint32_t)member;
 }
 static uint64_t p2p_flow_code(uint32_t x, int j, int dst) {
     return (1ull << 59) | ((uint64_t)x << 32) | ((uint64_t)(uint32_t)j << 16) | (uint64_t)(uint32_t)dst;
@@ -286,9 +286,9 @@ static uint64_t p2p_flow_code(uint32_t x, int j, int dst) {
  * per (GPU, group), reading Q24) or NULL.  Writes done[i] = barrier "this
  * collective is done on member i" (last flow touching it delivered).
  */
-static int build_collective(Graph *G, const int *members, int p, int kind, int algo, double S,
-                            const int *trig, const int *prev_done, int *done) {
-    int c = G->n_coll++;
+static int build_collective_code(Graph *G, uint64_t c, const int *members, int p, int kind, int algo, double S,
+                                 const int *trig, const int *prev_done, int *done) {
+    G->n_coll++;
     G->coll_payload = G->coll_payload + S;
     int sb = add_barrier(G, NF_COLL_START, (uint64_t)c);
     if (sb < 0) return -1;
@@ -360,6 +360,12 @@ static int build_collective(Graph *G, const int *members, int p, int kind, int a
     }
     iv_free(&fl);
     return 0;
+}
+
+/* collectives of DP / DDP / TP: one group, numbered in creation order */
+static int build_collective(Graph *G, const int *members, int p, int kind, int algo, double S,
+                            const int *trig, const int *prev_done, int *done) {
+    return build_collective_code(G, (uint64_t)G->n_coll, members, p, kind, algo, S, trig, prev_done, done);
 }
 
 /* ------------------------------------------------------------------ */
@@ -744,6 +750,251 @@ static int expand_pp(const Trace *T, const OPoint *pt, const int *ro, const uint
 }
 
 /* ------------------------------------------------------------------ */
+/* Extrapolation: HYBRID DP x TP x PP (R9; "often combined as      */
+/* hybrid parallelism"; Table 1 P:102 -- an extension, reading Q26)     */
+/* ------------------------------------------------------------------ */
+/* tiny open-addressing map uint64 -> int (plain, test infrastructure) */
+typedef struct { uint64_t *k; int *v; long cap, n; } HMap;
+static int hm_init(HMap *h, long cap) {
+    h->cap = 64; while (h->cap < 2 * cap + 64) h->cap *= 2; h->n = 0;
+    h->k = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)h->cap); h->v = (int *)malloc(sizeof(int) * (size_t)h->cap);
+    if (!h->k || !h->v) return -1;
+    for (long i = 0; i < h->cap; i++) h->k[i] = ~0ull;
+    return 0;
+}
+static void hm_free(HMap *h) { free(h->k); free(h->v); h->k = NULL; h->v = NULL; }
+static int hm_put(HMap *h, uint64_t key, int val) {
+    if (2 * (h->n + 1) > h->cap) {
+        HMap g; if (hm_init(&g, h->cap)) return -1;
+        for (long i = 0; i < h->cap; i++) if (h->k[i] != ~0ull) hm_put(&g, h->k[i], h->v[i]);
+        hm_free(h); *h = g;
+    }
+    long i = (long)((key * 0x9e3779b97f4a7c15ull) >> 20) & (h->cap - 1);
+    while (h->k[i] != ~0ull && h->k[i] != key) i = (i + 1) & (h->cap - 1);
+    if (h->k[i] == ~0ull) h->n++;
+    h->k[i] = key; h->v[i] = val;
+    return 0;
+}
+static int hm_get(const HMap *h, uint64_t key) {
+    long i = (long)((key * 0x9e3779b97f4a7c15ull) >> 20) & (h->cap - 1);
+    while (h->k[i] != ~0ull) { if (h->k[i] == key) return h->v[i]; i = (i + 1) & (h->cap - 1); }
+    return -1;
+}
+
+/* R7's TP collective rule for one output of one op (-1 = none) */
+static int tp_kind(const Trace *T, const OOp *op, uint32_t x, int tp_mode) {
+    if (tp_mode == TPM_PAPER) {
+        if ((op->tp_role & ROLE_GATHER) && op->phase == PH_FWD) return CK_AG;
+        if ((op->tp_role & ROLE_GATHER) && op->phase == PH_BWD && T->ts[x].category == CAT_AGRAD) return CK_AR;
+    } else {
+        if ((op->tp_role & 3) == ROLE_ROW && op->phase == PH_FWD) return CK_AR;
+        if ((op->tp_role & 3) == ROLE_COL && op->phase == PH_BWD && T->ts[x].category == CAT_AGRAD) return CK_AR;
+    }
+    return -1;
+}
+
+static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const uint32_t *first_layer, Graph *G) {
+    const int dp = pt->dp, tp = pt->tp, S = pt->pp, m = (int)pt->microbatches;
+    const uint32_t N = T->n_ops, L = T->n_layers;
+    const double r_b = (double)(pt->global_batch / ((uint32_t)dp * (uint32_t)m)) / (double)T->b0;
+    const int R = dp * S * tp;
+    int rc = -1;
+    int *stage_of_layer = (int *)malloc(sizeof(int) * L);
+    uint64_t *readers = (uint64_t *)calloc(T->n_ts ? T->n_ts : 1, sizeof(uint64_t));
+    int **pop = (int **)calloc((size_t)S, sizeof(int *)), **pmb = (int **)calloc((size_t)S, sizeof(int *));
+    long *plen = (long *)calloc((size_t)S, sizeof(long));
+    int **task = (int **)calloc((size_t)R, sizeof(int *));
+    int *members = (int *)malloc(sizeof(int) * (size_t)(dp > tp ? dp : tp) + sizeof(int));
+    int *trig = (int *)malloc(sizeof(int) * (size_t)(dp > tp ? dp : tp) + sizeof(int));
+    int *prev = (int *)malloc(sizeof(int) * (size_t)(dp > tp ? dp : tp) + sizeof(int));
+    int *done = (int *)malloc(sizeof(int) * (size_t)(dp > tp ? dp : tp) + sizeof(int));
+    IVec dtab = {0};          /* done barriers of TP collectives, tp per collective */
+    HMap tpc = {0}, p2p = {0};
+    if (!stage_of_layer || !readers || !pop || !pmb || !plen || !task || !members || !trig || !prev || !done) goto out;
+    if (hm_init(&tpc, 1024) || hm_init(&p2p, 1024)) goto out;
+    for (uint32_t l = 0, s = 0; l < L; l++) {
+        while ((int)s + 1 < S && first_layer[s + 1] <= l) s++;
+        stage_of_layer[l] = (int)s;
+    }
+    for (uint32_t o = 0; o < N; o++) {
+        const OOp *op = &T->ops[o];
+        for (uint32_t k = 0; k < op->n_in; k++) readers[T->io[op->io_off + k]] |= 1ull << stage_of_layer[op->layer];
+    }
+    /* the GPipe program of each stage (R8): FWD of 0..m-1, BWD of m-1..0, OPT once */
+    for (int s = 0; s < S; s++) {
+        pop[s] = (int *)malloc(sizeof(int) * ((size_t)N * (size_t)m + 1));
+        pmb[s] = (int *)malloc(sizeof(int) * ((size_t)N * (size_t)m + 1));
+        if (!pop[s] || !pmb[s]) goto out;
+        long np = 0;
+        for (int j = 0; j < m; j++)
+            for (uint32_t o = 0; o < N; o++)
+                if (T->ops[o].phase == PH_FWD && stage_of_layer[T->ops[o].layer] == s) { pop[s][np] = (int)o; pmb[s][np++] = j; }
+        for (int j = m - 1; j >= 0; j--)
+            for (uint32_t o = 0; o < N; o++)
+                if (T->ops[o].phase == PH_BWD && stage_of_layer[T->ops[o].layer] == s) { pop[s][np] = (int)o; pmb[s][np++] = j; }
+        for (uint32_t o = 0; o < N; o++)
+            if (T->ops[o].phase == PH_OPT && stage_of_layer[T->ops[o].layer] == s) { pop[s][np] = (int)o; pmb[s][np++] = 0; }
+        plen[s] = np;
+    }
+    /* rank r = (d*pp + s)*tp + t on GPU ring_order[r] (TP innermost) */
+    for (int r = 0; r < R; r++) {
+        const int s = (r / tp) % S;
+        task[r] = (int *)malloc(sizeof(int) * ((size_t)plen[s] + 1));
+        if (!task[r]) goto out;
+        for (long q = 0; q < plen[s]; q++)
+            task[r][q] = add_task(G, ro[r], q, op_time(T, (uint32_t)pop[s][q], r_b, tp, pt->tp_mode));
+    }
+    /* TP collectives: per group (d, s), one per (op, output, micro-batch) instance in program order */
+    if (tp > 1) {
+        for (int d = 0; d < dp; d++)
+            for (int s = 0; s < S; s++) {
+                const uint64_t gid = (uint64_t)(d * S + s);
+                const int base = (d * S + s) * tp;
+                for (int t = 0; t < tp; t++) members[t] = ro[base + t];
+                int have_prev = 0;
+                uint64_t seq = 0;
+                for (long q = 0; q < plen[s]; q++) {
+                    const OOp *op = &T->ops[pop[s][q]];
+                    for (uint32_t k = 0; k < op->n_out; k++) {
+                        const uint32_t x = T->io[op->io_off + op->n_in + k];
+                        const int kind = tp_kind(T, op, x, pt->tp_mode);
+                        if (kind < 0) continue;
+                        double Sb = (double)T->ts[x].bytes_b0;      /* full tensor (Q8) */
+                        if (T->ts[x].batch_scaled) Sb = Sb * r_b;
+                        for (int t = 0; t < tp; t++) trig[t] = task[base + t][q];
+                        if (build_collective_code(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, Sb, trig,
+                                                  have_prev ? prev : NULL, done)) goto out;
+                        seq++;
+                        memcpy(prev, done, sizeof(int) * (size_t)tp);
+                        have_prev = 1;
+                        if (hm_put(&tpc, (gid << 40) | ((uint64_t)x << 16) | (uint64_t)pmb[s][q], (int)dtab.n)) goto out;
+                        for (int t = 0; t < tp; t++) iv_push(&dtab, done[t]);
+                    }
+                }
+            }
+        /* same-stage readers of a communicated tensor wait for it on their GPU */
+        for (int r = 0; r < R; r++) {
+            const int d = r / (S * tp), s = (r / tp) % S, t = r % tp;
+            const uint64_t gid = (uint64_t)(d * S + s);
+            for (long q = 0; q < plen[s]; q++) {
+                const OOp *op = &T->ops[pop[s][q]];
+                for (uint32_t k = 0; k < op->n_in; k++) {
+                    const uint32_t x = T->io[op->io_off + k];
+                    const int po = T->prod[x];
+                    if (po < 0 || stage_of_layer[T->ops[po].layer] != s) continue;
+                    const int jp = (T->ops[po].phase == PH_OPT || op->phase == PH_OPT) ? 0 : pmb[s][q];
+                    const int di = hm_get(&tpc, (gid << 40) | ((uint64_t)x << 16) | (uint64_t)jp);
+                    if (di >= 0) g_dep(G, task[r][q], dtab.v[di + t]);
+                }
+            }
+        }
+    }
+    /* P2P along each pipeline (d, t): push every produced tensor to each other reading stage,
+     * FIFO per sending GPU; a TP-communicated tensor leaves after its collective is done there */
+    for (int r = 0; r < R; r++) {
+        const int d = r / (S * tp), s = (r / tp) % S, t = r % tp;
+        const uint64_t gid = (uint64_t)(d * S + s), pipe = (uint64_t)(d * tp + t);
+        int prev_send = -1;
+        for (long q = 0; q < plen[s]; q++) {
+            const int o = pop[s][q], j = pmb[s][q];
+            const OOp *op = &T->ops[o];
+            for (uint32_t k = 0; k < op->n_out; k++) {
+                const uint32_t x = T->io[op->io_off + op->n_in + k];
+                for (int ds = 0; ds < S; ds++) {
+                    if (ds == s || !(readers[x] & (1ull << ds))) continue;
+                    const int dg = ro[(d * S + ds) * tp + t];
+                    const int f = add_flow(G, ro[r], dg, tensor_bytes(T, x, r_b, tp, pt->tp_mode),
+                                           p2p_flow_code(x, j, dg), NF_P2P);
+                    g_dep(G, f, task[r][q]);
+                    if (prev_send >= 0) g_dep(G, f, prev_send);
+                    if (tp > 1) {
+                        const int di = hm_get(&tpc, (gid << 40) | ((uint64_t)x << 16) | (uint64_t)j);
+                        if (di >= 0) g_dep(G, f, dtab.v[di + t]);
+                    }
+                    prev_send = f;
+                    if (hm_put(&p2p, (((pipe << 24) | x) << 22) | ((uint64_t)j << 6) | (uint64_t)ds, f)) goto out;
+                }
+            }
+        }
+    }
+    for (int r = 0; r < R; r++) {
+        const int d = r / (S * tp), s = (r / tp) % S, t = r % tp;
+        const uint64_t pipe = (uint64_t)(d * tp + t);
+        for (long q = 0; q < plen[s]; q++) {
+            const OOp *op = &T->ops[pop[s][q]];
+            for (uint32_t k = 0; k < op->n_in; k++) {
+                const uint32_t x = T->io[op->io_off + k];
+                const int po = T->prod[x];
+                if (po < 0 || stage_of_layer[T->ops[po].layer] == s) continue;
+                const int jp = (T->ops[po].phase == PH_OPT || op->phase == PH_OPT) ? 0 : pmb[s][q];
+                const int f = hm_get(&p2p, (((pipe << 24) | x) << 22) | ((uint64_t)jp << 6) | (uint64_t)s);
+                if (f < 0) goto out;
+                g_dep(G, task[r][q], f);
+            }
+        }
+    }
+    /* DP: per group (s, t), one AllReduce per bucket of the stage's weight gradients, triggered by
+     * micro-batch 0's producer (the last one GPipe's backward runs); OPT waits for the last one */
+    if (dp > 1) {
+        WEnt *w = (WEnt *)malloc(sizeof(WEnt) * (T->n_ts ? T->n_ts : 1));
+        if (!w) goto out;
+        for (int s = 0; s < S; s++) {
+            int nw = 0;
+            for (uint32_t x = 0; x < T->n_ts; x++)
+                if (T->ts[x].category == CAT_WGRAD && T->prod[x] >= 0 && T->ops[T->prod[x]].phase != PH_OPT &&
+                    stage_of_layer[T->ops[T->prod[x]].layer] == s) {
+                    w[nw].x = x; w[nw].prod = T->prod[x]; nw++;
+                }
+            qsort(w, (size_t)nw, sizeof(WEnt), cmp_went);
+            long first_opt = -1;
+            for (long q = 0; q < plen[s]; q++) if (T->ops[pop[s][q]].phase == PH_OPT) { first_opt = q; break; }
+            for (int t = 0; t < tp; t++) {
+                const uint64_t gid = (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + t);
+                for (int d = 0; d < dp; d++) members[d] = ro[(d * S + s) * tp + t];
+                int have_prev = 0;
+                uint64_t seq = 0;
+                int i = 0;
+                while (i < nw) {
+                    int j = i;
+                    uint64_t sum = 0;
+                    double Sb = 0.0;
+                    for (;;) {
+                        sum += T->ts[w[j].x].bytes_b0;
+                        Sb = Sb + tensor_bytes(T, w[j].x, r_b, tp, pt->tp_mode);
+                        j++;
+                        if (pt->bucket_bytes == 0 || sum >= pt->bucket_bytes || j == nw) break;
+                    }
+                    /* program position of (producer of the bucket's last gradient, micro-batch 0) */
+                    long qt = -1;
+                    for (long q = 0; q < plen[s]; q++)
+                        if (pop[s][q] == w[j - 1].prod && pmb[s][q] == 0) { qt = q; break; }
+                    if (qt < 0) { free(w); goto out; }
+                    for (int d = 0; d < dp; d++) trig[d] = task[(d * S + s) * tp + t][qt];
+                    if (build_collective_code(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, Sb, trig,
+                                              have_prev ? prev : NULL, done)) { free(w); goto out; }
+                    seq++;
+                    memcpy(prev, done, sizeof(int) * (size_t)dp);
+                    have_prev = 1;
+                    i = j;
+                }
+                if (have_prev && first_opt >= 0)
+                    for (int d = 0; d < dp; d++) g_dep(G, task[(d * S + s) * tp + t][first_opt], prev[d]);
+            }
+        }
+        free(w);
+    }
+    rc = 0;
+out:
+    free(stage_of_layer); free(readers);
+    if (pop) for (int s = 0; s < S; s++) { free(pop[s]); free(pmb[s]); }
+    free(pop); free(pmb); free(plen);
+    if (task) for (int r = 0; r < R; r++) free(task[r]);
+    free(task); free(members); free(trig); free(prev); free(done);
+    iv_free(&dtab); hm_free(&tpc); hm_free(&p2p);
+    return rc;
+}
+
+/* ------------------------------------------------------------------ */
 /* Water-filling (R14; "bandwidth sharing between streams",        */
 /* P:210 "allocate bandwidth for the links on the route", reading Q18:  */
 /* max-min fair progressive filling).                                   */
@@ -1118,8 +1369,16 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
         free(fl);
         break;
     }
+    case ST_HYBRID: {
+        uint32_t *fl = (uint32_t *)malloc(sizeof(uint32_t) * pt->pp);
+        if (have_plan) memcpy(fl, plan, sizeof(uint32_t) * pt->pp);
+        else if (auto_partition(T, pt->pp, fl)) { free(fl); free(ro); return -1; }
+        rc = expand_hybrid(T, pt, ro, fl, G);
+        free(fl);
+        break;
+    }
     default:
-        *status = PT_BAD_CONFIG; /* HYBRID: not built in this oracle revision */
+        *status = PT_BAD_CONFIG;
         break;
     }
     free(ro);

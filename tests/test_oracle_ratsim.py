@@ -18,6 +18,7 @@ STRATS = [
     ("tp_paper", lambda p: W.make_point(0, W.ST_TP, tp=p, B=4, tp_mode=W.TPM_PAPER)),
     ("tp_tree", lambda p: W.make_point(0, W.ST_TP, tp=p, B=4, algo=W.ALG_TREE)),
     ("pp", lambda p: W.make_point(0, W.ST_PP, pp=min(p, 3), m=2, B=4)),
+    ("hybrid", lambda p: W.make_point(0, W.ST_HYBRID, dp=2 if p >= 4 else 1, tp=2, pp=1, m=2, B=8)),
 ]
 
 
