@@ -7,7 +7,7 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
-SRC = [os.path.join(HERE, "csrc", f) for f in ("ts_host.cu", "ts_kernels.cu", "ts_k3.cu")]
+SRC = [os.path.join(HERE, "csrc", f) for f in ("ts_host.cu", "ts_kernels.cu", "ts_k3.cu", "ts_k3h.cu")]
 HDR = [os.path.join(HERE, "csrc", "ts_internal.h"), os.path.join(ROOT, "include", "triosim.h")]
 OUT = os.path.join(HERE, "libtriosim.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

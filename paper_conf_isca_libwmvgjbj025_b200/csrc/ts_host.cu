@@ -82,6 +82,11 @@ struct Sweep {
     DevBuf<StageEnt> d_ents;
     DevBuf<SendEnt> d_sends;
     DevBuf<RecvEnt> d_recvs;
+    DevBuf<HStage> d_hst;
+    DevBuf<HEnt> d_hents;
+    DevBuf<HSend> d_hsends;
+    std::vector<uint32_t> hyb_list;
+    DevBuf<uint32_t> d_hyb_list;
     DevBuf<TopoDev> d_topo;
     DevBuf<double> d_bw, d_lat;
     DevBuf<uint32_t> d_rt_off, d_ro;
@@ -159,7 +164,8 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
             triosim_destroy(ctx);
             return TRIOSIM_ECUDA;
         }
-        ctx->occ[i] = k3_max_blocks_per_sm(W_OF[i / N_MODES], i % N_MODES);
+        ctx->occ[i] = (i % N_MODES) == MODE_HYBRID ? k3h_max_blocks_per_sm(W_OF[i / N_MODES])
+                                                   : k3_max_blocks_per_sm(W_OF[i / N_MODES], i % N_MODES);
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
         triosim_destroy(ctx);
@@ -415,7 +421,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     S->cost.assign(n_pts, 0.0);
     S->mode.assign(n_pts, 0);
     std::vector<PointDesc> pdesc(n_pts);
-    std::map<std::tuple<int, int, int, int, int, uint64_t, int, int>, uint32_t> cls_of;
+    std::map<std::tuple<int, int, int, int, int, int, int, uint64_t, int, int>, uint32_t> cls_of;
     std::vector<uint32_t> plan_pool;
     const uint32_t N = (uint32_t)T.ops.size(), NT = (uint32_t)T.ts.size();
 
@@ -466,23 +472,26 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             if (!ok) { setst(TRIOSIM_PT_BAD_PLAN); continue; }
             plan_key = pt.stage_plan;
         }
-        if (pt.strategy == TRIOSIM_HYBRID) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
         // GPU kernel limits
-        const uint32_t lanes = pt.strategy == TRIOSIM_TP ? tpd : pt.strategy == TRIOSIM_PP ? pp : dp;
+        const uint32_t lanes = pt.strategy == TRIOSIM_TP ? tpd : pt.strategy == TRIOSIM_PP ? pp
+                             : pt.strategy == TRIOSIM_HYBRID ? dp * tpd * pp : dp;
         int W = 2;
         while (W < (int)lanes) W <<= 1;
         while (W <= 32 && (int)tp.n_links > std::max(8, 4 * W)) W <<= 1;
         if (W > 32) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
         // structural class
-        const int mode = pt.strategy == TRIOSIM_PP ? MODE_PIPE : MODE_COLL;
+        const bool hyb = pt.strategy == TRIOSIM_HYBRID;
+        const int mode = hyb ? MODE_HYBRID : pt.strategy == TRIOSIM_PP ? MODE_PIPE : MODE_COLL;
         uint32_t b_loc = pt.strategy == TRIOSIM_TP ? pt.global_batch
-                       : pt.strategy == TRIOSIM_PP ? pt.global_batch / mb : pt.global_batch / dp;
-        int key_mode = pt.strategy == TRIOSIM_TP ? pt.tp_mode : 0;
-        int key_algo = mode == MODE_COLL ? pt.coll_algo : 0;
-        uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP) ? pt.bucket_bytes : 0;
-        int key_m = mode == MODE_PIPE ? (int)mb : 0;
-        auto key = std::make_tuple((int)pt.strategy, (int)lanes, (int)b_loc, key_mode, key_algo, key_bucket, key_m,
-                                   mode == MODE_PIPE ? plan_key : -2);
+                       : pt.strategy == TRIOSIM_PP ? pt.global_batch / mb
+                       : hyb ? pt.global_batch / (dp * mb) : pt.global_batch / dp;
+        int key_mode = (pt.strategy == TRIOSIM_TP || hyb) ? pt.tp_mode : 0;
+        int key_algo = mode != MODE_PIPE ? pt.coll_algo : 0;
+        uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP || hyb) ? pt.bucket_bytes : 0;
+        int key_m = (mode == MODE_PIPE || hyb) ? (int)mb : 0;
+        auto key = std::make_tuple((int)pt.strategy, (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
+                                   hyb ? (int)tpd : 0, key_algo, key_bucket, key_m,
+                                   (mode == MODE_PIPE || hyb) ? plan_key : -2);
         auto ci = cls_of.find(key);
         uint32_t c;
         if (ci == cls_of.end()) {
@@ -492,13 +501,14 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.strategy = pt.strategy;
             cd.tp_mode = key_mode;
             cd.algo = key_algo;
-            cd.p = lanes;
-            cd.m = mode == MODE_PIPE ? mb : 1;
-            cd.tpdeg = pt.strategy == TRIOSIM_TP ? tpd : 1;
+            cd.p = hyb ? pp : lanes;
+            cd.m = (mode == MODE_PIPE || hyb) ? mb : 1;
+            cd.tpdeg = (pt.strategy == TRIOSIM_TP || hyb) ? tpd : 1;
+            cd.dp = hyb ? dp : 1;
             cd.b_loc = b_loc;
             cd.bucket_bytes = key_bucket;
             cd.r_b = (double)b_loc / (double)T.b0;
-            if (mode == MODE_PIPE) {
+            if (mode == MODE_PIPE || hyb) {
                 if (plan_key < 0) {
                     auto ap = T.auto_plans.find((int)pp);
                     if (ap == T.auto_plans.end()) ap = T.auto_plans.emplace((int)pp, auto_partition(T, (int)pp)).first;
@@ -523,11 +533,14 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         S->width[i] = W;
         // K3 variant: tree-capable collectives only for classes that use the tree algorithm
         S->mode[i] = (mode == MODE_COLL && pt.coll_algo == TRIOSIM_ALGO_TREE) ? MODE_TREE : mode;
+        if (hyb) S->mode[i] = MODE_HYBRID;
         double cost;
         if (mode == MODE_COLL) {
             double ncol = pt.strategy == TRIOSIM_TP ? n_tp_coll[pt.tp_mode == TRIOSIM_TP_PAPER ? 0 : 1]
                         : (key_bucket == 0 ? T.n_wgrad : std::ceil((double)T.wgrad_bytes / (double)key_bucket));
             cost = (double)N * 2 + ncol * 2.0 * lanes * 8.0;
+        } else if (hyb) {
+            cost = (double)mb * N * 2.0 / pp + (double)mb * 16.0 * lanes;
         } else {
             cost = (double)mb * N * 2.0 / lanes + (double)mb * 2.0 * 8.0 * lanes;
         }
@@ -536,6 +549,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
 
     // per-class pools
     uint32_t dur_n = 0, hook_n = 0, coll_n = 0, scr_i = 0, scr_u = 0, stage_n = 0, ent_n = 0, send_n = 0, recv_n = 0;
+    uint32_t hst_n = 0, hent_n = 0, hsend_n = 0;
     for (uint32_t c = 0; c < S->classes.size(); c++) {
         ClassDesc &cd = S->classes[c];
         cd.dur_off = dur_n; dur_n += N;
@@ -545,6 +559,20 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.coll_cap = (cd.strategy == TRIOSIM_TP) ? T.n_out_total : T.n_wgrad;
             cd.coll_off = coll_n; coll_n += cd.coll_cap;
             if (cd.strategy == TRIOSIM_TP) { cd.scratch_off = scr_i; scr_i += NT; }
+        } else if (cd.mode == MODE_HYBRID) {
+            S->hyb_list.push_back(c);
+            cd.stage_off = stage_n; stage_n += cd.p;
+            cd.hst_off = hst_n; hst_n += cd.p;
+            cd.ent_off = hent_n; cd.ent_cap = N; hent_n += N;
+            cd.send_cap = T.n_out_total * (cd.p > 1 ? cd.p - 1 : 1);
+            cd.send_off = hsend_n; hsend_n += cd.send_cap;
+            cd.recv_cap = T.n_in_total;
+            cd.recv_off = recv_n; recv_n += cd.recv_cap;
+            cd.tcol_cap = T.n_out_total;
+            cd.tcol_off = coll_n; coll_n += cd.tcol_cap;
+            cd.dcol_cap = T.n_wgrad;
+            cd.dcol_off = coll_n; coll_n += cd.dcol_cap;
+            cd.scratch_off = scr_u; scr_u += NT;
         } else {
             S->pipe_list.push_back(c);
             cd.stage_off = stage_n; stage_n += cd.p;
@@ -606,6 +634,10 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     CK(S->d_cls.upload(S->classes));
     CK(S->d_coll_list.upload(S->coll_list));
     CK(S->d_pipe_list.upload(S->pipe_list));
+    CK(S->d_hyb_list.upload(S->hyb_list));
+    CK(S->d_hst.alloc(hst_n));
+    CK(S->d_hents.alloc(hent_n));
+    CK(S->d_hsends.alloc(hsend_n));
     CK(S->d_dur.alloc(dur_n));
     CK(S->d_hooks.alloc(hook_n));
     CK(S->d_colls.alloc(coll_n));
@@ -674,6 +706,9 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     CK(launch_k2_pipe(S.d_cls.p, S.d_pipe_list.p, (uint32_t)S.pipe_list.size(), T.dev, S.d_dur.p, S.d_plans.p,
                       S.d_stages.p, S.d_ents.p, S.d_sends.p, S.d_recvs.p, S.d_scr_u64.p, st));
     if (!S.pipe_list.empty()) ctx->n_k2++;
+    CK(launch_k2_hybrid(S.d_cls.p, S.d_hyb_list.p, (uint32_t)S.hyb_list.size(), T.dev, S.d_plans.p, S.d_stages.p,
+                        S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, st));
+    if (!S.hyb_list.empty()) ctx->n_k2++;
     // K3 per segment width, forked onto side streams so the widths run concurrently
     const bool full = first == 0 && count == S.n_pts;
     CK(cudaMemsetAsync(S.d_counter.p, 0, N_GROUPS * sizeof(unsigned int), st));
@@ -702,6 +737,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         a.rt_links = S.d_rt_links.p; a.ro = S.d_ro.p;
         a.hooks = S.d_hooks.p; a.colls = S.d_colls.p; a.dur = S.d_dur.p;
         a.stages = S.d_stages.p; a.ents = S.d_ents.p; a.sends = S.d_sends.p; a.recvs = S.d_recvs.p;
+        a.hst = S.d_hst.p; a.hents = S.d_hents.p; a.hsends = S.d_hsends.p;
         a.out = S.d_res.p;
         a.alg_ops = S.d_alg.p;
         const int nseg = 32 / W;
@@ -710,7 +746,8 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)ctx->occ[w];
         if (blocks > cap) blocks = cap;
         CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
-        CK(launch_k3(W, mode, a, (int)blocks, ctx->side[w]));
+        if (mode == MODE_HYBRID) CK(launch_k3_hybrid(W, a, (int)blocks, ctx->side[w]));
+        else CK(launch_k3(W, mode, a, (int)blocks, ctx->side[w]));
         ctx->n_k3++;
         CK(cudaEventRecord(ctx->ev_join[w], ctx->side[w]));
         launched[w] = 1;

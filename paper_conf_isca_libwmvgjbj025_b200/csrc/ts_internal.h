@@ -7,7 +7,7 @@
 
 namespace ts {
 
-enum { MODE_COLL = 0, MODE_PIPE = 1, MODE_TREE = 2 };  // K3 variants: ring-only collectives, GPipe, tree-capable collectives
+enum { MODE_COLL = 0, MODE_PIPE = 1, MODE_TREE = 2, MODE_HYBRID = 3 };  // K3 variants: ring-only collectives, GPipe, tree-capable collectives, DP x TP x PP
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 constexpr int MAX_HOPS = 8;
@@ -76,6 +76,30 @@ struct RecvEnt {
     uint32_t e;      // index in the producer stage's send list of that phase
 };
 
+// HYBRID (DP x TP x PP): per stage, on top of StageInfo
+struct HStage {
+    uint32_t TF, TB, TO;      // TP collectives per micro-batch (F, B) and once (O) of one TP group
+    uint32_t tcol_off;        // CollEnt list [F TF][B TB][O TO]
+    uint32_t ndp, dcol_off;   // DP buckets of this stage (one DP group per t)
+    uint32_t first_opt;       // index of the first OPT op inside the stage's OPT list, or 0xffffffff
+    uint32_t pad;
+};
+struct HEnt {                 // per stage op entry (hybrid): the PIPE entry plus TP / DP hooks
+    uint32_t op;
+    uint16_t nsend, nrecv;
+    uint32_t recv_off;
+    uint16_t tp_nsig, dp_nsig;   // TP collectives triggered (every instance); DP buckets (instance 0)
+    int32_t tpw;                 // TP collective to wait for: (phase << 24) | index, or -1
+    uint32_t pad;
+};
+struct HSend {
+    double bytes;
+    uint32_t x;
+    uint16_t dst, pidx;
+    int32_t tpg;                 // TP collective of the tensor on the sender: (phase << 24) | index, or -1
+    uint32_t pad;
+};
+
 struct ClassDesc {
     // set by the host
     uint32_t mode, strategy, tp_mode, algo;
@@ -85,7 +109,8 @@ struct ClassDesc {
     uint32_t dur_off, hook_off, coll_off, coll_cap;
     uint32_t plan_off, stage_off, ent_off, ent_cap;
     uint32_t send_off, send_cap, recv_off, recv_cap;
-    uint32_t scratch_off, pad0;
+    uint32_t scratch_off, dp;            // dp: HYBRID data-parallel degree
+    uint32_t hst_off, tcol_off, tcol_cap, dcol_off, dcol_cap, pad1;   // HYBRID pools
     // written by K2
     uint32_t n_coll, need_ring, need_tree, n_prog_max;
     double coll_payload;
@@ -124,6 +149,9 @@ struct K3Args {
     const StageEnt *ents;
     const SendEnt *sends;
     const RecvEnt *recvs;
+    const HStage *hst;
+    const HEnt *hents;
+    const HSend *hsends;
     triosim_result *out;
     unsigned long long *alg_ops;   // method fp64 operations performed
 };
@@ -136,10 +164,15 @@ cudaError_t launch_k2_coll(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T, const double *dur,
                            const uint32_t *plan_pool, StageInfo *stages, StageEnt *ents, SendEnt *sends,
                            RecvEnt *recvs, unsigned long long *scratch_u64, cudaStream_t s);
+cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
+                             const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
+                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
+cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s);      // ts_k3h.cu
+int k3h_max_blocks_per_sm(int W);
 int k3_max_blocks_per_sm(int W, int mode);
 constexpr int N_WIDTHS = 5;             // W = 2, 4, 8, 16, 32
-constexpr int N_MODES = 3;
+constexpr int N_MODES = 4;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 
 }  // namespace ts

@@ -1,0 +1,737 @@
+// ts_k3h.cu -- K3 for HYBRID DP x TP x PP points (R9; Table 1).
+//
+// One point per W-lane segment; lane r = rank (d, s, t) with r = (d*pp + s)*tp + t.  Each lane
+// runs its stage's GPipe program (R8) and owns THREE flow slots: its TP-group collective step,
+// its DP-group collective step and its FIFO P2P send.  The TP group {(d,s,.)} is a contiguous lane
+// range, the DP group {(.,s,t)} a strided one; both run R10's ring / tree collectives through one
+// routine parameterised by (first lane, stride, size).  Instants, R14's progressive filling over
+// all flow slots and R19's hash follow ts_k3.cu.
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "ts_internal.h"
+
+namespace ts {
+
+#define FULL 0xffffffffu
+namespace {
+
+enum { CS_IDLE = 0, CS_RUN = 1 };
+enum { FS_NONE = 0, FS_LAT = 1, FS_ACT = 2 };
+enum { EV_COLL_START = 1, EV_RELEASE = 2, EV_ACTIVATE = 3, EV_DELIVER = 4, EV_TASK_START = 5, EV_TASK_END = 6 };
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    return z ^ (z >> 31);
+}
+__device__ __forceinline__ uint64_t emix(uint64_t v) { return (v ^ (v >> 29)) * 0xbf58476d1ce4e5b9ull; }
+__device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
+
+template <int W>
+__device__ __forceinline__ double seg_min(double v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) {
+        const double w = __shfl_xor_sync(FULL, v, o);
+        v = w < v ? w : v;
+    }
+    return v;
+}
+template <int W>
+__device__ __forceinline__ double seg_max(double v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) {
+        const double w = __shfl_xor_sync(FULL, v, o);
+        v = w > v ? w : v;
+    }
+    return v;
+}
+template <int W>
+__device__ __forceinline__ unsigned long long seg_sum_u64(unsigned long long v) {
+#pragma unroll
+    for (int o = W / 2; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+
+struct Topo {
+    uint32_t n_gpus, link_off, rt_off, ro_off;
+};
+
+struct Flow {
+    int st;
+    double t_act, rem, rate, t_upd, t_drain, bytes;
+    int len;
+    uint32_t hl[4];
+    uint64_t code;
+};
+
+// one collective group (TP or DP) as seen by one member lane
+struct Group {
+    bool member;
+    int p, i;                 // group size, my member index
+    int lane0, stride;        // lane of member k = lane0 + k * stride
+    int pred;                 // lane of member (i - 1) mod p
+    unsigned mask;            // lanes of the group
+    uint64_t gid;
+    uint32_t ncoll, trig, donec, cur;
+    bool running, tree_cur, ldone, uprel, upd, dnrel, dnd, fup;
+    int K, D;
+    double cS, chunk;
+    uint32_t flow_deliv;      // deliveries of this group's flows (for counts)
+};
+
+__device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[h >> 1] >> (16 * (h & 1))) & 0xffff; }
+
+__device__ __forceinline__ int route_len(const K3Args &a, const Topo &T, uint32_t s, uint32_t d) {
+    return a.rt_len[T.rt_off + s * T.n_gpus + d];
+}
+
+// release flow f along src -> dst: route latency fold (R12), link ids cached (<= 8 hops)
+__device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f, uint32_t src, uint32_t dst,
+                                        double bytes, uint64_t code, double t, double lats, uint64_t &alg) {
+    const uint32_t k = T.rt_off + src * T.n_gpus + dst;
+    const int len = a.rt_len[k];
+    const uint32_t off = a.rt_off[k];
+    double L = 0.0;
+    f.hl[0] = f.hl[1] = f.hl[2] = f.hl[3] = 0;
+#pragma unroll
+    for (int h = 0; h < MAX_HOPS; h++)
+        if (h < len) {
+            const uint32_t e = a.rt_links[off + h];
+            f.hl[h >> 1] |= e << (16 * (h & 1));
+            L = L + a.link_lat[T.link_off + e] * lats;
+        }
+    f.len = len;
+    f.st = FS_LAT;
+    f.bytes = bytes;
+    f.t_act = t + L;
+    f.code = code;
+    alg += 2 * len + 1;
+}
+
+}  // namespace
+
+template <int W>
+__global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
+    constexpr int NSEG = 32 / W;
+    constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
+    __shared__ double s_res[K3_WARPS][NSEG * LMAX];
+    __shared__ int s_n[K3_WARPS][NSEG * LMAX];
+    __shared__ int s_k[K3_WARPS][NSEG * LMAX];
+    __shared__ uint32_t s_cnt[K3_WARPS][32];
+
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int seg = lane / W, li = lane % W, sbase = seg * W;
+    const unsigned smask = (W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase;
+    double *lres = &s_res[wid][seg * LMAX];
+    int *ln = &s_n[wid][seg * LMAX];
+    int *lk = &s_k[wid][seg * LMAX];
+    uint32_t *cnt = &s_cnt[wid][0];   // indexed by warp lane
+    for (int q = lane; q < NSEG * LMAX; q += 32) { s_n[wid][q] = 0; s_k[wid][q] = 0; }
+    __syncwarp();
+
+    // ---- segment-uniform ----
+    bool have = false, exhausted = false;
+    uint32_t pidx = 0;
+    double t = 0.0, bws = 1.0, lats = 1.0;
+    int R = 1, S = 1, tp = 1, dp = 1;
+    uint32_t m = 1;
+    bool tree_algo = false;
+    const ClassDesc *C = nullptr;
+    Topo TR = {0, 0, 0, 0};
+    uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
+    bool bon = false;
+    double bstart = 0.0, cbusy = 0.0;
+    // ---- lane ----
+    bool used = false;
+    int d = 0, s = 0, tt = 0;
+    uint32_t gpu = 0, pos = 0, run_start = 0, run_end = 0, nprog = 0;
+    int cst = CS_IDLE;
+    double t_end = 0.0, busy = 0.0;
+    uint32_t ntask = 0, nflow = 0, np2p = 0;
+    StageInfo SI;
+    SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
+    SI.ent_off = SI.send_off = SI.recv_off = 0;
+    HStage HS;
+    HS.TF = HS.TB = HS.TO = HS.tcol_off = HS.ndp = HS.dcol_off = 0;
+    HS.first_opt = 0xffffffffu;
+    uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
+    Group GT, GD;
+    GT.member = GD.member = false;
+    Flow FT, FD, FP;
+    FT.st = FD.st = FP.st = FS_NONE;
+    uint64_t acc = 0, alg = 0, tmix = 0;
+    bool nev = false;
+
+#define EV(kind, code)                                                        \
+    do {                                                                      \
+        acc += emix(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code)));   \
+        nev = true;                                                           \
+    } while (0)
+
+    auto grp_init = [&](Group &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll) {
+        G.member = member;
+        G.p = p;
+        G.i = i;
+        G.lane0 = lane0;
+        G.stride = stride;
+        G.pred = lane0 + ((i + p - 1) % p) * stride;
+        G.mask = 0;
+        for (int k = 0; k < p; k++) G.mask |= 1u << (lane0 + k * stride);
+        G.gid = gid;
+        G.ncoll = ncoll;
+        G.trig = G.donec = G.cur = 0;
+        G.running = G.tree_cur = G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = G.fup = false;
+        G.K = G.D = 0;
+        G.cS = G.chunk = 0.0;
+        G.flow_deliv = 0;
+    };
+    auto gpu_of_member = [&](const Group &G, int k) -> uint32_t { return a.ro[TR.ro_off + (G.lane0 - sbase) + k * G.stride]; };
+    auto tp_seq = [&](uint32_t P, uint32_t j, uint32_t e) -> uint32_t {
+        return P == 0 ? j * HS.TF + e : P == 1 ? m * HS.TF + (m - 1 - j) * HS.TB + e : m * (HS.TF + HS.TB) + e;
+    };
+
+    // R10 for one group: done on this member, finish, start, releases (all lanes call it)
+    auto grp_pass = [&](Group &G, Flow &F, bool is_tp, bool &more) {
+        const int Dp = __shfl_sync(FULL, G.D, G.pred);
+        unsigned upb = 0, dnb = 0;
+        if (__any_sync(FULL, G.tree_cur)) {
+            upb = __ballot_sync(FULL, G.upd);
+            dnb = __ballot_sync(FULL, G.dnd);
+        }
+        auto mb = [&](unsigned b, int k) -> bool { return (b >> (G.lane0 + k * G.stride)) & 1u; };
+        const int c1 = 2 * G.i + 1, c2 = 2 * G.i + 2;
+        if (G.member && G.running && !G.ldone) {
+            bool dn;
+            if (!G.tree_cur) {
+                dn = G.D == G.K && Dp == G.K;
+            } else {
+                const bool ku = (c1 >= G.p || mb(upb, c1)) && (c2 >= G.p || mb(upb, c2));
+                const bool kd = (c1 >= G.p || mb(dnb, c1)) && (c2 >= G.p || mb(dnb, c2));
+                dn = (G.i == 0 || (G.upd && G.dnd)) && ku && kd;
+            }
+            if (dn) {
+                G.ldone = true;
+                G.donec = G.cur + 1;
+            }
+        }
+        const bool allfin = (__ballot_sync(FULL, !G.member || G.ldone) & G.mask) == G.mask;
+        if (G.member && G.running && allfin) {
+            G.running = false;
+            G.cur++;
+        }
+        const bool allrdy = (__ballot_sync(FULL, !G.member || G.trig > G.cur) & G.mask) == G.mask;
+        bool started = false;
+        if (G.member && !G.running && G.cur < G.ncoll && allrdy) {
+            CollEnt ce;
+            if (is_tp) {
+                const uint32_t c = G.cur;
+                uint32_t off;
+                if (c < m * HS.TF) off = c % HS.TF;
+                else if (c < m * (HS.TF + HS.TB)) off = HS.TF + (c - m * HS.TF) % HS.TB;
+                else off = HS.TF + HS.TB + (c - m * (HS.TF + HS.TB));
+                ce = a.colls[HS.tcol_off + off];
+            } else {
+                ce = a.colls[HS.dcol_off + G.cur];
+            }
+            G.running = started = true;
+            G.tree_cur = tree_algo && ce.kind == CK_AR;
+            G.cS = ce.S;
+            G.chunk = ce.S / (double)G.p;
+            G.K = ce.kind == CK_AR ? 2 * (G.p - 1) : (G.p - 1);
+            G.D = 0;
+            G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = false;
+            if (G.i == 0) {
+                EV(EV_COLL_START, (G.gid << 20) | G.cur);
+                alg += 1;
+            }
+        }
+        if (G.member && G.running && F.st == FS_NONE) {
+            const uint64_t cc = (G.gid << 20) | G.cur;
+            bool rel = false;
+            if (!G.tree_cur) {
+                if (G.D < G.K && (G.D == 0 || Dp >= G.D)) {
+                    release(a, TR, F, gpu, gpu_of_member(G, (G.i + 1) % G.p), G.chunk,
+                            (cc << 32) | ((uint64_t)G.D << 16) | (uint64_t)G.i, t, lats, alg);
+                    rel = true;
+                }
+            } else if (G.i >= 1) {
+                const unsigned ub = started ? 0u : upb, db = started ? 0u : dnb;
+                const bool ku = (c1 >= G.p || mb(ub, c1)) && (c2 >= G.p || mb(ub, c2));
+                const int par = (G.i - 1) / 2;
+                if (!G.uprel && ku) {
+                    release(a, TR, F, gpu, gpu_of_member(G, par), G.cS, (cc << 32) | (uint64_t)G.i, t, lats, alg);
+                    G.fup = G.uprel = rel = true;
+                } else if (G.uprel && G.upd && !G.dnrel &&
+                           (par == 0 ? ((G.p <= 1 || mb(ub, 1)) && (G.p <= 2 || mb(ub, 2))) : mb(db, par))) {
+                    release(a, TR, F, gpu_of_member(G, par), gpu, G.cS, (cc << 32) | (1ull << 16) | (uint64_t)G.i, t,
+                            lats, alg);
+                    G.fup = false;
+                    G.dnrel = rel = true;
+                }
+            }
+            if (rel) {
+                EV(EV_RELEASE, F.code);
+                if (F.t_act == t) more = true;
+            }
+        }
+    };
+    // (b)/(c) for one flow slot; returns true if delivered
+    auto flow_step = [&](Flow &F, bool &dirty) -> bool {
+        if (F.st == FS_ACT && F.t_drain == t) {
+            F.st = FS_NONE;
+            EV(EV_DELIVER, F.code);
+            dirty = true;
+            return true;
+        }
+        if (F.st == FS_LAT && F.t_act == t) {
+            EV(EV_ACTIVATE, F.code);
+            if (F.bytes == 0.0 || F.len == 0) {
+                F.st = FS_NONE;
+                EV(EV_DELIVER, F.code);
+                return true;
+            }
+            F.st = FS_ACT;
+            F.rem = F.bytes;
+            F.t_upd = t;
+            F.rate = 0.0;
+            F.t_drain = dinf();
+            dirty = true;
+        }
+        return false;
+    };
+    auto grp_delivered = [&](Group &G) {
+        G.flow_deliv++;
+        if (G.tree_cur) {
+            if (G.fup) G.upd = true; else G.dnd = true;
+        } else {
+            G.D++;
+        }
+    };
+    // decode program position q of this stage -> (phase, micro-batch, index in phase list)
+    auto decode = [&](uint32_t q, uint32_t &P, uint32_t &j, uint32_t &idx) {
+        if (q < m * SI.nF) { P = 0; j = q / SI.nF; idx = q % SI.nF; }
+        else if (q < m * (SI.nF + SI.nB)) { const uint32_t r = q - m * SI.nF; P = 1; j = m - 1 - r / SI.nB; idx = r % SI.nB; }
+        else { P = 2; j = 0; idx = q - m * (SI.nF + SI.nB); }
+    };
+    auto ent_at = [&](uint32_t P, uint32_t idx) -> HEnt {
+        return a.hents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx];
+    };
+    auto has_wait = [&](const HEnt &en, uint32_t P, uint32_t idx) -> bool {
+        return en.nrecv > 0 || en.tpw >= 0 || (P == 2 && idx == HS.first_opt && GD.ncoll > 0);
+    };
+    auto has_sig = [&](const HEnt &en, uint32_t j) -> bool {
+        return en.nsend > 0 || en.tp_nsig > 0 || (en.dp_nsig > 0 && j == 0);
+    };
+
+    for (;;) {
+        // ------------------------------ refill ------------------------------
+        const bool need = !have && !exhausted;
+        bool fresh = false, rbad = false, rlong = false;
+        if (__any_sync(FULL, need)) {
+            uint32_t it = 0;
+            if (need && li == 0) it = atomicAdd(a.counter, 1u);
+            it = __shfl_sync(FULL, it, sbase);
+            if (need) {
+                if (it >= a.n_work) {
+                    exhausted = true;
+                } else {
+                    fresh = have = true;
+                    const PointDesc pd = a.pts[a.work[it]];
+                    pidx = pd.idx;
+                    bws = pd.bw_scale;
+                    lats = pd.lat_scale;
+                    C = &a.cls[pd.cls];
+                    {
+                        const TopoDev td = a.topo[pd.topo];
+                        TR.n_gpus = td.n_gpus; TR.link_off = td.link_off; TR.rt_off = td.rt_off; TR.ro_off = td.ro_off;
+                    }
+                    S = (int)C->p;
+                    tp = (int)C->tpdeg;
+                    dp = (int)C->dp;
+                    R = dp * S * tp;
+                    m = C->m;
+                    tree_algo = C->algo == TRIOSIM_ALGO_TREE;
+                    t = 0.0;
+                    tmix = mix64(0ull);
+                    ninst = nwf = nrounds = maxact = 0;
+                    bon = false;
+                    bstart = cbusy = 0.0;
+                    used = li < R;
+                    pos = run_start = run_end = 0;
+                    cst = CS_IDLE;
+                    t_end = busy = 0.0;
+                    ntask = nflow = np2p = 0;
+                    sq = dcnt = 0;
+                    FT.st = FD.st = FP.st = FS_NONE;
+                    acc = alg = 0;
+                    nev = false;
+                    const int r = used ? li : 0;
+                    d = r / (S * tp);
+                    s = (r / tp) % S;
+                    tt = r % tp;
+                    SI = a.stages[C->stage_off + s];
+                    HS = a.hst[C->hst_off + s];
+                    nprog = used ? m * (SI.nF + SI.nB) + SI.nO : 0;
+                    nsend_tot = used ? m * (SI.SF + SI.SB) + SI.SO : 0;
+                    gpu = a.ro[TR.ro_off + r];
+                    const uint32_t ntp = tp > 1 ? m * (HS.TF + HS.TB) + HS.TO : 0;
+                    const uint32_t ndp = dp > 1 ? HS.ndp : 0;
+                    grp_init(GT, used && tp > 1, tp, tt, sbase + (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp);
+                    grp_init(GD, used && dp > 1, dp, d, sbase + s * tp + tt, S * tp,
+                             (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp);
+                    if (used) {
+                        // route checks of every pair this rank's flows will use (R3)
+                        auto chk = [&](uint32_t x, uint32_t y) {
+                            const int l = route_len(a, TR, x, y);
+                            if (l == NO_ROUTE) rbad = true;
+                            else if (l > MAX_HOPS) rlong = true;
+                        };
+                        for (int gk = 0; gk < 2; gk++) {
+                            const Group &G = gk == 0 ? GT : GD;
+                            if (!G.member || G.ncoll == 0) continue;
+                            if (C->need_ring) chk(gpu, gpu_of_member(G, (G.i + 1) % G.p));
+                            if (C->need_tree && G.i >= 1) {
+                                const uint32_t par = gpu_of_member(G, (G.i - 1) / 2);
+                                chk(gpu, par);
+                                chk(par, gpu);
+                            }
+                        }
+                        unsigned long long dm = SI.dst_mask;
+                        while (dm) {
+                            const int ds = __ffsll((long long)dm) - 1;
+                            dm &= dm - 1;
+                            chk(gpu, a.ro[TR.ro_off + (d * S + ds) * tp + tt]);
+                        }
+                    }
+                }
+            }
+            if (__any_sync(FULL, fresh && (rbad || rlong))) {
+                const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
+                const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
+                if (fresh && (bad || lng)) {
+                    if (li == 0) {
+                        triosim_result rr = {};
+                        rr.status = bad ? TRIOSIM_PT_NO_ROUTE : TRIOSIM_PT_TOO_LARGE;
+                        a.out[pidx] = rr;
+                    }
+                    have = used = false;
+                    GT.member = GD.member = false;
+                }
+            }
+        }
+        if (__all_sync(FULL, !have && exhausted)) break;
+
+        // ------------------------------ one instant ------------------------------
+        bool dirty = false;
+        for (;;) {
+            for (;;) {
+                bool more = false;
+                // (a) completions
+                if (used && cst == CS_RUN && t_end == t) {
+                    cst = CS_IDLE;
+                    pos = run_end;
+                    uint32_t P, j, idx;
+                    decode(pos - 1, P, j, idx);
+                    const HEnt en = ent_at(P, idx);
+                    GT.trig += en.tp_nsig;
+                    if (j == 0) GD.trig += en.dp_nsig;
+                    if (has_sig(en, j)) EV(EV_TASK_END, ((uint64_t)gpu << 40) | (pos - 1));
+                }
+                // (b) / (c) for the three flow slots
+                if (used) {
+                    if (flow_step(FT, dirty)) { nflow++; grp_delivered(GT); }
+                    if (flow_step(FD, dirty)) { nflow++; grp_delivered(GD); }
+                    if (flow_step(FP, dirty)) { nflow++; np2p++; dcnt++; }
+                }
+                cnt[lane] = dcnt;
+                __syncwarp();
+                // (d) both groups, then this rank's next P2P send
+                grp_pass(GT, FT, true, more);
+                grp_pass(GD, FD, false, more);
+                if (used && FP.st == FS_NONE && sq < nsend_tot) {
+                    uint32_t P, j, e;
+                    if (sq < m * SI.SF) { P = 0; j = sq / SI.SF; e = sq % SI.SF; }
+                    else if (sq < m * (SI.SF + SI.SB)) { const uint32_t r = sq - m * SI.SF; P = 1; j = m - 1 - r / SI.SB; e = r % SI.SB; }
+                    else { P = 2; j = 0; e = sq - m * (SI.SF + SI.SB); }
+                    const HSend se = a.hsends[SI.send_off + (P == 0 ? 0 : P == 1 ? SI.SF : SI.SF + SI.SB) + e];
+                    const uint32_t prodpos = P == 0 ? j * SI.nF + se.pidx
+                                           : P == 1 ? m * SI.nF + (m - 1 - j) * SI.nB + se.pidx
+                                                    : m * (SI.nF + SI.nB) + se.pidx;
+                    const uint32_t donepos = (cst == CS_RUN) ? run_start : pos;
+                    const bool gate = se.tpg < 0 ||
+                                      GT.donec > tp_seq((uint32_t)se.tpg >> 24, j, (uint32_t)se.tpg & 0xffffffu);
+                    if (donepos > prodpos && gate) {
+                        const uint32_t dg = a.ro[TR.ro_off + (d * S + se.dst) * tp + tt];
+                        release(a, TR, FP, gpu, dg, se.bytes,
+                                (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg, t, lats, alg);
+                        EV(EV_RELEASE, FP.code);
+                        sq++;
+                        if (FP.t_act == t) more = true;
+                    }
+                }
+                // (e) compute start
+                if (used && cst == CS_IDLE && pos < nprog) {
+                    uint32_t P, j, idx;
+                    decode(pos, P, j, idx);
+                    HEnt en = ent_at(P, idx);
+                    bool ok = true;
+                    for (uint32_t r = 0; r < en.nrecv && ok; r++) {
+                        const RecvEnt re = a.recvs[en.recv_off + r];
+                        const StageInfo &ps = a.stages[C->stage_off + re.src];
+                        const uint32_t jp = (re.phase == 2 || P == 2) ? 0 : j;
+                        const uint32_t seqi = re.phase == 0 ? jp * ps.SF + re.e
+                                            : re.phase == 1 ? m * ps.SF + (m - 1 - jp) * ps.SB + re.e
+                                                            : m * (ps.SF + ps.SB) + re.e;
+                        if (!(cnt[sbase + (d * S + re.src) * tp + tt] > seqi)) ok = false;
+                    }
+                    if (ok && en.tpw >= 0) {
+                        const uint32_t pp_ = (uint32_t)en.tpw >> 24, ee = (uint32_t)en.tpw & 0xffffffu;
+                        const uint32_t jp = (pp_ == 2 || P == 2) ? 0 : j;
+                        if (!(GT.donec > tp_seq(pp_, jp, ee))) ok = false;
+                    }
+                    if (ok && P == 2 && idx == HS.first_opt && GD.ncoll > 0 && GD.donec < GD.ncoll) ok = false;
+                    if (ok) {
+                        if (has_wait(en, P, idx)) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
+                        run_start = pos;
+                        const double *du = a.dur + C->dur_off;
+                        double te = t + du[en.op];
+                        busy = busy + du[en.op];
+                        bool sig = has_sig(en, j);
+                        uint32_t q = pos + 1;
+                        while (!sig && q < nprog) {
+                            uint32_t P2, j2, i2;
+                            decode(q, P2, j2, i2);
+                            const HEnt e2 = ent_at(P2, i2);
+                            if (has_wait(e2, P2, i2)) break;
+                            te = te + du[e2.op];
+                            busy = busy + du[e2.op];
+                            sig = has_sig(e2, j2);
+                            q++;
+                        }
+                        ntask += q - pos;
+                        alg += 2 * (q - pos);
+                        run_end = q;
+                        t_end = te;
+                        cst = CS_RUN;
+                        if (te == t) more = true;
+                    }
+                }
+                __syncwarp();
+                if (!__any_sync(FULL, more)) break;
+            }
+
+            // (f) R14 over every in-transit flow of the segment (up to three per lane)
+            const unsigned dball = __ballot_sync(FULL, dirty);
+            if (!dball) break;
+            const bool segdirty = (dball & smask) != 0;
+            dirty = false;
+            const bool aT = segdirty && used && FT.st == FS_ACT;
+            const bool aD = segdirty && used && FD.st == FS_ACT;
+            const bool aP = segdirty && used && FP.st == FS_ACT;
+            auto progress = [&](Flow &F, bool on) {
+                if (on && F.t_upd < t) {
+                    const double r = F.rem - F.rate * (t - F.t_upd);
+                    F.rem = r > 0.0 ? r : 0.0;
+                    F.t_upd = t;
+                    alg += 4;
+                }
+            };
+            progress(FT, aT);
+            progress(FD, aD);
+            progress(FP, aP);
+            auto zero = [&](const Flow &F, bool on) {
+                if (on)
+                    for (int h = 0; h < F.len; h++) ln[hop(F.hl, h)] = 0;
+            };
+            zero(FT, aT);
+            zero(FD, aD);
+            zero(FP, aP);
+            __syncwarp();
+            auto count = [&](const Flow &F, bool on) {
+                if (on) {
+                    alg += F.len;
+                    for (int h = 0; h < F.len; h++) {
+                        const int e = hop(F.hl, h);
+                        atomicAdd(&ln[e], 1);
+                        lres[e] = a.link_bw[TR.link_off + e] * bws;
+                    }
+                }
+            };
+            count(FT, aT);
+            count(FD, aD);
+            count(FP, aP);
+            __syncwarp();
+            bool uT = aT, uD = aD, uP = aP;
+            uint32_t rounds = 0;
+            auto fmin = [&](const Flow &F, bool on) -> double {
+                double my = dinf();
+                if (on) {
+                    for (int h = 0; h < F.len; h++) {
+                        const int e = hop(F.hl, h);
+                        const double sh = lres[e] / (double)ln[e];
+                        my = sh < my ? sh : my;
+                    }
+                    alg += 2 * F.len;
+                }
+                return my;
+            };
+            while (__any_sync(FULL, uT || uD || uP)) {
+                const bool segact = (__ballot_sync(FULL, uT || uD || uP) & smask) != 0;
+                const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
+                double my = mT < mD ? mT : mD;
+                my = mP < my ? mP : my;
+                const double sm = seg_min<W>(my);
+                const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
+                unsigned own = 0;
+                auto freeze = [&](Flow &F, bool in, int slot) {
+                    if (in) {
+                        F.rate = sm;
+                        for (int h = 0; h < F.len; h++)
+                            if (atomicAdd(&lk[hop(F.hl, h)], 1) == 0) own |= 1u << (slot * 8 + h);
+                    }
+                };
+                freeze(FT, iT, 0);
+                freeze(FD, iD, 1);
+                freeze(FP, iP, 2);
+                __syncwarp();
+                auto update = [&](const Flow &F, int slot) {
+                    for (int h = 0; h < F.len; h++)
+                        if ((own >> (slot * 8 + h)) & 1u) {
+                            const int e = hop(F.hl, h);
+                            const int kk = lk[e];
+                            const double r = lres[e] - sm * (double)kk;
+                            lres[e] = r > 0.0 ? r : 0.0;
+                            ln[e] -= kk;
+                            lk[e] = 0;
+                            alg += 3;
+                        }
+                };
+                if (own) {
+                    update(FT, 0);
+                    update(FD, 1);
+                    update(FP, 2);
+                }
+                __syncwarp();
+                if (segact) rounds++;
+                uT = uT && !iT;
+                uD = uD && !iD;
+                uP = uP && !iP;
+            }
+            const uint32_t nact = __popc(__ballot_sync(FULL, aT) & smask) + __popc(__ballot_sync(FULL, aD) & smask) +
+                                  __popc(__ballot_sync(FULL, aP) & smask);
+            if (segdirty) {
+                nwf++;
+                nrounds += rounds;
+                if (nact > maxact) maxact = nact;
+            }
+            bool again = false;
+            auto drain = [&](Flow &F, bool on) {
+                if (on) {
+                    F.t_drain = (F.rem == 0.0) ? t : t + F.rem / F.rate;
+                    alg += 2;
+                    if (F.t_drain == t) again = true;
+                }
+            };
+            drain(FT, aT);
+            drain(FD, aD);
+            drain(FP, aP);
+            if (!__any_sync(FULL, again)) break;
+        }
+
+        // ------------------------------ end of instant ------------------------------
+        const bool any_ev = (__ballot_sync(FULL, nev) & smask) != 0;
+        if (have && any_ev) ninst++;
+        nev = false;
+        const bool infl = (__ballot_sync(FULL, used && (FT.st != FS_NONE || FD.st != FS_NONE || FP.st != FS_NONE)) &
+                           smask) != 0;
+        if (have) {
+            if (infl && !bon) { bon = true; bstart = t; }
+            else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
+        }
+        const bool lane_done = !used || (cst == CS_IDLE && pos >= nprog && FT.st == FS_NONE && FD.st == FS_NONE &&
+                                         FP.st == FS_NONE && sq >= nsend_tot && GT.cur >= GT.ncoll * (GT.member ? 1u : 0u) &&
+                                         GD.cur >= GD.ncoll * (GD.member ? 1u : 0u) && !GT.running && !GD.running);
+        const bool alldone = (__ballot_sync(FULL, lane_done) & smask) == smask;
+        const bool fin = have && alldone;
+        double cand = dinf();
+        if (used) {
+            if (cst == CS_RUN) cand = t_end;
+            const Flow *fs[3] = {&FT, &FD, &FP};
+#pragma unroll
+            for (int k = 0; k < 3; k++) {
+                if (fs[k]->st == FS_LAT && fs[k]->t_act < cand) cand = fs[k]->t_act;
+                if (fs[k]->st == FS_ACT && fs[k]->t_drain < cand) cand = fs[k]->t_drain;
+            }
+        }
+        const double tn = seg_min<W>(cand);
+        const bool stuck = have && !fin && !(tn < dinf());
+        if (__any_sync(FULL, fin || stuck)) {
+            const double bmax = seg_max<W>(used ? busy : 0.0);
+            const unsigned long long ntk = seg_sum_u64<W>(ntask);
+            const unsigned long long nfl = seg_sum_u64<W>(nflow);
+            const unsigned long long npp = seg_sum_u64<W>(np2p);
+            const unsigned long long alg_s = seg_sum_u64<W>(alg);
+            const unsigned long long H = seg_sum_u64<W>(acc);
+            if ((fin || stuck) && li == 0) {
+                triosim_result rr;
+                rr.iter_time_s = fin ? t : 0.0;
+                rr.compute_busy_max_s = fin ? bmax : 0.0;
+                rr.comm_busy_s = fin ? cbusy : 0.0;
+                rr.exposed_comm_s = fin ? t - bmax : 0.0;
+                rr.coll_payload_bytes = fin ? C->coll_payload : 0.0;
+                rr.n_compute = fin ? ntk : 0;
+                rr.n_flows = fin ? nfl : 0;
+                rr.n_collectives = fin ? C->n_coll : 0;
+                rr.n_p2p = fin ? npp : 0;
+                rr.n_instants = fin ? ninst : 0;
+                rr.n_wf_calls = fin ? nwf : 0;
+                rr.n_wf_rounds = fin ? nrounds : 0;
+                rr.order_hash = fin ? H : 0;
+                rr.status = fin ? TRIOSIM_PT_OK : TRIOSIM_PT_DEADLOCK;
+                rr.max_active_flows = fin ? maxact : 0;
+                a.out[pidx] = rr;
+                if (a.alg_ops) atomicAdd(a.alg_ops, alg_s);
+            }
+            if (fin || stuck) {
+                have = used = false;
+                GT.member = GD.member = false;
+            }
+        }
+        if (have) {
+            t = tn;
+            tmix = mix64((uint64_t)__double_as_longlong(t));
+        }
+    }
+#undef EV
+}
+
+template <int W>
+static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
+    k3_hybrid<W><<<grid, K3_THREADS, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
+    switch (W) {
+    case 2: return launch_h<2>(a, grid, s);
+    case 4: return launch_h<4>(a, grid, s);
+    case 8: return launch_h<8>(a, grid, s);
+    case 16: return launch_h<16>(a, grid, s);
+    case 32: return launch_h<32>(a, grid, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+int k3h_max_blocks_per_sm(int W) {
+    int nb = 0;
+    switch (W) {
+    case 2: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<2>, K3_THREADS, 0); break;
+    case 4: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<4>, K3_THREADS, 0); break;
+    case 8: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<8>, K3_THREADS, 0); break;
+    case 16: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<16>, K3_THREADS, 0); break;
+    default: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<32>, K3_THREADS, 0); break;
+    }
+    return nb > 0 ? nb : 1;
+}
+
+}  // namespace ts

@@ -407,4 +407,312 @@ cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, con
     k2_pipe<<<n, K2P_THREADS, 0, s>>>(cls, list, T, dur, plan_pool, stages, ents, sends, recvs, scratch);
     return cudaGetLastError();
 }
+
+// ------------------------------------------------------------------------------------
+// K2 (HYBRID): one CTA per DP x TP x PP class; thread s builds stage s (R9)
+// ------------------------------------------------------------------------------------
+__device__ __forceinline__ int tp_kind_dev(uint32_t role, uint32_t phase, uint8_t cat, uint32_t tp_mode) {
+    if (tp_mode == TRIOSIM_TP_PAPER) {
+        if ((role & TRIOSIM_ROLE_GATHER) && phase == PH_FWD) return CK_AG;
+        if ((role & TRIOSIM_ROLE_GATHER) && phase == PH_BWD && cat == TRIOSIM_CAT_AGRAD) return CK_AR;
+    } else {
+        if ((role & 3u) == TRIOSIM_ROLE_ROW && phase == PH_FWD) return CK_AR;
+        if ((role & 3u) == TRIOSIM_ROLE_COL && phase == PH_BWD && cat == TRIOSIM_CAT_AGRAD) return CK_AR;
+    }
+    return -1;
+}
+
+__global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const uint32_t *list, TraceDev T,
+                                                         const uint32_t *plan_pool, StageInfo *stages, HStage *hst,
+                                                         HEnt *ents, HSend *sends, RecvEnt *recvs, CollEnt *colls,
+                                                         unsigned long long *scratch) {
+    ClassDesc &C = cls[list[blockIdx.x]];
+    __shared__ uint16_t s_stage[K2P_MAX_LAYERS];
+    __shared__ uint32_t s_cnt[64][6];
+    const int tid = threadIdx.x, nt = blockDim.x;
+    const int S = (int)C.p, tp = (int)C.tpdeg, dp = (int)C.dp;
+    const uint32_t m = C.m;
+    const uint32_t *fl = plan_pool + C.plan_off;
+    for (uint32_t l = tid; l < T.n_layers; l += nt) {
+        int s = 0;
+        while (s + 1 < S && fl[s + 1] <= l) s++;
+        s_stage[l] = (uint16_t)s;
+    }
+    unsigned long long *readers = scratch + C.scratch_off;
+    for (uint32_t x = tid; x < T.n_ts; x += nt) readers[x] = 0ull;
+    __syncthreads();
+    for (uint32_t o = tid; o < T.n_ops; o += nt) {
+        const triosim_op op = T.ops[o];
+        const unsigned long long bit = 1ull << s_stage[op.layer];
+        for (uint32_t k = 0; k < op.n_in; k++) atomicOr(&readers[T.io[op.io_off + k]], bit);
+    }
+    __syncthreads();
+    StageInfo *SI = stages + C.stage_off;
+    HStage *HS = hst + C.hst_off;
+    // pass 1: sizes of every per-stage list
+    if (tid < S) {
+        const int s = tid;
+        uint32_t n[3] = {0, 0, 0}, sn[3] = {0, 0, 0}, tn[3] = {0, 0, 0}, nrecv = 0;
+        unsigned long long dmask = 0;
+        for (uint32_t o = 0; o < T.n_ops; o++) {
+            const triosim_op op = T.ops[o];
+            if (s_stage[op.layer] != s) continue;
+            n[op.phase]++;
+            for (uint32_t k = 0; k < op.n_out; k++) {
+                const uint32_t x = T.io[op.io_off + op.n_in + k];
+                const unsigned long long r = readers[x] & ~(1ull << s);
+                sn[op.phase] += __popcll(r);
+                dmask |= r;
+                if (tp > 1 && tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode) >= 0) tn[op.phase]++;
+            }
+            for (uint32_t k = 0; k < op.n_in; k++) {
+                const int32_t po = T.prod[T.io[op.io_off + k]];
+                if (po >= 0 && s_stage[T.layer[po]] != s) nrecv++;
+            }
+        }
+        uint32_t nb = 0;
+        if (dp > 1) {
+            const int nw = T.scal[0];
+            uint64_t sum = 0;
+            bool open = false;
+            for (int i = 0; i < nw; i++) {
+                const uint32_t x = T.wgrad[i];
+                if (s_stage[T.layer[T.prod[x]]] != s) continue;
+                sum += T.ts[x].bytes_b0;
+                open = true;
+                if (C.bucket_bytes == 0 || sum >= C.bucket_bytes) { nb++; sum = 0; open = false; }
+            }
+            if (open) nb++;
+        }
+        SI[s].nF = n[0]; SI[s].nB = n[1]; SI[s].nO = n[2];
+        SI[s].SF = sn[0]; SI[s].SB = sn[1]; SI[s].SO = sn[2];
+        SI[s].dst_mask = dmask;
+        HS[s].TF = tn[0]; HS[s].TB = tn[1]; HS[s].TO = tn[2];
+        HS[s].ndp = nb;
+        HS[s].first_opt = n[2] > 0 ? 0u : 0xffffffffu;
+        s_cnt[s][0] = n[0] + n[1] + n[2];
+        s_cnt[s][1] = sn[0] + sn[1] + sn[2];
+        s_cnt[s][2] = nrecv;
+        s_cnt[s][3] = tn[0] + tn[1] + tn[2];
+        s_cnt[s][4] = nb;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        uint32_t e = 0, sd = 0, rv = 0, tc = 0, dc = 0;
+        for (int s = 0; s < S; s++) {
+            SI[s].ent_off = C.ent_off + e;
+            SI[s].send_off = C.send_off + sd;
+            SI[s].recv_off = C.recv_off + rv;
+            HS[s].tcol_off = C.tcol_off + tc;
+            HS[s].dcol_off = C.dcol_off + dc;
+            e += s_cnt[s][0]; sd += s_cnt[s][1]; rv += s_cnt[s][2]; tc += s_cnt[s][3]; dc += s_cnt[s][4];
+        }
+    }
+    __syncthreads();
+    // pass 2: op entries, sends, TP lists (program order), DP buckets (production order)
+    if (tid < S) {
+        const int s = tid;
+        const StageInfo si = SI[s];
+        const HStage hs = HS[s];
+        const uint32_t eoff[3] = {si.ent_off, si.ent_off + si.nF, si.ent_off + si.nF + si.nB};
+        const uint32_t soff[3] = {si.send_off, si.send_off + si.SF, si.send_off + si.SF + si.SB};
+        const uint32_t toff[3] = {hs.tcol_off, hs.tcol_off + hs.TF, hs.tcol_off + hs.TF + hs.TB};
+        uint32_t ei[3] = {0, 0, 0}, sj[3] = {0, 0, 0}, tj[3] = {0, 0, 0};
+        for (uint32_t o = 0; o < T.n_ops; o++) {
+            const triosim_op op = T.ops[o];
+            if (s_stage[op.layer] != s) continue;
+            const int P = op.phase;
+            uint32_t nsend = 0, ntp = 0;
+            for (uint32_t k = 0; k < op.n_out; k++) {
+                const uint32_t x = T.io[op.io_off + op.n_in + k];
+                unsigned long long r = readers[x] & ~(1ull << s);
+                while (r) {
+                    const int d = __ffsll((long long)r) - 1;
+                    r &= r - 1;
+                    HSend se;
+                    se.bytes = tensor_bytes(T, x, C.r_b, C.tpdeg, C.tp_mode);
+                    se.x = x;
+                    se.dst = (uint16_t)d;
+                    se.pidx = (uint16_t)ei[P];
+                    se.tpg = -1;
+                    se.pad = 0;
+                    sends[soff[P] + sj[P]++] = se;
+                    nsend++;
+                }
+                if (tp > 1) {
+                    const int kind = tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode);
+                    if (kind >= 0) {
+                        CollEnt ce;
+                        ce.S = (double)T.ts[x].bytes_b0;
+                        if (T.ts[x].batch_scaled) ce.S = ce.S * C.r_b;
+                        ce.kind = (uint32_t)kind;
+                        ce.pad = x;
+                        colls[toff[P] + tj[P]++] = ce;
+                        ntp++;
+                    }
+                }
+            }
+            HEnt en;
+            en.op = o;
+            en.nsend = (uint16_t)nsend;
+            en.nrecv = 0;
+            en.recv_off = 0;
+            en.tp_nsig = (uint16_t)ntp;
+            en.dp_nsig = 0;
+            en.tpw = -1;
+            en.pad = 0;
+            ents[eoff[P] + ei[P]++] = en;
+        }
+        if (dp > 1) {
+            const int nw = T.scal[0];
+            uint64_t sum = 0;
+            double Sb = 0.0;
+            uint32_t b = 0;
+            int32_t last_prod = -1;
+            bool open = false;
+            for (int i = 0; i <= nw; i++) {
+                const bool end = i == nw;
+                if (!end) {
+                    const uint32_t x = T.wgrad[i];
+                    if (s_stage[T.layer[T.prod[x]]] != s) continue;
+                    sum += T.ts[x].bytes_b0;
+                    Sb = Sb + tensor_bytes(T, x, C.r_b, C.tpdeg, C.tp_mode);
+                    last_prod = T.prod[x];
+                    open = true;
+                }
+                if (open && (end || C.bucket_bytes == 0 || sum >= C.bucket_bytes)) {
+                    CollEnt ce;
+                    ce.S = Sb;
+                    ce.kind = CK_AR;
+                    ce.pad = 0;
+                    colls[hs.dcol_off + b++] = ce;
+                    // trigger: (producer of the bucket's last gradient, micro-batch 0)
+                    const int P = (int)(T.info[last_prod] & INFO_PHASE_MASK);
+                    const uint32_t cntP = P == 0 ? si.nF : P == 1 ? si.nB : si.nO;
+                    for (uint32_t q = 0; q < cntP; q++)
+                        if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig++; break; }
+                    sum = 0;
+                    Sb = 0.0;
+                    open = false;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    // pass 3: receive lists, TP waits of same-stage readers, TP gates of sends
+    if (tid < S) {
+        const int s = tid;
+        const StageInfo si = SI[s];
+        const HStage hs = HS[s];
+        const uint32_t tcnt[3] = {hs.TF, hs.TB, hs.TO};
+        const uint32_t toff[3] = {hs.tcol_off, hs.tcol_off + hs.TF, hs.tcol_off + hs.TF + hs.TB};
+        uint32_t rv = si.recv_off;
+        const uint32_t total = si.nF + si.nB + si.nO;
+        for (uint32_t q = 0; q < total; q++) {
+            HEnt &en = ents[si.ent_off + q];
+            const triosim_op op = T.ops[en.op];
+            en.recv_off = rv;
+            uint32_t nr = 0;
+            int32_t tpw = -1;
+            for (uint32_t k = 0; k < op.n_in; k++) {
+                const uint32_t x = T.io[op.io_off + k];
+                const int32_t po = T.prod[x];
+                if (po < 0) continue;
+                const int ps = s_stage[T.layer[po]];
+                const int pph = (int)(T.info[po] & INFO_PHASE_MASK);
+                if (ps == s) {
+                    if (tp > 1)
+                        for (uint32_t e = 0; e < tcnt[pph]; e++)
+                            if (colls[toff[pph] + e].pad == x) {
+                                const int32_t key = (pph << 24) | (int32_t)e;
+                                if (key > tpw) tpw = key;
+                                break;
+                            }
+                    continue;
+                }
+                const StageInfo pi = SI[ps];
+                const uint32_t base = pi.send_off + (pph == 0 ? 0 : pph == 1 ? pi.SF : pi.SF + pi.SB);
+                const uint32_t cnt = pph == 0 ? pi.SF : pph == 1 ? pi.SB : pi.SO;
+                uint32_t e = 0;
+                while (e < cnt && !(sends[base + e].x == x && sends[base + e].dst == s)) e++;
+                RecvEnt re;
+                re.src = (uint16_t)ps;
+                re.phase = (uint8_t)pph;
+                re.pad = 0;
+                re.e = e;
+                recvs[rv++] = re;
+                nr++;
+            }
+            en.nrecv = (uint16_t)nr;
+            en.tpw = tpw;
+        }
+        if (tp > 1) {
+            const uint32_t scnt = si.SF + si.SB + si.SO;
+            for (uint32_t q = 0; q < scnt; q++) {
+                HSend &se = sends[si.send_off + q];
+                const int P = q < si.SF ? 0 : q < si.SF + si.SB ? 1 : 2;
+                for (uint32_t e = 0; e < tcnt[P]; e++)
+                    if (colls[toff[P] + e].pad == se.x) { se.tpg = (P << 24) | (int32_t)e; break; }
+            }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        // class totals; collective payloads folded in canonical creation order (R9): TP groups
+        // (d, s) then DP groups (s, t)
+        uint64_t ncomp = 0, nflow = 0, ncoll = 0;
+        uint32_t pmax = 0, any_ag = 0, any_ar = 0;
+        double payload = 0.0;
+        for (int s = 0; s < S; s++) {
+            const uint32_t prog = m * (SI[s].nF + SI[s].nB) + SI[s].nO;
+            ncomp += (uint64_t)prog * dp * tp;
+            if (prog > pmax) pmax = prog;
+            nflow += ((uint64_t)m * (SI[s].SF + SI[s].SB) + SI[s].SO) * dp * tp;
+        }
+        for (int d = 0; d < dp && tp > 1; d++)
+            for (int s = 0; s < S; s++) {
+                const HStage hs = HS[s];
+                const uint32_t part[3][2] = {{hs.tcol_off, hs.TF}, {hs.tcol_off + hs.TF, hs.TB},
+                                             {hs.tcol_off + hs.TF + hs.TB, hs.TO}};
+                for (uint32_t j = 0; j < m; j++)
+                    for (uint32_t e = 0; e < part[0][1]; e++) payload = payload + colls[part[0][0] + e].S;
+                for (uint32_t j = 0; j < m; j++)
+                    for (uint32_t e = 0; e < part[1][1]; e++) payload = payload + colls[part[1][0] + e].S;
+                for (uint32_t e = 0; e < part[2][1]; e++) payload = payload + colls[part[2][0] + e].S;
+                for (uint32_t e = 0; e < hs.TF + hs.TB + hs.TO; e++) {
+                    const uint32_t kind = colls[hs.tcol_off + e].kind;
+                    const uint64_t reps = e < hs.TF + hs.TB ? m : 1;
+                    const uint64_t per = kind == CK_AG ? (uint64_t)(tp - 1) * tp
+                                       : C.algo == TRIOSIM_ALGO_TREE ? 2ull * (tp - 1) : 2ull * (tp - 1) * tp;
+                    nflow += reps * per;
+                    ncoll += reps;
+                    if (kind == CK_AG) any_ag = 1; else any_ar = 1;
+                }
+            }
+        for (int s = 0; s < S && dp > 1; s++)
+            for (int t = 0; t < tp; t++)
+                for (uint32_t b = 0; b < HS[s].ndp; b++) {
+                    payload = payload + colls[HS[s].dcol_off + b].S;
+                    nflow += C.algo == TRIOSIM_ALGO_TREE ? 2ull * (dp - 1) : 2ull * (dp - 1) * dp;
+                    ncoll++;
+                    any_ar = 1;
+                }
+        C.n_compute = ncomp;
+        C.n_flows = nflow;
+        C.n_coll = (uint32_t)ncoll;
+        C.coll_payload = payload;
+        C.n_prog_max = pmax;
+        C.need_ring = any_ag || (any_ar && C.algo == TRIOSIM_ALGO_RING);
+        C.need_tree = any_ar && C.algo == TRIOSIM_ALGO_TREE;
+    }
+}
+
+cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
+                             const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
+                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    k2_hybrid<<<n, K2P_THREADS, 0, s>>>(cls, list, T, plan_pool, stages, hst, ents, sends, recvs, colls, scratch);
+    return cudaGetLastError();
+}
+
 }  // namespace ts

@@ -81,6 +81,32 @@ def test_random_small_all_strategies(ctx, seed):
     assert (got["status"] == 0).sum() > 300
 
 
+@pytest.mark.parametrize("seed", range(4))
+def test_random_hybrid(ctx, seed):
+    """HYBRID DP x TP x PP (R9) on random traces / topologies: every degree split, both TP modes,
+    ring and tree, buckets, micro-batches; compared point by point with the oracle."""
+    rng = np.random.Generator(np.random.PCG64(900 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=2)
+    topos = [W.random_topology(rng, n_gpus=g, n_switch=int(rng.integers(0, 3)), p_edge=0.2) for g in (4, 8, 12)]
+    topos += [W.star(16, 50e9, 1e-6), W.mesh(4, 4, 40e9, 2e-6), W.perturb(W.cube_mesh8(60e9, 1e-6), seed)]
+    pts = []
+    for _ in range(250):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        while True:
+            dp, tp, pp = (int(rng.integers(1, 5)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 4)))
+            if dp * tp * pp <= G and pp <= tr.n_layers:
+                break
+        m = int(rng.integers(1, 4))
+        pts.append(W.make_point(ti, W.ST_HYBRID, dp=dp, tp=tp, pp=pp, m=m, B=dp * m * int(rng.integers(1, 3)),
+                                bucket=int(rng.choice([0, 1 << 12, 1 << 30])), tp_mode=int(rng.integers(0, 2)),
+                                algo=int(rng.integers(0, 2)), bw=float(rng.uniform(0.3, 3)), lat=float(rng.uniform(0, 2))))
+    sw = W.Sweep("hyb", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    check(got, sw, list(range(len(pts))))
+    assert (got["status"] == 0).sum() > 200
+
+
 def test_statuses_and_edge_cases(ctx):
     tr = W.mlp_trace()
     topos = [W.ring(4, 10e9, 1e-6), W.ring(32, 10e9, 1e-6), W.ring(40, 10e9, 1e-6), W.star(32, 10e9, 1e-6)]
@@ -97,7 +123,7 @@ def test_statuses_and_edge_cases(ctx):
         P(0, W.ST_PP, pp=2, m=1, B=4, plan=7),           # plan index out of range
         P(9, W.ST_DP, dp=1, B=1),                        # topology out of range
         P(0, 7, dp=1, B=1),                              # unknown strategy
-        P(0, W.ST_HYBRID, dp=2, tp=2, pp=1, m=1, B=4),   # hybrid: reserved
+        P(0, W.ST_HYBRID, dp=2, tp=2, pp=1, m=1, B=4),   # hybrid DP x TP
         P(0, W.ST_DP, dp=1, B=64, bw=-1.0),              # bad scale
         P(3, W.ST_DDP, dp=2, B=128),                     # no route back
         P(1, W.ST_DDP, dp=32, B=32 * 64, bucket=1 << 20),  # 32 lanes: W = 32
@@ -109,7 +135,7 @@ def test_statuses_and_edge_cases(ctx):
     sw = W.Sweep("edge", tr, topos, pts, plans=[[0, 2], [0, 0]])
     got = ctx.run_sweep(sw)
     check(got, sw, list(range(len(pts))))
-    assert list(got["status"][:11]) == [1, 2, 1, 0, 6, 6, 7, 7, 7, 7, 3]
+    assert list(got["status"][:11]) == [1, 2, 1, 0, 6, 6, 7, 7, 0, 7, 3]
     # beyond the warp kernel's limits -- more than 32 lanes, a route longer than 8 hops (tree
     # edges across a 32-GPU ring) -- is reported, never silently wrong
     big = W.Sweep("big", tr, topos, W.points_array([P(2, W.ST_DDP, dp=40, B=40 * 64),
