@@ -31,13 +31,15 @@ from paper_conf_isca_libwmvgjbj025_b200 import workloads as W  # noqa: E402
 
 METRIC = "simulated design points/sec"
 UNIT = "points/s"
-CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1}
+CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1, "c5": W.sweep_c5}
 WORKLOAD = {"c2": "configs[1]: ResNet-50 DP/DDP, 2-16 simulated GPUs on an NVLink-style ring, 10k-point "
                   "bandwidth x latency x batch x bucket sweep",
             "c3": "configs[2]: BERT-large Megatron/paper TP 2/4/8, ring/star/mesh/cube-mesh/ring-graph/"
                   "double-ring topologies incl. asymmetric",
             "c4": "configs[3]: GPT-2 XL GPipe 4-16 stages x 8-64 micro-batches on 2D meshes",
-            "c1": "configs[0]: 4-layer MLP DDP on 2 GPUs, one uniform link"}
+            "c1": "configs[0]: 4-layer MLP DDP on 2 GPUs, one uniform link",
+            "c5": "configs[4] (<= 32 simulated GPUs): GPT-3-class DP x TP x PP, hierarchical 2:1 / 4:1 "
+                  "topology incl. a seeded slow-link subset"}
 FP64_LANES_PER_SM = 64     # B200 FP64 pipe: 64 DFMA/DADD/DMUL lanes per SM per clock
 N_SMS = 148
 

@@ -477,7 +477,8 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
                              : pt.strategy == TRIOSIM_HYBRID ? dp * tpd * pp : dp;
         int W = 2;
         while (W < (int)lanes) W <<= 1;
-        while (W <= 32 && (int)tp.n_links > std::max(8, 4 * W)) W <<= 1;
+        const bool hyb_pt = pt.strategy == TRIOSIM_HYBRID;
+        while (W <= 32 && (int)tp.n_links > (hyb_pt ? lmax_hybrid(W) : lmax_warp(W))) W <<= 1;
         if (W > 32) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
         // structural class
         const bool hyb = pt.strategy == TRIOSIM_HYBRID;

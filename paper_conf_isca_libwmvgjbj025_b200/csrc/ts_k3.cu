@@ -116,7 +116,7 @@ __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[
 template <int W, int MODE>
 __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Args a) {
     constexpr int NSEG = 32 / W;
-    constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
+    constexpr int LMAX = lmax_warp(W);
     constexpr bool COLL = MODE != MODE_PIPE;   // DP / DDP / TP collectives
     constexpr bool TREE = MODE == MODE_TREE;   // ... some of which may be tree AllReduces
     __shared__ double s_res[K3_WARPS][NSEG * LMAX];

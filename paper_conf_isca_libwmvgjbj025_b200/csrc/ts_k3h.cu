@@ -113,7 +113,7 @@ __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f,
 template <int W>
 __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
     constexpr int NSEG = 32 / W;
-    constexpr int LMAX = (4 * W < 8) ? 8 : 4 * W;
+    constexpr int LMAX = lmax_hybrid(W);
     __shared__ double s_res[K3_WARPS][NSEG * LMAX];
     __shared__ int s_n[K3_WARPS][NSEG * LMAX];
     __shared__ int s_k[K3_WARPS][NSEG * LMAX];

@@ -439,6 +439,11 @@ def gpt2_xl_trace(b0=8, seed=4) -> Trace:
     return transformer_trace("gpt2-xl", 48, 1600, 25, 6400, 1024, 50257, b0, seed, causal_head=True)
 
 
+def gpt3_trace(n_layers=96, b0=1, seed=5) -> Trace:
+    """GPT-3-class decoder (h = 12288, 96 heads, seq 2048, fp16 activations), configs[4]."""
+    return transformer_trace("gpt3-175b", n_layers, 12288, 96, 4 * 12288, 2048, 50257, b0, seed, causal_head=True)
+
+
 def random_trace(rng, n_layers=3, max_ops_per_layer=3, b0=4, max_time=1e-3, bytes_hi=1 << 20, dyadic=False,
                  roles=True) -> Trace:
     """Small random layered trace with FWD/BWD/OPT structure, for property tests."""
@@ -564,6 +569,38 @@ def double_ring(p, bw=1.0, lat=1.0):
             e += [(base + i, base + (i + h // 2) % h, bw, lat) for i in range(h // 2)]
     e += [(i, i + h, bw, lat) for i in range(h)]
     return _mk(f"doublering{p}", p, p, e, list(range(h)) + list(range(p - 1, h - 1, -1)))
+
+
+def hierarchical(n_nodes, gpus_per_node=8, intra=1.0, nic=0.1, oversub=2.0, lat_intra=1.0, lat_nic=2.0,
+                 lat_spine=2.0, nodes_per_leaf=2, n_spines=1):
+    """configs[4]'s hierarchical topology: nodes of `gpus_per_node` GPUs on an NVSwitch-like node switch
+    (bandwidth `intra`), every GPU also on a NIC link (`nic`) to its leaf switch, leaves to `n_spines`
+    spine switches with 1/`oversub` of the leaf's NIC bandwidth.  Node switches are numbered before
+    leaves, so intra-node routes go through the node switch (R12's lexicographic tie break)."""
+    G = n_nodes * gpus_per_node
+    n_leaves = (n_nodes + nodes_per_leaf - 1) // nodes_per_leaf
+    node_sw = [G + k for k in range(n_nodes)]
+    leaf = [G + n_nodes + k for k in range(n_leaves)]
+    spine = [G + n_nodes + n_leaves + k for k in range(n_spines)]
+    e = []
+    for g in range(G):
+        k = g // gpus_per_node
+        e.append((g, node_sw[k], intra, lat_intra))
+        e.append((g, leaf[k // nodes_per_leaf], nic, lat_nic))
+    up = nic * gpus_per_node * nodes_per_leaf / oversub / n_spines
+    for lf in leaf:
+        for sp in spine:
+            e.append((lf, sp, up, lat_spine))
+    return _mk(f"hier{n_nodes}x{gpus_per_node}o{oversub:g}", G + n_nodes + n_leaves + n_spines, G, e, list(range(G)))
+
+
+def perturb_subset(topo: Topology, seed: int, frac=0.25) -> Topology:
+    """P:356's random slow-down (bandwidth / U[1,10]) applied to a seeded subset of the links."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    links = topo.links.copy()
+    sel = rng.random(len(links)) < frac
+    links["bw_Bps"][sel] = links["bw_Bps"][sel] / rng.uniform(1.0, 10.0, int(sel.sum()))
+    return Topology(f"{topo.name}~s{seed}", topo.n_nodes, topo.n_gpus, links, topo.ring_order.copy())
 
 
 def perturb(topo: Topology, seed: int) -> Topology:
@@ -697,3 +734,36 @@ def sweep_c4(trace=None, seed=4, n_bw=25, n_lat=8) -> Sweep:
     arr = points_array(pts)
     perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
     return Sweep("c4_gpt2xl_pp", tr, topos, arr[perm])
+
+
+def sweep_c5(trace=None, seed=5, max_gpus=32, n_bw=4, n_lat=2) -> Sweep:
+    """configs[4] within the warp kernel's 32-GPU limit: GPT-3-class HYBRID DP x TP x PP on 8-32
+    simulated GPUs of a hierarchical topology (2:1 / 4:1 oversubscribed, also with a seeded slow
+    link subset), every (TP, PP, DP) split with TP <= 8 inside a node and TP*PP >= 4, micro-batches
+    8-32, 2 GiB gradient buckets."""
+    tr = trace if trace is not None else gpt3_trace()
+    topos, pts = [], []
+    for N in (8, 16, 32):
+        if N > max_gpus:
+            continue
+        for ov in (2.0, 4.0):
+            base = hierarchical(max(N // 8, 1), 8, intra=1.0, nic=0.125, oversub=ov)
+            for asym in (0, 1):
+                ti = len(topos)
+                topos.append(base if asym == 0 else perturb_subset(base, 500 + 10 * N + int(ov)))
+                for tp in (1, 2, 4, 8):
+                    for pp in (1, 2, 4, 8, 16):
+                        if N % (tp * pp) or pp > tr.n_layers or tp * pp < 4:
+                            continue   # a 175B model needs >= 4-way model parallelism to fit
+                        dp = N // (tp * pp)
+                        for m in (8, 16, 32):
+                            if pp == 1 and m > 8:
+                                continue
+                            for bw in np.logspace(np.log10(100e9), np.log10(900e9), n_bw):
+                                for lat in np.logspace(np.log10(1e-6), np.log10(5e-6), n_lat):
+                                    pts.append(make_point(ti, ST_HYBRID, dp=dp, tp=tp, pp=pp, m=m, B=dp * m,
+                                                          bucket=2048 * MiB, bw=float(bw), lat=float(lat)))
+    arr = points_array(pts)
+    perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
+    return Sweep("c5_gpt3_hybrid", tr, topos, arr[perm])
+

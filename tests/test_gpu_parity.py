@@ -217,3 +217,16 @@ def test_c4_gpt2xl_pp_sampled(ctx):
     # cheap points plus a few of the largest (S=16, m=64)
     big = [i for i, pt in enumerate(sw.points) if pt["pp"] == 16 and pt["microbatches"] == 64][:3]
     check(got, sw, sorted(set(sample(len(sw.points), 300, 4) + big)))
+
+
+def test_c5_gpt3_hybrid_sampled(ctx):
+    """configs[4] (GPT-3-class DP x TP x PP on a hierarchical asymmetric topology, 8-32 GPUs): a seeded
+    subset of the lighter points (m = 8; the heaviest points have ~2M instants each) on the GPU, every
+    point must simulate, 16 of them against the oracle."""
+    full = W.sweep_c5()
+    light = [i for i, p in enumerate(full.points) if p["microbatches"] == 8 and p["tp"] <= 4]
+    sub = [light[i] for i in sample(len(light), 120, 55)]
+    sw = W.Sweep(full.name, full.trace, full.topos, full.points[sub])
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all(), np.unique(got["status"], return_counts=True)
+    check(got, sw, sample(len(sw.points), 16, 5))
