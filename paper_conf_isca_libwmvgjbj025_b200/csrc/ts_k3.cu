@@ -575,13 +575,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
             }
             const bool anygen = __any_sync(FULL, gen);
             if (anygen) {
+                // link counters are 0 here: every complete progressive filling returns them to 0
                 if (gen) {
                     alg += flen;
-#pragma unroll
-                    for (int h = 0; h < MAX_HOPS; h++) if (h < flen) ln[hop(hl, h)] = 0;
-                }
-                __syncwarp();
-                if (gen) {
 #pragma unroll
                     for (int h = 0; h < MAX_HOPS; h++)
                         if (h < flen) {

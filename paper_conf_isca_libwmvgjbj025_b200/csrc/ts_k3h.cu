@@ -539,77 +539,116 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
             progress(FT, aT);
             progress(FD, aD);
             progress(FP, aP);
-            auto zero = [&](const Flow &F, bool on) {
-                if (on)
-                    for (int h = 0; h < F.len; h++) ln[hop(F.hl, h)] = 0;
-            };
-            zero(FT, aT);
-            zero(FD, aD);
-            zero(FP, aP);
-            __syncwarp();
+            // link counters are 0 here: every complete progressive filling returns them to 0
             auto count = [&](const Flow &F, bool on) {
                 if (on) {
                     alg += F.len;
-                    for (int h = 0; h < F.len; h++) {
-                        const int e = hop(F.hl, h);
-                        atomicAdd(&ln[e], 1);
-                        lres[e] = a.link_bw[TR.link_off + e] * bws;
-                    }
+#pragma unroll
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if (h < F.len) {
+                            const int e = hop(F.hl, h);
+                            atomicAdd(&ln[e], 1);
+                            lres[e] = a.link_bw[TR.link_off + e] * bws;
+                        }
                 }
             };
             count(FT, aT);
             count(FD, aD);
             count(FP, aP);
             __syncwarp();
-            bool uT = aT, uD = aD, uP = aP;
-            uint32_t rounds = 0;
+            // if no link carries two active flows, R14 is exactly "rate = smallest residual on the
+            // route" (n_e = 1: res_e / 1.0 == res_e) and the rounds are the distinct rates
+            auto alone = [&](const Flow &F, bool on) -> bool {
+                bool ok = true;
+                if (on) {
+#pragma unroll
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if (h < F.len && ln[hop(F.hl, h)] != 1) ok = false;
+                }
+                return ok;
+            };
+            const bool disj = (__ballot_sync(FULL, alone(FT, aT) && alone(FD, aD) && alone(FP, aP)) & smask) == smask;
             auto fmin = [&](const Flow &F, bool on) -> double {
                 double my = dinf();
                 if (on) {
-                    for (int h = 0; h < F.len; h++) {
-                        const int e = hop(F.hl, h);
-                        const double sh = lres[e] / (double)ln[e];
-                        my = sh < my ? sh : my;
-                    }
+#pragma unroll
+                    for (int h = 0; h < MAX_HOPS; h++)
+                        if (h < F.len) {
+                            const int e = hop(F.hl, h);
+                            const double sh = lres[e] / (double)ln[e];
+                            my = sh < my ? sh : my;
+                        }
                     alg += 2 * F.len;
                 }
                 return my;
             };
+            if (disj) {
+                auto solo = [&](Flow &F, bool on) {
+                    if (on) {
+                        F.rate = fmin(F, true);
+#pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if (h < F.len) ln[hop(F.hl, h)] = 0;
+                    }
+                };
+                solo(FT, aT);
+                solo(FD, aD);
+                solo(FP, aP);
+            }
+            __syncwarp();
+            bool uT = aT, uD = aD, uP = aP;
+            uint32_t rounds = 0;
             while (__any_sync(FULL, uT || uD || uP)) {
                 const bool segact = (__ballot_sync(FULL, uT || uD || uP) & smask) != 0;
-                const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
+                double mT, mD, mP;
+                if (disj) {
+                    mT = uT ? FT.rate : dinf();
+                    mD = uD ? FD.rate : dinf();
+                    mP = uP ? FP.rate : dinf();
+                } else {
+                    mT = fmin(FT, uT);
+                    mD = fmin(FD, uD);
+                    mP = fmin(FP, uP);
+                }
                 double my = mT < mD ? mT : mD;
                 my = mP < my ? mP : my;
                 const double sm = seg_min<W>(my);
                 const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
                 unsigned own = 0;
-                auto freeze = [&](Flow &F, bool in, int slot) {
-                    if (in) {
-                        F.rate = sm;
-                        for (int h = 0; h < F.len; h++)
-                            if (atomicAdd(&lk[hop(F.hl, h)], 1) == 0) own |= 1u << (slot * 8 + h);
-                    }
-                };
-                freeze(FT, iT, 0);
-                freeze(FD, iD, 1);
-                freeze(FP, iP, 2);
-                __syncwarp();
-                auto update = [&](const Flow &F, int slot) {
-                    for (int h = 0; h < F.len; h++)
-                        if ((own >> (slot * 8 + h)) & 1u) {
-                            const int e = hop(F.hl, h);
-                            const int kk = lk[e];
-                            const double r = lres[e] - sm * (double)kk;
-                            lres[e] = r > 0.0 ? r : 0.0;
-                            ln[e] -= kk;
-                            lk[e] = 0;
-                            alg += 3;
+                {
+                    // (disj is per segment: every lane still reaches both __syncwarp()s)
+                    auto freeze = [&](Flow &F, bool in, int slot) {
+                        if (in) {
+                            F.rate = sm;
+#pragma unroll
+                            for (int h = 0; h < MAX_HOPS; h++)
+                                if (h < F.len && atomicAdd(&lk[hop(F.hl, h)], 1) == 0) own |= 1u << (slot * 8 + h);
                         }
-                };
-                if (own) {
-                    update(FT, 0);
-                    update(FD, 1);
-                    update(FP, 2);
+                    };
+                    if (!disj) {
+                        freeze(FT, iT, 0);
+                        freeze(FD, iD, 1);
+                        freeze(FP, iP, 2);
+                    }
+                    __syncwarp();
+                    auto update = [&](const Flow &F, int slot) {
+#pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if ((own >> (slot * 8 + h)) & 1u) {
+                                const int e = hop(F.hl, h);
+                                const int kk = lk[e];
+                                const double r = lres[e] - sm * (double)kk;
+                                lres[e] = r > 0.0 ? r : 0.0;
+                                ln[e] -= kk;
+                                lk[e] = 0;
+                                alg += 3;
+                            }
+                    };
+                    if (own) {
+                        update(FT, 0);
+                        update(FD, 1);
+                        update(FP, 2);
+                    }
                 }
                 __syncwarp();
                 if (segact) rounds++;
@@ -656,12 +695,13 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         double cand = dinf();
         if (used) {
             if (cst == CS_RUN) cand = t_end;
-            const Flow *fs[3] = {&FT, &FD, &FP};
-#pragma unroll
-            for (int k = 0; k < 3; k++) {
-                if (fs[k]->st == FS_LAT && fs[k]->t_act < cand) cand = fs[k]->t_act;
-                if (fs[k]->st == FS_ACT && fs[k]->t_drain < cand) cand = fs[k]->t_drain;
-            }
+            auto cf = [&](const Flow &F) {
+                if (F.st == FS_LAT && F.t_act < cand) cand = F.t_act;
+                if (F.st == FS_ACT && F.t_drain < cand) cand = F.t_drain;
+            };
+            cf(FT);
+            cf(FD);
+            cf(FP);
         }
         const double tn = seg_min<W>(cand);
         const bool stuck = have && !fin && !(tn < dinf());
