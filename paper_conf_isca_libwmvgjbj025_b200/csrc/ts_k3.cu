@@ -172,7 +172,8 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
     SI.ent_off = SI.send_off = SI.recv_off = 0;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
-    uint64_t acc = 0, alg = 0;   // acc: this lane's part of the order hash (R19)
+    uint64_t acc = 0;            // this lane's part of the order hash (R19)
+    uint32_t alg = 0;            // fp64 operations of the method performed by this lane (wraps per point only beyond 4e9)
     uint64_t tmix = 0;           // mix64(bits(t)) of the current instant
     bool nev = false;            // this lane recorded an event at the current instant
 
@@ -594,49 +595,51 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
             bool unf = act && !uni;
             const bool segany = (__ballot_sync(FULL, act) & smask) != 0;
             uint32_t rounds = (uni && segany) ? 1u : 0u;
-            while (__any_sync(FULL, unf)) {
-                const bool segact = (__ballot_sync(FULL, unf) & smask) != 0;
-                double my = dinf();
-                if (unf) {
-                    if (fast) {
-                        my = rate;
-                    } else {
-#pragma unroll
-                        for (int h = 0; h < MAX_HOPS; h++)
-                            if (h < flen) {
-                                const int e = hop(hl, h);
-                                const double sh = lres[e] / (double)ln[e];
-                                my = sh < my ? sh : my;
-                            }
-                        alg += 2 * flen;
-                    }
-                }
-                const double s = TS_SEGMIN_REDUX ? seg_min_redux(my, smask) : seg_min_shfl<W>(my);
-                const bool inF = unf && my == s;
-                unsigned own = 0;
-                if (inF && !fast) {
-                    rate = s;
-#pragma unroll
-                    for (int h = 0; h < MAX_HOPS; h++)
-                        if (h < flen && atomicAdd(&lk[hop(hl, h)], 1) == 0) own |= 1u << h;
-                }
-                if (anygen) __syncwarp();
-                if (inF && !fast) {
-#pragma unroll
-                    for (int h = 0; h < MAX_HOPS; h++)
-                        if ((own >> h) & 1u) {
-                            const int e = hop(hl, h);
-                            const int kk = lk[e];
-                            const double r = lres[e] - s * (double)kk;
-                            lres[e] = r > 0.0 ? r : 0.0;
-                            ln[e] -= kk;
-                            lk[e] = 0;
-                            alg += 3;
+            if (__any_sync(FULL, unf)) {   // guard: keeps the loop's hoisted address math off the fast path
+                while (__any_sync(FULL, unf)) {
+                    const bool segact = (__ballot_sync(FULL, unf) & smask) != 0;
+                    double my = dinf();
+                    if (unf) {
+                        if (fast) {
+                            my = rate;
+                        } else {
+    #pragma unroll
+                            for (int h = 0; h < MAX_HOPS; h++)
+                                if (h < flen) {
+                                    const int e = hop(hl, h);
+                                    const double sh = lres[e] / (double)ln[e];
+                                    my = sh < my ? sh : my;
+                                }
+                            alg += 2 * flen;
                         }
+                    }
+                    const double s = TS_SEGMIN_REDUX ? seg_min_redux(my, smask) : seg_min_shfl<W>(my);
+                    const bool inF = unf && my == s;
+                    unsigned own = 0;
+                    if (inF && !fast) {
+                        rate = s;
+    #pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if (h < flen && atomicAdd(&lk[hop(hl, h)], 1) == 0) own |= 1u << h;
+                    }
+                    if (anygen) __syncwarp();
+                    if (inF && !fast) {
+    #pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if ((own >> h) & 1u) {
+                                const int e = hop(hl, h);
+                                const int kk = lk[e];
+                                const double r = lres[e] - s * (double)kk;
+                                lres[e] = r > 0.0 ? r : 0.0;
+                                ln[e] -= kk;
+                                lk[e] = 0;
+                                alg += 3;
+                            }
+                    }
+                    if (anygen) __syncwarp();
+                    if (segact) rounds++;
+                    unf = unf && !inF;
                 }
-                if (anygen) __syncwarp();
-                if (segact) rounds++;
-                unf = unf && !inF;
             }
             const uint32_t nact = __popc(__ballot_sync(FULL, act) & smask);  // (all lanes vote)
             if (segdirty) {
@@ -658,9 +661,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
         if (have && any_ev) ninst++;
         nev = false;
         const bool infl = (__ballot_sync(FULL, used && fst != FS_NONE) & smask) != 0;
-        if (have) {
-            if (infl && !bon) { bon = true; bstart = t; }
-            else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
+        if (have && infl != bon) {   // an interval with >= 1 flow in flight opens or closes (R18)
+            if (bon) cbusy = cbusy + (t - bstart);
+            else bstart = t;
+            bon = !bon;
         }
         bool lane_done = !used || (cst == CS_IDLE && pos >= nprog && fst == FS_NONE);
         if constexpr (!COLL) lane_done = lane_done && (!used || sq >= nsend_tot);
@@ -678,7 +682,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
             const double bmax = seg_max<W>(used ? busy : 0.0);
             const uint32_t ntk = seg_sum_u32<W>(ntask);
             const uint32_t nfl = seg_sum_u32<W>(nflow);
-            const unsigned long long alg_s = seg_sum_u64<W>(alg);
+            const unsigned long long alg_s = seg_sum_u64<W>((unsigned long long)alg);
             const unsigned long long H = seg_sum_u64<W>(acc);
             if ((fin || stuck) && li == 0) {
                 triosim_result r;
