@@ -103,8 +103,8 @@ struct Sweep {
     cudaStream_t last_stream = nullptr;
 };
 
-int w_index(int W) { return W == 2 ? 0 : W == 4 ? 1 : W == 8 ? 2 : W == 16 ? 3 : 4; }
-const int W_OF[5] = {2, 4, 8, 16, 32};
+int w_index(int W) { int i = 0; while ((2 << i) < W) i++; return i; }
+const int W_OF[N_WIDTHS] = {2, 4, 8, 16, 32, 64, 128, 256};
 
 }  // namespace
 
@@ -164,8 +164,8 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
             triosim_destroy(ctx);
             return TRIOSIM_ECUDA;
         }
-        ctx->occ[i] = (i % N_MODES) == MODE_HYBRID ? k3h_max_blocks_per_sm(W_OF[i / N_MODES])
-                                                   : k3_max_blocks_per_sm(W_OF[i / N_MODES], i % N_MODES);
+        const int Wi = W_OF[i / N_MODES], md = i % N_MODES;
+        ctx->occ[i] = md == MODE_HYBRID ? k3h_max_blocks_per_sm(Wi) : Wi <= 32 ? k3_max_blocks_per_sm(Wi, md) : 1;
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
         triosim_destroy(ctx);
@@ -437,7 +437,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     }
 
     for (uint64_t i = 0; i < n_pts; i++) {
-        const triosim_point &pt = pts[i];
+        triosim_point pt = pts[i];
         auto setst = [&](int st) { S->status[i] = st; };
         // R3, in order
         if (pt.topo >= n_topos) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
@@ -472,24 +472,40 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             if (!ok) { setst(TRIOSIM_PT_BAD_PLAN); continue; }
             plan_key = pt.stage_plan;
         }
-        // GPU kernel limits
+        // GPU kernel limits: warp segments (<= 32 lanes, lmax_warp links) for DP / DDP / TP / PP; the
+        // HYBRID kernel (warp segments up to 32 ranks, one point per CTA up to 256 ranks, LMAX_CTA links)
+        // for HYBRID and for DDP / TP / PP points beyond the warp kernels -- DDP = (dp,1,1,1),
+        // TP = (1,tp,1,1), PP = (1,1,pp,m) reproduce those strategies bit for bit (R9, pinned)
         const uint32_t lanes = pt.strategy == TRIOSIM_TP ? tpd : pt.strategy == TRIOSIM_PP ? pp
                              : pt.strategy == TRIOSIM_HYBRID ? dp * tpd * pp : dp;
-        int W = 2;
-        while (W < (int)lanes) W <<= 1;
-        const bool hyb_pt = pt.strategy == TRIOSIM_HYBRID;
-        while (W <= 32 && (int)tp.n_links > (hyb_pt ? lmax_hybrid(W) : lmax_warp(W))) W <<= 1;
-        if (W > 32) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
+        auto lm = [&](bool h, int w) { return !h ? lmax_warp(w) : w <= 32 ? lmax_hybrid(w) : LMAX_CTA; };
+        int W0 = 2;
+        while (W0 < (int)lanes) W0 <<= 1;
+        int W = 0;
+        if (pt.strategy != TRIOSIM_HYBRID)
+            for (int w = W0; w <= 32; w <<= 1)
+                if ((int)tp.n_links <= lm(false, w)) { W = w; break; }
+        if (W == 0 && (pt.strategy == TRIOSIM_HYBRID || pt.strategy == TRIOSIM_DDP || pt.strategy == TRIOSIM_TP ||
+                       pt.strategy == TRIOSIM_PP)) {
+            if (pt.strategy != TRIOSIM_HYBRID) {
+                if (pt.strategy != TRIOSIM_PP) pt.microbatches = 1;
+                pt.strategy = TRIOSIM_HYBRID;
+            }
+            for (int w = W0; w <= 256; w <<= 1)
+                if ((int)tp.n_links <= lm(true, w)) { W = w; break; }
+        }
+        if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
+        const uint32_t mbe = pt.microbatches;   // after a DDP / TP -> HYBRID mapping this is 1
         // structural class
         const bool hyb = pt.strategy == TRIOSIM_HYBRID;
         const int mode = hyb ? MODE_HYBRID : pt.strategy == TRIOSIM_PP ? MODE_PIPE : MODE_COLL;
         uint32_t b_loc = pt.strategy == TRIOSIM_TP ? pt.global_batch
-                       : pt.strategy == TRIOSIM_PP ? pt.global_batch / mb
-                       : hyb ? pt.global_batch / (dp * mb) : pt.global_batch / dp;
+                       : pt.strategy == TRIOSIM_PP ? pt.global_batch / mbe
+                       : hyb ? pt.global_batch / (dp * mbe) : pt.global_batch / dp;
         int key_mode = (pt.strategy == TRIOSIM_TP || hyb) ? pt.tp_mode : 0;
         int key_algo = mode != MODE_PIPE ? pt.coll_algo : 0;
         uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP || hyb) ? pt.bucket_bytes : 0;
-        int key_m = (mode == MODE_PIPE || hyb) ? (int)mb : 0;
+        int key_m = (mode == MODE_PIPE || hyb) ? (int)mbe : 0;
         auto key = std::make_tuple((int)pt.strategy, (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
                                    hyb ? (int)tpd : 0, key_algo, key_bucket, key_m,
                                    (mode == MODE_PIPE || hyb) ? plan_key : -2);
@@ -503,7 +519,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.tp_mode = key_mode;
             cd.algo = key_algo;
             cd.p = hyb ? pp : lanes;
-            cd.m = (mode == MODE_PIPE || hyb) ? mb : 1;
+            cd.m = (mode == MODE_PIPE || hyb) ? mbe : 1;
             cd.tpdeg = (pt.strategy == TRIOSIM_TP || hyb) ? tpd : 1;
             cd.dp = hyb ? dp : 1;
             cd.b_loc = b_loc;
@@ -541,9 +557,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
                         : (key_bucket == 0 ? T.n_wgrad : std::ceil((double)T.wgrad_bytes / (double)key_bucket));
             cost = (double)N * 2 + ncol * 2.0 * lanes * 8.0;
         } else if (hyb) {
-            cost = (double)mb * N * 2.0 / pp + (double)mb * 16.0 * lanes;
+            cost = (double)mbe * N * 2.0 / pp + (double)mbe * 16.0 * lanes;
         } else {
-            cost = (double)mb * N * 2.0 / lanes + (double)mb * 2.0 * 8.0 * lanes;
+            cost = (double)mbe * N * 2.0 / lanes + (double)mbe * 2.0 * 8.0 * lanes;
         }
         S->cost[i] = cost;
     }
@@ -741,9 +757,14 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         a.hst = S.d_hst.p; a.hents = S.d_hents.p; a.hsends = S.d_hsends.p;
         a.out = S.d_res.p;
         a.alg_ops = S.d_alg.p;
-        const int nseg = 32 / W;
-        const uint64_t warps = (n + nseg - 1) / nseg;
-        uint64_t blocks = (warps + K3_WARPS - 1) / K3_WARPS;
+        uint64_t blocks;
+        if (W <= 32) {
+            const int nseg = 32 / W;
+            const uint64_t warps = (n + nseg - 1) / nseg;
+            blocks = (warps + K3_WARPS - 1) / K3_WARPS;
+        } else {
+            blocks = n;   // one point per CTA
+        }
         const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)ctx->occ[w];
         if (blocks > cap) blocks = cap;
         CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));

@@ -174,7 +174,8 @@ int k3_max_blocks_per_sm(int W, int mode);
 // links per segment the K3 kernels keep in shared memory
 __host__ __device__ constexpr int lmax_warp(int W) { return 4 * W < 8 ? 8 : 4 * W; }
 __host__ __device__ constexpr int lmax_hybrid(int W) { return 8 * W < 16 ? 16 : 8 * W; }
-constexpr int N_WIDTHS = 5;             // W = 2, 4, 8, 16, 32
+constexpr int LMAX_CTA = 2048;          // links of a one-point-per-CTA hybrid segment
+constexpr int N_WIDTHS = 8;             // W = 2, 4, 8, 16, 32 (warp segments), 64, 128, 256 (hybrid CTAs)
 constexpr int N_MODES = 4;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 

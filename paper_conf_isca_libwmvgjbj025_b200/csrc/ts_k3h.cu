@@ -1,6 +1,7 @@
 // ts_k3h.cu -- K3 for HYBRID DP x TP x PP points (R9; Table 1).
 //
-// One point per W-lane segment; lane r = rank (d, s, t) with r = (d*pp + s)*tp + t.  Each lane
+// One point per segment: W lanes of a warp (NW = 1), or NW whole warps = one CTA (NW = 2..8, up to
+// 256 ranks).  Lane r = rank (d, s, t) with r = (d*pp + s)*tp + t.  Each lane
 // runs its stage's GPipe program (R8) and owns THREE flow slots: its TP-group collective step,
 // its DP-group collective step and its FIFO P2P send.  The TP group {(d,s,.)} is a contiguous lane
 // range, the DP group {(.,s,t)} a strided one; both run R10's ring / tree collectives through one
@@ -64,13 +65,38 @@ struct Flow {
     uint64_t code;
 };
 
+// bits over the lanes of one segment
+template <int NW>
+struct Mask {
+    uint32_t w[NW];
+    __device__ __forceinline__ bool test(int k) const { return (w[k >> 5] >> (k & 31)) & 1u; }
+    __device__ __forceinline__ bool covers(const Mask &m) const {
+        bool ok = true;
+#pragma unroll
+        for (int i = 0; i < NW; i++) ok = ok && ((w[i] & m.w[i]) == m.w[i]);
+        return ok;
+    }
+    __device__ __forceinline__ bool any() const {
+        uint32_t x = 0;
+#pragma unroll
+        for (int i = 0; i < NW; i++) x |= w[i];
+        return x != 0;
+    }
+    __device__ __forceinline__ uint32_t popc() const {
+        uint32_t x = 0;
+#pragma unroll
+        for (int i = 0; i < NW; i++) x += __popc(w[i]);
+        return x;
+    }
+};
 // one collective group (TP or DP) as seen by one member lane
+template <int NW>
 struct Group {
     bool member;
     int p, i;                 // group size, my member index
-    int lane0, stride;        // lane of member k = lane0 + k * stride
-    int pred;                 // lane of member (i - 1) mod p
-    unsigned mask;            // lanes of the group
+    int lane0, stride;        // segment lane of member k = lane0 + k * stride
+    int pred;                 // segment lane of member (i - 1) mod p
+    Mask<NW> mask;            // lanes of the group
     uint64_t gid;
     uint32_t ncoll, trig, donec, cur;
     bool running, tree_cur, ldone, uprel, upd, dnrel, dnd, fup;
@@ -110,24 +136,118 @@ __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f,
 
 }  // namespace
 
-template <int W>
-__global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
-    constexpr int NSEG = 32 / W;
-    constexpr int LMAX = lmax_hybrid(W);
-    __shared__ double s_res[K3_WARPS][NSEG * LMAX];
-    __shared__ int s_n[K3_WARPS][NSEG * LMAX];
-    __shared__ int s_k[K3_WARPS][NSEG * LMAX];
-    __shared__ uint32_t s_cnt[K3_WARPS][32];
+
+template <int W, int NW>
+__global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(const K3Args a) {
+    constexpr int SL = NW == 1 ? W : 32 * NW;           // lanes per segment
+    constexpr int NSEG = NW == 1 ? 32 / W : 1;          // segments per warp (NW = 1)
+    constexpr int LMAX = NW == 1 ? lmax_hybrid(W) : LMAX_CTA;
+    constexpr int NSLOT = NW == 1 ? K3_WARPS : 1;       // segment-array slots of the block
+    __shared__ double s_res[NSLOT][NSEG * LMAX];
+    __shared__ int s_n[NSLOT][NSEG * LMAX];
+    __shared__ int s_k[NSLOT][NSEG * LMAX];
+    __shared__ uint32_t s_cnt[NSLOT][NW == 1 ? 32 : SL];
+    __shared__ uint32_t s_bal[2][NW];
+    __shared__ double s_red[2][NW];
+    __shared__ unsigned long long s_red64[2][NW];
+    __shared__ int s_xch[2][NW == 1 ? 1 : SL];
+    __shared__ uint32_t s_item;
 
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int seg = lane / W, li = lane % W, sbase = seg * W;
-    const unsigned smask = (W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase;
-    double *lres = &s_res[wid][seg * LMAX];
-    int *ln = &s_n[wid][seg * LMAX];
-    int *lk = &s_k[wid][seg * LMAX];
-    uint32_t *cnt = &s_cnt[wid][0];   // indexed by warp lane
-    for (int q = lane; q < NSEG * LMAX; q += 32) { s_n[wid][q] = 0; s_k[wid][q] = 0; }
-    __syncwarp();
+    const int seg = NW == 1 ? lane / W : 0;
+    const int li = NW == 1 ? lane % W : (int)threadIdx.x;     // lane inside the segment
+    const int sbase = NW == 1 ? seg * W : 0;                 // segment's first warp lane (NW = 1)
+    const unsigned smask = NW == 1 ? ((W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase) : FULL;
+    const int slot = NW == 1 ? wid : 0;
+    double *lres = &s_res[slot][seg * LMAX];
+    int *ln = &s_n[slot][seg * LMAX];
+    int *lk = &s_k[slot][seg * LMAX];
+    uint32_t *cnt = &s_cnt[slot][sbase];                     // indexed by segment lane
+    for (int q = (NW == 1 ? lane : (int)threadIdx.x); q < NSEG * LMAX; q += (NW == 1 ? 32 : 32 * NW)) {
+        s_n[slot][q] = 0;
+        s_k[slot][q] = 0;
+    }
+    int bb = 0;   // double-buffer toggle of the block-level exchanges (NW > 1)
+
+    // ---- segment primitives: a segment is W lanes of a warp, or the whole CTA ----
+    auto ssync = [&]() {
+        if constexpr (NW == 1) __syncwarp(); else __syncthreads();
+    };
+    auto vany = [&](bool p) -> bool {          // any lane of the warp / CTA (loop control)
+        if constexpr (NW == 1) return __any_sync(FULL, p); else return __syncthreads_or(p) != 0;
+    };
+    auto vall = [&](bool p) -> bool {
+        if constexpr (NW == 1) return __all_sync(FULL, p); else return __syncthreads_and(p) != 0;
+    };
+    auto bal = [&](bool p) -> Mask<NW> {       // segment ballot, bit k = segment lane k
+        Mask<NW> m;
+        if constexpr (NW == 1) {
+            m.w[0] = (__ballot_sync(FULL, p) & smask) >> sbase;
+        } else {
+            const unsigned b = __ballot_sync(FULL, p);
+            if (lane == 0) s_bal[bb][wid] = b;
+            __syncthreads();
+#pragma unroll
+            for (int i = 0; i < NW; i++) m.w[i] = s_bal[bb][i];
+            bb ^= 1;
+        }
+        return m;
+    };
+    auto sany = [&](bool p) -> bool { return bal(p).any(); };
+    auto smin = [&](double v) -> double {
+        if constexpr (NW == 1) {
+            return seg_min<W>(v);
+        } else {
+            v = seg_min<32>(v);
+            if (lane == 0) s_red[bb][wid] = v;
+            __syncthreads();
+            double r = s_red[bb][0];
+#pragma unroll
+            for (int i = 1; i < NW; i++) r = s_red[bb][i] < r ? s_red[bb][i] : r;
+            bb ^= 1;
+            return r;
+        }
+    };
+    auto smax = [&](double v) -> double {
+        if constexpr (NW == 1) {
+            return seg_max<W>(v);
+        } else {
+            v = seg_max<32>(v);
+            if (lane == 0) s_red[bb][wid] = v;
+            __syncthreads();
+            double r = s_red[bb][0];
+#pragma unroll
+            for (int i = 1; i < NW; i++) r = s_red[bb][i] > r ? s_red[bb][i] : r;
+            bb ^= 1;
+            return r;
+        }
+    };
+    auto ssum = [&](unsigned long long v) -> unsigned long long {
+        if constexpr (NW == 1) {
+            return seg_sum_u64<W>(v);
+        } else {
+            v = seg_sum_u64<32>(v);
+            if (lane == 0) s_red64[bb][wid] = v;
+            __syncthreads();
+            unsigned long long r = 0;
+#pragma unroll
+            for (int i = 0; i < NW; i++) r += s_red64[bb][i];
+            bb ^= 1;
+            return r;
+        }
+    };
+    auto xch = [&](int v, int src) -> int {    // value of segment lane src
+        if constexpr (NW == 1) {
+            return __shfl_sync(FULL, v, sbase + src);
+        } else {
+            s_xch[bb][threadIdx.x] = v;
+            __syncthreads();
+            const int r = s_xch[bb][src];
+            bb ^= 1;
+            return r;
+        }
+    };
+    ssync();
 
     // ---- segment-uniform ----
     bool have = false, exhausted = false;
@@ -155,7 +275,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
     HS.TF = HS.TB = HS.TO = HS.tcol_off = HS.ndp = HS.dcol_off = 0;
     HS.first_opt = 0xffffffffu;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
-    Group GT, GD;
+    Group<NW> GT, GD;
     GT.member = GD.member = false;
     Flow FT, FD, FP;
     FT.st = FD.st = FP.st = FS_NONE;
@@ -168,15 +288,16 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         nev = true;                                                           \
     } while (0)
 
-    auto grp_init = [&](Group &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll) {
+    auto grp_init = [&](Group<NW> &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll) {
         G.member = member;
         G.p = p;
         G.i = i;
         G.lane0 = lane0;
         G.stride = stride;
         G.pred = lane0 + ((i + p - 1) % p) * stride;
-        G.mask = 0;
-        for (int k = 0; k < p; k++) G.mask |= 1u << (lane0 + k * stride);
+#pragma unroll
+        for (int w = 0; w < NW; w++) G.mask.w[w] = 0;
+        for (int k = 0; k < p; k++) G.mask.w[(lane0 + k * stride) >> 5] |= 1u << ((lane0 + k * stride) & 31);
         G.gid = gid;
         G.ncoll = ncoll;
         G.trig = G.donec = G.cur = 0;
@@ -185,20 +306,22 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         G.cS = G.chunk = 0.0;
         G.flow_deliv = 0;
     };
-    auto gpu_of_member = [&](const Group &G, int k) -> uint32_t { return a.ro[TR.ro_off + (G.lane0 - sbase) + k * G.stride]; };
+    auto gpu_of_member = [&](const Group<NW> &G, int k) -> uint32_t { return a.ro[TR.ro_off + G.lane0 + k * G.stride]; };
     auto tp_seq = [&](uint32_t P, uint32_t j, uint32_t e) -> uint32_t {
         return P == 0 ? j * HS.TF + e : P == 1 ? m * HS.TF + (m - 1 - j) * HS.TB + e : m * (HS.TF + HS.TB) + e;
     };
 
     // R10 for one group: done on this member, finish, start, releases (all lanes call it)
-    auto grp_pass = [&](Group &G, Flow &F, bool is_tp, bool &more) {
-        const int Dp = __shfl_sync(FULL, G.D, G.pred);
-        unsigned upb = 0, dnb = 0;
-        if (__any_sync(FULL, G.tree_cur)) {
-            upb = __ballot_sync(FULL, G.upd);
-            dnb = __ballot_sync(FULL, G.dnd);
+    auto grp_pass = [&](Group<NW> &G, Flow &F, bool is_tp, bool &more) {
+        const int Dp = xch(G.D, G.pred);
+        Mask<NW> upb, dnb, zero;
+#pragma unroll
+        for (int w = 0; w < NW; w++) upb.w[w] = dnb.w[w] = zero.w[w] = 0;
+        if (vany(G.tree_cur)) {
+            upb = bal(G.upd);
+            dnb = bal(G.dnd);
         }
-        auto mb = [&](unsigned b, int k) -> bool { return (b >> (G.lane0 + k * G.stride)) & 1u; };
+        auto mb = [&](const Mask<NW> &b, int k) -> bool { return b.test(G.lane0 + k * G.stride); };
         const int c1 = 2 * G.i + 1, c2 = 2 * G.i + 2;
         if (G.member && G.running && !G.ldone) {
             bool dn;
@@ -214,12 +337,12 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                 G.donec = G.cur + 1;
             }
         }
-        const bool allfin = (__ballot_sync(FULL, !G.member || G.ldone) & G.mask) == G.mask;
+        const bool allfin = bal(!G.member || G.ldone).covers(G.mask);
         if (G.member && G.running && allfin) {
             G.running = false;
             G.cur++;
         }
-        const bool allrdy = (__ballot_sync(FULL, !G.member || G.trig > G.cur) & G.mask) == G.mask;
+        const bool allrdy = bal(!G.member || G.trig > G.cur).covers(G.mask);
         bool started = false;
         if (G.member && !G.running && G.cur < G.ncoll && allrdy) {
             CollEnt ce;
@@ -255,7 +378,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                     rel = true;
                 }
             } else if (G.i >= 1) {
-                const unsigned ub = started ? 0u : upb, db = started ? 0u : dnb;
+                const Mask<NW> ub = started ? zero : upb, db = started ? zero : dnb;
                 const bool ku = (c1 >= G.p || mb(ub, c1)) && (c2 >= G.p || mb(ub, c2));
                 const int par = (G.i - 1) / 2;
                 if (!G.uprel && ku) {
@@ -299,7 +422,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         }
         return false;
     };
-    auto grp_delivered = [&](Group &G) {
+    auto grp_delivered = [&](Group<NW> &G) {
         G.flow_deliv++;
         if (G.tree_cur) {
             if (G.fup) G.upd = true; else G.dnd = true;
@@ -327,10 +450,17 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         // ------------------------------ refill ------------------------------
         const bool need = !have && !exhausted;
         bool fresh = false, rbad = false, rlong = false;
-        if (__any_sync(FULL, need)) {
+        if (vany(need)) {
             uint32_t it = 0;
-            if (need && li == 0) it = atomicAdd(a.counter, 1u);
-            it = __shfl_sync(FULL, it, sbase);
+            if constexpr (NW == 1) {
+                if (need && li == 0) it = atomicAdd(a.counter, 1u);
+                it = __shfl_sync(FULL, it, sbase);
+            } else {
+                if (need && threadIdx.x == 0) s_item = atomicAdd(a.counter, 1u);
+                __syncthreads();
+                it = s_item;
+                __syncthreads();
+            }
             if (need) {
                 if (it >= a.n_work) {
                     exhausted = true;
@@ -376,8 +506,8 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                     gpu = a.ro[TR.ro_off + r];
                     const uint32_t ntp = tp > 1 ? m * (HS.TF + HS.TB) + HS.TO : 0;
                     const uint32_t ndp = dp > 1 ? HS.ndp : 0;
-                    grp_init(GT, used && tp > 1, tp, tt, sbase + (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp);
-                    grp_init(GD, used && dp > 1, dp, d, sbase + s * tp + tt, S * tp,
+                    grp_init(GT, used && tp > 1, tp, tt, (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp);
+                    grp_init(GD, used && dp > 1, dp, d, s * tp + tt, S * tp,
                              (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp);
                     if (used) {
                         // route checks of every pair this rank's flows will use (R3)
@@ -387,7 +517,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                             else if (l > MAX_HOPS) rlong = true;
                         };
                         for (int gk = 0; gk < 2; gk++) {
-                            const Group &G = gk == 0 ? GT : GD;
+                            const Group<NW> &G = gk == 0 ? GT : GD;
                             if (!G.member || G.ncoll == 0) continue;
                             if (C->need_ring) chk(gpu, gpu_of_member(G, (G.i + 1) % G.p));
                             if (C->need_tree && G.i >= 1) {
@@ -405,9 +535,9 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                     }
                 }
             }
-            if (__any_sync(FULL, fresh && (rbad || rlong))) {
-                const bool bad = (__ballot_sync(FULL, fresh && rbad) & smask) != 0;
-                const bool lng = (__ballot_sync(FULL, fresh && rlong) & smask) != 0;
+            if (vany(fresh && (rbad || rlong))) {
+                const bool bad = sany(fresh && rbad);
+                const bool lng = sany(fresh && rlong);
                 if (fresh && (bad || lng)) {
                     if (li == 0) {
                         triosim_result rr = {};
@@ -419,7 +549,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                 }
             }
         }
-        if (__all_sync(FULL, !have && exhausted)) break;
+        if (vall(!have && exhausted)) break;
 
         // ------------------------------ one instant ------------------------------
         bool dirty = false;
@@ -443,8 +573,8 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                     if (flow_step(FD, dirty)) { nflow++; grp_delivered(GD); }
                     if (flow_step(FP, dirty)) { nflow++; np2p++; dcnt++; }
                 }
-                cnt[lane] = dcnt;
-                __syncwarp();
+                cnt[li] = dcnt;
+                ssync();
                 // (d) both groups, then this rank's next P2P send
                 grp_pass(GT, FT, true, more);
                 grp_pass(GD, FD, false, more);
@@ -482,7 +612,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                         const uint32_t seqi = re.phase == 0 ? jp * ps.SF + re.e
                                             : re.phase == 1 ? m * ps.SF + (m - 1 - jp) * ps.SB + re.e
                                                             : m * (ps.SF + ps.SB) + re.e;
-                        if (!(cnt[sbase + (d * S + re.src) * tp + tt] > seqi)) ok = false;
+                        if (!(cnt[(d * S + re.src) * tp + tt] > seqi)) ok = false;
                     }
                     if (ok && en.tpw >= 0) {
                         const uint32_t pp_ = (uint32_t)en.tpw >> 24, ee = (uint32_t)en.tpw & 0xffffffu;
@@ -516,14 +646,13 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                         if (te == t) more = true;
                     }
                 }
-                __syncwarp();
-                if (!__any_sync(FULL, more)) break;
+                ssync();
+                if (!vany(more)) break;
             }
 
             // (f) R14 over every in-transit flow of the segment (up to three per lane)
-            const unsigned dball = __ballot_sync(FULL, dirty);
-            if (!dball) break;
-            const bool segdirty = (dball & smask) != 0;
+            if (!vany(dirty)) break;
+            const bool segdirty = sany(dirty);
             dirty = false;
             const bool aT = segdirty && used && FT.st == FS_ACT;
             const bool aD = segdirty && used && FD.st == FS_ACT;
@@ -555,7 +684,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
             count(FT, aT);
             count(FD, aD);
             count(FP, aP);
-            __syncwarp();
+            ssync();
             // if no link carries two active flows, R14 is exactly "rate = smallest residual on the
             // route" (n_e = 1: res_e / 1.0 == res_e) and the rounds are the distinct rates
             auto alone = [&](const Flow &F, bool on) -> bool {
@@ -567,7 +696,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                 }
                 return ok;
             };
-            const bool disj = (__ballot_sync(FULL, alone(FT, aT) && alone(FD, aD) && alone(FP, aP)) & smask) == smask;
+            const bool disj = !sany(!(alone(FT, aT) && alone(FD, aD) && alone(FP, aP)));
             auto fmin = [&](const Flow &F, bool on) -> double {
                 double my = dinf();
                 if (on) {
@@ -595,11 +724,11 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                 solo(FD, aD);
                 solo(FP, aP);
             }
-            __syncwarp();
+            ssync();
             bool uT = aT, uD = aD, uP = aP;
             uint32_t rounds = 0;
-            while (__any_sync(FULL, uT || uD || uP)) {
-                const bool segact = (__ballot_sync(FULL, uT || uD || uP) & smask) != 0;
+            while (vany(uT || uD || uP)) {
+                const bool segact = sany(uT || uD || uP);
                 double mT, mD, mP;
                 if (disj) {
                     mT = uT ? FT.rate : dinf();
@@ -612,7 +741,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                 }
                 double my = mT < mD ? mT : mD;
                 my = mP < my ? mP : my;
-                const double sm = seg_min<W>(my);
+                const double sm = smin(my);
                 const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
                 unsigned own = 0;
                 {
@@ -630,7 +759,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                         freeze(FD, iD, 1);
                         freeze(FP, iP, 2);
                     }
-                    __syncwarp();
+                    ssync();
                     auto update = [&](const Flow &F, int slot) {
 #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
@@ -650,14 +779,13 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
                         update(FP, 2);
                     }
                 }
-                __syncwarp();
+                ssync();
                 if (segact) rounds++;
                 uT = uT && !iT;
                 uD = uD && !iD;
                 uP = uP && !iP;
             }
-            const uint32_t nact = __popc(__ballot_sync(FULL, aT) & smask) + __popc(__ballot_sync(FULL, aD) & smask) +
-                                  __popc(__ballot_sync(FULL, aP) & smask);
+            const uint32_t nact = bal(aT).popc() + bal(aD).popc() + bal(aP).popc();
             if (segdirty) {
                 nwf++;
                 nrounds += rounds;
@@ -674,15 +802,14 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
             drain(FT, aT);
             drain(FD, aD);
             drain(FP, aP);
-            if (!__any_sync(FULL, again)) break;
+            if (!vany(again)) break;
         }
 
         // ------------------------------ end of instant ------------------------------
-        const bool any_ev = (__ballot_sync(FULL, nev) & smask) != 0;
+        const bool any_ev = sany(nev);
         if (have && any_ev) ninst++;
         nev = false;
-        const bool infl = (__ballot_sync(FULL, used && (FT.st != FS_NONE || FD.st != FS_NONE || FP.st != FS_NONE)) &
-                           smask) != 0;
+        const bool infl = sany(used && (FT.st != FS_NONE || FD.st != FS_NONE || FP.st != FS_NONE));
         if (have) {
             if (infl && !bon) { bon = true; bstart = t; }
             else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
@@ -690,7 +817,7 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
         const bool lane_done = !used || (cst == CS_IDLE && pos >= nprog && FT.st == FS_NONE && FD.st == FS_NONE &&
                                          FP.st == FS_NONE && sq >= nsend_tot && GT.cur >= GT.ncoll * (GT.member ? 1u : 0u) &&
                                          GD.cur >= GD.ncoll * (GD.member ? 1u : 0u) && !GT.running && !GD.running);
-        const bool alldone = (__ballot_sync(FULL, lane_done) & smask) == smask;
+        const bool alldone = !sany(!lane_done);
         const bool fin = have && alldone;
         double cand = dinf();
         if (used) {
@@ -703,15 +830,15 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
             cf(FD);
             cf(FP);
         }
-        const double tn = seg_min<W>(cand);
+        const double tn = smin(cand);
         const bool stuck = have && !fin && !(tn < dinf());
-        if (__any_sync(FULL, fin || stuck)) {
-            const double bmax = seg_max<W>(used ? busy : 0.0);
-            const unsigned long long ntk = seg_sum_u64<W>(ntask);
-            const unsigned long long nfl = seg_sum_u64<W>(nflow);
-            const unsigned long long npp = seg_sum_u64<W>(np2p);
-            const unsigned long long alg_s = seg_sum_u64<W>(alg);
-            const unsigned long long H = seg_sum_u64<W>(acc);
+        if (vany(fin || stuck)) {
+            const double bmax = smax(used ? busy : 0.0);
+            const unsigned long long ntk = ssum(ntask);
+            const unsigned long long nfl = ssum(nflow);
+            const unsigned long long npp = ssum(np2p);
+            const unsigned long long alg_s = ssum(alg);
+            const unsigned long long H = ssum(acc);
             if ((fin || stuck) && li == 0) {
                 triosim_result rr;
                 rr.iter_time_s = fin ? t : 0.0;
@@ -745,32 +872,37 @@ __global__ void __launch_bounds__(K3_THREADS, 1) k3_hybrid(const K3Args a) {
 #undef EV
 }
 
-template <int W>
+template <int W, int NW>
 static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
-    k3_hybrid<W><<<grid, K3_THREADS, 0, s>>>(a);
+    k3_hybrid<W, NW><<<grid, NW == 1 ? K3_THREADS : 32 * NW, 0, s>>>(a);
     return cudaGetLastError();
 }
 
+// W <= 32: W-lane segments in 256-thread CTAs; W = 64..256: one point per CTA of W threads
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
     switch (W) {
-    case 2: return launch_h<2>(a, grid, s);
-    case 4: return launch_h<4>(a, grid, s);
-    case 8: return launch_h<8>(a, grid, s);
-    case 16: return launch_h<16>(a, grid, s);
-    case 32: return launch_h<32>(a, grid, s);
+    case 2: return launch_h<2, 1>(a, grid, s);
+    case 4: return launch_h<4, 1>(a, grid, s);
+    case 8: return launch_h<8, 1>(a, grid, s);
+    case 16: return launch_h<16, 1>(a, grid, s);
+    case 32: return launch_h<32, 1>(a, grid, s);
+    case 64: return launch_h<32, 2>(a, grid, s);
+    case 128: return launch_h<32, 4>(a, grid, s);
+    case 256: return launch_h<32, 8>(a, grid, s);
     default: return cudaErrorInvalidValue;
     }
 }
 
-int k3h_max_blocks_per_sm(int W) {
+template <int W, int NW>
+static int occ_h() {
     int nb = 0;
-    switch (W) {
-    case 2: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<2>, K3_THREADS, 0); break;
-    case 4: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<4>, K3_THREADS, 0); break;
-    case 8: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<8>, K3_THREADS, 0); break;
-    case 16: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<16>, K3_THREADS, 0); break;
-    default: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<32>, K3_THREADS, 0); break;
-    }
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW>, NW == 1 ? K3_THREADS : 32 * NW, 0);
+    return nb;
+}
+
+int k3h_max_blocks_per_sm(int W) {
+    const int nb = W == 2 ? occ_h<2, 1>() : W == 4 ? occ_h<4, 1>() : W == 8 ? occ_h<8, 1>() : W == 16 ? occ_h<16, 1>()
+                 : W == 32 ? occ_h<32, 1>() : W == 64 ? occ_h<32, 2>() : W == 128 ? occ_h<32, 4>() : occ_h<32, 8>();
     return nb > 0 ? nb : 1;
 }
 

@@ -107,6 +107,30 @@ def test_random_hybrid(ctx, seed):
     assert (got["status"] == 0).sum() > 200
 
 
+@pytest.mark.parametrize("seed", range(2))
+def test_large_points_cta_kernel(ctx, seed):
+    """More than 32 simulated GPUs (configs[4] scale): DDP / TP / PP points map to their exactly
+    equivalent HYBRID form and run one point per CTA (64-256 ranks); compared with the oracle."""
+    rng = np.random.Generator(np.random.PCG64(1300 + seed))
+    tr = W.transformer_trace("tiny-gpt", 8, 64, 4, 256, 16, 100, 2, 11 + seed)
+    topos = [W.ring(64, 50e9, 1e-6), W.star(64, 80e9, 1e-6), W.hierarchical(8, 8, 1.0, 0.125, 2.0),
+             W.perturb_subset(W.hierarchical(32, 8, 1.0, 0.125, 4.0), 7 + seed)]
+    P = W.make_point
+    pts = [P(0, W.ST_DDP, dp=64, B=128, bucket=1 << 14, bw=2e9, lat=1e-6),
+           P(1, W.ST_DDP, dp=48, B=96, bucket=0, bw=5e9, lat=2e-6, algo=W.ALG_TREE),
+           P(1, W.ST_TP, tp=64, B=4, tp_mode=W.TPM_MEGATRON),
+           P(1, W.ST_TP, tp=48, B=4, tp_mode=W.TPM_PAPER, algo=W.ALG_TREE),
+           P(2, W.ST_HYBRID, dp=4, tp=8, pp=2, m=4, B=16, bucket=1 << 16, bw=100e9, lat=1e-6),
+           P(2, W.ST_HYBRID, dp=8, tp=4, pp=2, m=2, B=16, bucket=0, bw=100e9, lat=2e-6, tp_mode=W.TPM_PAPER),
+           P(3, W.ST_HYBRID, dp=8, tp=8, pp=4, m=4, B=32, bucket=1 << 18, bw=300e9, lat=1e-6),
+           P(3, W.ST_HYBRID, dp=16, tp=4, pp=4, m=2, B=32, bucket=1 << 18, bw=300e9, lat=1e-6, algo=W.ALG_TREE),
+           P(3, W.ST_PP, pp=8, m=4, B=8, bw=300e9, lat=1e-6)]
+    sw = W.Sweep("large", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all(), got["status"]
+    check(got, sw, list(range(len(pts))))
+
+
 def test_statuses_and_edge_cases(ctx):
     tr = W.mlp_trace()
     topos = [W.ring(4, 10e9, 1e-6), W.ring(32, 10e9, 1e-6), W.ring(40, 10e9, 1e-6), W.star(32, 10e9, 1e-6)]
@@ -136,9 +160,9 @@ def test_statuses_and_edge_cases(ctx):
     got = ctx.run_sweep(sw)
     check(got, sw, list(range(len(pts))))
     assert list(got["status"][:11]) == [1, 2, 1, 0, 6, 6, 7, 7, 0, 7, 3]
-    # beyond the warp kernel's limits -- more than 32 lanes, a route longer than 8 hops (tree
-    # edges across a 32-GPU ring) -- is reported, never silently wrong
-    big = W.Sweep("big", tr, topos, W.points_array([P(2, W.ST_DDP, dp=40, B=40 * 64),
+    # beyond the kernels' limits -- DataParallel (after-backward) with more than 32 GPUs, a route longer
+    # than 8 hops (tree edges across a 32-GPU ring) -- is reported, never silently wrong
+    big = W.Sweep("big", tr, topos, W.points_array([P(2, W.ST_DP, dp=40, B=40 * 64),
                                                     P(1, W.ST_DDP, dp=32, B=32 * 64, algo=W.ALG_TREE)]))
     assert list(ctx.run_sweep(big)["status"]) == [W.PT_TOO_LARGE, W.PT_TOO_LARGE]
     # empty sweep
