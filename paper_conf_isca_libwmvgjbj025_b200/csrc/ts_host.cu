@@ -98,13 +98,15 @@ struct Sweep {
     DevBuf<uint32_t> d_work[N_GROUPS];
     DevBuf<uint32_t> d_work_tmp[N_GROUPS];
     std::vector<int> mode;                   // per point
+    uint32_t lmax[N_GROUPS] = {};            // hybrid CTA groups: largest topology (links) among their points
+    int occ[N_GROUPS] = {};                  // hybrid CTA groups: resident CTAs per SM at that smem
     DevBuf<unsigned int> d_counter;
     DevBuf<unsigned long long> d_alg;
     cudaStream_t last_stream = nullptr;
 };
 
 int w_index(int W) { int i = 0; while ((2 << i) < W) i++; return i; }
-const int W_OF[N_WIDTHS] = {2, 4, 8, 16, 32, 64, 128, 256};
+const int W_OF[N_WIDTHS] = {2, 4, 8, 16, 32, 64, 128, 256, 512, 1024};
 
 }  // namespace
 
@@ -165,7 +167,8 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
             return TRIOSIM_ECUDA;
         }
         const int Wi = W_OF[i / N_MODES], md = i % N_MODES;
-        ctx->occ[i] = md == MODE_HYBRID ? k3h_max_blocks_per_sm(Wi) : Wi <= 32 ? k3_max_blocks_per_sm(Wi, md) : 1;
+        ctx->occ[i] = md == MODE_HYBRID ? (Wi <= 32 ? k3h_max_blocks_per_sm(Wi, 0) : 1)
+                                        : Wi <= 32 ? k3_max_blocks_per_sm(Wi, md) : 1;
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
         triosim_destroy(ctx);
@@ -473,7 +476,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             plan_key = pt.stage_plan;
         }
         // GPU kernel limits: warp segments (<= 32 lanes, lmax_warp links) for DP / DDP / TP / PP; the
-        // HYBRID kernel (warp segments up to 32 ranks, one point per CTA up to 256 ranks, LMAX_CTA links)
+        // HYBRID kernel (warp segments up to 32 ranks, one point per CTA up to 1024 ranks, LMAX_CTA links)
         // for HYBRID and for DDP / TP / PP points beyond the warp kernels -- DDP = (dp,1,1,1),
         // TP = (1,tp,1,1), PP = (1,1,pp,m) reproduce those strategies bit for bit (R9, pinned)
         const uint32_t lanes = pt.strategy == TRIOSIM_TP ? tpd : pt.strategy == TRIOSIM_PP ? pp
@@ -491,7 +494,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
                 if (pt.strategy != TRIOSIM_PP) pt.microbatches = 1;
                 pt.strategy = TRIOSIM_HYBRID;
             }
-            for (int w = W0; w <= 256; w <<= 1)
+            for (int w = W0; w <= 1024; w <<= 1)
                 if ((int)tp.n_links <= lm(true, w)) { W = w; break; }
         }
         if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
@@ -678,7 +681,17 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         if (S->cost[a] != S->cost[b]) return S->cost[a] > S->cost[b];
         return pdesc[a].cls < pdesc[b].cls;
     });
-    for (uint64_t i : order) S->work[N_MODES * w_index(S->width[i]) + S->mode[i]].push_back((uint32_t)i);
+    for (uint64_t i : order) {
+        const int g = N_MODES * w_index(S->width[i]) + S->mode[i];
+        S->work[g].push_back((uint32_t)i);
+        if (S->width[i] > 32) {
+            const uint32_t nl = HT[pts[i].topo].n_links;
+            const uint32_t r = (nl + 63) / 64 * 64;
+            if (r > S->lmax[g]) S->lmax[g] = r;
+        }
+    }
+    for (int g = 0; g < N_GROUPS; g++)
+        if (S->lmax[g]) S->occ[g] = k3h_max_blocks_per_sm(W_OF[g / N_MODES], S->lmax[g]);
     for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
         CK(S->d_work_tmp[w].alloc(S->work[w].size()));
@@ -757,6 +770,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         a.hst = S.d_hst.p; a.hents = S.d_hents.p; a.hsends = S.d_hsends.p;
         a.out = S.d_res.p;
         a.alg_ops = S.d_alg.p;
+        a.lmax = S.lmax[w];
         uint64_t blocks;
         if (W <= 32) {
             const int nseg = 32 / W;
@@ -765,7 +779,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         } else {
             blocks = n;   // one point per CTA
         }
-        const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)ctx->occ[w];
+        const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)(S.lmax[w] ? S.occ[w] : ctx->occ[w]);
         if (blocks > cap) blocks = cap;
         CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
         if (mode == MODE_HYBRID) CK(launch_k3_hybrid(W, a, (int)blocks, ctx->side[w]));

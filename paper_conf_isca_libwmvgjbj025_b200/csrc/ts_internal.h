@@ -133,7 +133,7 @@ struct PointDesc {
 struct K3Args {
     const PointDesc *pts;
     const uint32_t *work;
-    uint32_t n_work, pad;
+    uint32_t n_work, lmax;         // lmax: links per segment in dynamic smem (one-point-per-CTA hybrid)
     unsigned int *counter;
     const ClassDesc *cls;
     const TopoDev *topo;
@@ -169,13 +169,14 @@ cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, c
                              RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s);      // ts_k3h.cu
-int k3h_max_blocks_per_sm(int W);
+int k3h_max_blocks_per_sm(int W, uint32_t lmax);   // lmax: dynamic-smem links (W > 32)
+size_t k3h_dyn_smem(int W, uint32_t lmax);
 int k3_max_blocks_per_sm(int W, int mode);
 // links per segment the K3 kernels keep in shared memory
 __host__ __device__ constexpr int lmax_warp(int W) { return 4 * W < 8 ? 8 : 4 * W; }
 __host__ __device__ constexpr int lmax_hybrid(int W) { return 8 * W < 16 ? 16 : 8 * W; }
-constexpr int LMAX_CTA = 2048;          // links of a one-point-per-CTA hybrid segment
-constexpr int N_WIDTHS = 8;             // W = 2, 4, 8, 16, 32 (warp segments), 64, 128, 256 (hybrid CTAs)
+constexpr int LMAX_CTA = 12288;         // links of a one-point-per-CTA hybrid segment (dynamic smem, 16 B/link)
+constexpr int N_WIDTHS = 10;            // W = 2, 4, 8, 16, 32 (warp segments), 64 ... 1024 (hybrid CTAs)
 constexpr int N_MODES = 4;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 

@@ -1,7 +1,7 @@
 // ts_k3h.cu -- K3 for HYBRID DP x TP x PP points (R9; Table 1).
 //
 // One point per segment: W lanes of a warp (NW = 1), or NW whole warps = one CTA (NW = 2..8, up to
-// 256 ranks).  Lane r = rank (d, s, t) with r = (d*pp + s)*tp + t.  Each lane
+// 1024 ranks).  Lane r = rank (d, s, t) with r = (d*pp + s)*tp + t.  Each lane
 // runs its stage's GPipe program (R8) and owns THREE flow slots: its TP-group collective step,
 // its DP-group collective step and its FIFO P2P send.  The TP group {(d,s,.)} is a contiguous lane
 // range, the DP group {(.,s,t)} a strided one; both run R10's ring / tree collectives through one
@@ -65,38 +65,26 @@ struct Flow {
     uint64_t code;
 };
 
-// bits over the lanes of one segment
-template <int NW>
-struct Mask {
-    uint32_t w[NW];
-    __device__ __forceinline__ bool test(int k) const { return (w[k >> 5] >> (k & 31)) & 1u; }
-    __device__ __forceinline__ bool covers(const Mask &m) const {
-        bool ok = true;
-#pragma unroll
-        for (int i = 0; i < NW; i++) ok = ok && ((w[i] & m.w[i]) == m.w[i]);
-        return ok;
-    }
-    __device__ __forceinline__ bool any() const {
-        uint32_t x = 0;
-#pragma unroll
-        for (int i = 0; i < NW; i++) x |= w[i];
-        return x != 0;
-    }
-    __device__ __forceinline__ uint32_t popc() const {
-        uint32_t x = 0;
-#pragma unroll
-        for (int i = 0; i < NW; i++) x += __popc(w[i]);
-        return x;
+// one boolean per segment lane: ballot bits (warp segments) or a shared-memory byte array (CTA)
+template <bool CTA>
+struct LaneFlags {
+    uint32_t bits;      // warp segment: ballot bits (0 = all false)
+    const uint8_t *p;   // CTA: flag bytes (nullptr = all false)
+    uint8_t sel;
+    __device__ __forceinline__ bool test(int k) const {
+        if constexpr (CTA) return p != nullptr && (p[k] & sel) != 0;
+        else return (bits >> k) & 1u;
     }
 };
 // one collective group (TP or DP) as seen by one member lane
-template <int NW>
 struct Group {
     bool member;
     int p, i;                 // group size, my member index
     int lane0, stride;        // segment lane of member k = lane0 + k * stride
     int pred;                 // segment lane of member (i - 1) mod p
-    Mask<NW> mask;            // lanes of the group
+    bool cross;               // segment-uniform: some group of this kind spans several warps (CTA only)
+    uint32_t wmask;           // warp-lane bits of the members when the group lies inside this lane's warp
+    int slot;                 // counter slot of a cross-warp group (CTA only)
     uint64_t gid;
     uint32_t ncoll, trig, donec, cur;
     bool running, tree_cur, ldone, uprel, upd, dnrel, dnd, fup;
@@ -141,16 +129,21 @@ template <int W, int NW>
 __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(const K3Args a) {
     constexpr int SL = NW == 1 ? W : 32 * NW;           // lanes per segment
     constexpr int NSEG = NW == 1 ? 32 / W : 1;          // segments per warp (NW = 1)
-    constexpr int LMAX = NW == 1 ? lmax_hybrid(W) : LMAX_CTA;
+    constexpr int LMAXW = lmax_hybrid(W);               // warp segments: static link arrays
     constexpr int NSLOT = NW == 1 ? K3_WARPS : 1;       // segment-array slots of the block
-    __shared__ double s_res[NSLOT][NSEG * LMAX];
-    __shared__ int s_n[NSLOT][NSEG * LMAX];
-    __shared__ int s_k[NSLOT][NSEG * LMAX];
+    // warp segments keep their link arrays in static smem; a one-point CTA sizes them to the sweep's
+    // largest topology (a.lmax links, dynamic smem: residual f64, unfrozen and frozen counts)
+    __shared__ double s_res[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
+    __shared__ int s_n[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
+    __shared__ int s_k[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
+    extern __shared__ double s_dyn[];
+    const int LMAX = NW == 1 ? LMAXW : (int)a.lmax;
     __shared__ uint32_t s_cnt[NSLOT][NW == 1 ? 32 : SL];
-    __shared__ uint32_t s_bal[2][NW];
     __shared__ double s_red[2][NW];
     __shared__ unsigned long long s_red64[2][NW];
     __shared__ int s_xch[2][NW == 1 ? 1 : SL];
+    __shared__ int s_gc[3][NW == 1 ? 1 : SL];          // cross-warp group counters (rotating triple buffer)
+    __shared__ uint8_t s_fl[2][NW == 1 ? 1 : SL];      // tree flags exchange (CTA)
     __shared__ uint32_t s_item;
 
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -159,15 +152,20 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     const int sbase = NW == 1 ? seg * W : 0;                 // segment's first warp lane (NW = 1)
     const unsigned smask = NW == 1 ? ((W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase) : FULL;
     const int slot = NW == 1 ? wid : 0;
-    double *lres = &s_res[slot][seg * LMAX];
-    int *ln = &s_n[slot][seg * LMAX];
-    int *lk = &s_k[slot][seg * LMAX];
+    double *lres = NW == 1 ? &s_res[slot][seg * LMAX] : s_dyn;
+    int *ln = NW == 1 ? &s_n[slot][seg * LMAX] : (int *)(s_dyn + LMAX);
+    int *lk = NW == 1 ? &s_k[slot][seg * LMAX] : (int *)(s_dyn + LMAX) + LMAX;
     uint32_t *cnt = &s_cnt[slot][sbase];                     // indexed by segment lane
     for (int q = (NW == 1 ? lane : (int)threadIdx.x); q < NSEG * LMAX; q += (NW == 1 ? 32 : 32 * NW)) {
-        s_n[slot][q] = 0;
-        s_k[slot][q] = 0;
+        ln[q - seg * LMAX] = 0;   // (NW == 1: each lane clears its warp's slot through segment 0's base)
+        lk[q - seg * LMAX] = 0;
+    }
+    if constexpr (NW > 1) {
+        s_gc[0][threadIdx.x] = s_gc[1][threadIdx.x] = s_gc[2][threadIdx.x] = 0;
     }
     int bb = 0;   // double-buffer toggle of the block-level exchanges (NW > 1)
+    int fb = 0;   // double-buffer toggle of the tree-flag exchange (NW > 1)
+    int gcb = 0;  // rotating buffer of the cross-warp group counters (NW > 1)
 
     // ---- segment primitives: a segment is W lanes of a warp, or the whole CTA ----
     auto ssync = [&]() {
@@ -179,21 +177,43 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     auto vall = [&](bool p) -> bool {
         if constexpr (NW == 1) return __all_sync(FULL, p); else return __syncthreads_and(p) != 0;
     };
-    auto bal = [&](bool p) -> Mask<NW> {       // segment ballot, bit k = segment lane k
-        Mask<NW> m;
-        if constexpr (NW == 1) {
-            m.w[0] = (__ballot_sync(FULL, p) & smask) >> sbase;
-        } else {
-            const unsigned b = __ballot_sync(FULL, p);
-            if (lane == 0) s_bal[bb][wid] = b;
-            __syncthreads();
-#pragma unroll
-            for (int i = 0; i < NW; i++) m.w[i] = s_bal[bb][i];
-            bb ^= 1;
-        }
-        return m;
+    auto sany = [&](bool p) -> bool {          // any lane of the segment
+        if constexpr (NW == 1) return (__ballot_sync(FULL, p) & smask) != 0; else return __syncthreads_or(p) != 0;
     };
-    auto sany = [&](bool p) -> bool { return bal(p).any(); };
+    auto scount = [&](bool p) -> uint32_t {    // lanes of the segment with p
+        if constexpr (NW == 1) return __popc(__ballot_sync(FULL, p) & smask); else return __syncthreads_count(p);
+    };
+    // upd / dnd flags of every segment lane (tree collectives)
+    using LF = LaneFlags<(NW > 1)>;
+    auto flags2 = [&](bool u, bool dn, LF &fu, LF &fd) {
+        if constexpr (NW == 1) {
+            fu.bits = (__ballot_sync(FULL, u) & smask) >> sbase;
+            fd.bits = (__ballot_sync(FULL, dn) & smask) >> sbase;
+            fu.p = fd.p = nullptr;
+        } else {
+            s_fl[fb][threadIdx.x] = (uint8_t)((u ? 1 : 0) | (dn ? 2 : 0));
+            __syncthreads();
+            fu.p = fd.p = s_fl[fb];
+            fu.bits = fd.bits = 0;
+            fb ^= 1;
+        }
+        fu.sel = 1;
+        fd.sel = 2;
+    };
+    // every member of G satisfies pred (called by all lanes; non-members pass anything)
+    auto gall = [&](const Group &G, bool pred) -> bool {
+        if (NW == 1 || !G.cross) {
+            const unsigned b = __ballot_sync(FULL, !G.member || pred);
+            return (b & G.wmask) == G.wmask;
+        } else {
+            const int cb = gcb;
+            gcb = gcb == 2 ? 0 : gcb + 1;
+            s_gc[gcb][threadIdx.x] = 0;    // next call's buffer: its last readers passed a barrier since
+            if (G.member && pred) atomicAdd(&s_gc[cb][G.slot], 1);
+            __syncthreads();
+            return !G.member || s_gc[cb][G.slot] == G.p;
+        }
+    };
     auto smin = [&](double v) -> double {
         if constexpr (NW == 1) {
             return seg_min<W>(v);
@@ -275,7 +295,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     HS.TF = HS.TB = HS.TO = HS.tcol_off = HS.ndp = HS.dcol_off = 0;
     HS.first_opt = 0xffffffffu;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
-    Group<NW> GT, GD;
+    Group GT, GD;
     GT.member = GD.member = false;
     Flow FT, FD, FP;
     FT.st = FD.st = FP.st = FS_NONE;
@@ -288,16 +308,22 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         nev = true;                                                           \
     } while (0)
 
-    auto grp_init = [&](Group<NW> &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll) {
+    auto grp_init = [&](Group &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll,
+                        int slot) {
         G.member = member;
         G.p = p;
         G.i = i;
         G.lane0 = lane0;
         G.stride = stride;
         G.pred = lane0 + ((i + p - 1) % p) * stride;
-#pragma unroll
-        for (int w = 0; w < NW; w++) G.mask.w[w] = 0;
-        for (int k = 0; k < p; k++) G.mask.w[(lane0 + k * stride) >> 5] |= 1u << ((lane0 + k * stride) & 31);
+        G.slot = slot;
+        G.wmask = 0;
+        const int last = lane0 + (p - 1) * stride;
+        const bool inwarp = NW == 1 || (lane0 >> 5) == (last >> 5);
+        if (member && inwarp)
+            for (int k = 0; k < p; k++) G.wmask |= 1u << ((sbase + lane0 + k * stride) & 31);
+        if constexpr (NW == 1) G.cross = false;               // (segments of a warp refill independently)
+        else G.cross = sany(member && !inwarp);               // (a CTA segment refills as a whole)
         G.gid = gid;
         G.ncoll = ncoll;
         G.trig = G.donec = G.cur = 0;
@@ -306,22 +332,20 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         G.cS = G.chunk = 0.0;
         G.flow_deliv = 0;
     };
-    auto gpu_of_member = [&](const Group<NW> &G, int k) -> uint32_t { return a.ro[TR.ro_off + G.lane0 + k * G.stride]; };
+    auto gpu_of_member = [&](const Group &G, int k) -> uint32_t { return a.ro[TR.ro_off + G.lane0 + k * G.stride]; };
     auto tp_seq = [&](uint32_t P, uint32_t j, uint32_t e) -> uint32_t {
         return P == 0 ? j * HS.TF + e : P == 1 ? m * HS.TF + (m - 1 - j) * HS.TB + e : m * (HS.TF + HS.TB) + e;
     };
 
     // R10 for one group: done on this member, finish, start, releases (all lanes call it)
-    auto grp_pass = [&](Group<NW> &G, Flow &F, bool is_tp, bool &more) {
+    auto grp_pass = [&](Group &G, Flow &F, bool is_tp, bool &more) {
         const int Dp = xch(G.D, G.pred);
-        Mask<NW> upb, dnb, zero;
-#pragma unroll
-        for (int w = 0; w < NW; w++) upb.w[w] = dnb.w[w] = zero.w[w] = 0;
-        if (vany(G.tree_cur)) {
-            upb = bal(G.upd);
-            dnb = bal(G.dnd);
-        }
-        auto mb = [&](const Mask<NW> &b, int k) -> bool { return b.test(G.lane0 + k * G.stride); };
+        LF upb, dnb, zero;
+        upb.bits = dnb.bits = zero.bits = 0;
+        upb.p = dnb.p = zero.p = nullptr;
+        upb.sel = dnb.sel = zero.sel = 1;
+        if (vany(G.tree_cur)) flags2(G.upd, G.dnd, upb, dnb);
+        auto mb = [&](const LF &b, int k) -> bool { return b.test(G.lane0 + k * G.stride); };
         const int c1 = 2 * G.i + 1, c2 = 2 * G.i + 2;
         if (G.member && G.running && !G.ldone) {
             bool dn;
@@ -337,12 +361,12 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 G.donec = G.cur + 1;
             }
         }
-        const bool allfin = bal(!G.member || G.ldone).covers(G.mask);
+        const bool allfin = gall(G, G.ldone);
         if (G.member && G.running && allfin) {
             G.running = false;
             G.cur++;
         }
-        const bool allrdy = bal(!G.member || G.trig > G.cur).covers(G.mask);
+        const bool allrdy = gall(G, G.trig > G.cur);
         bool started = false;
         if (G.member && !G.running && G.cur < G.ncoll && allrdy) {
             CollEnt ce;
@@ -378,7 +402,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     rel = true;
                 }
             } else if (G.i >= 1) {
-                const Mask<NW> ub = started ? zero : upb, db = started ? zero : dnb;
+                const LF ub = started ? zero : upb, db = started ? zero : dnb;
                 const bool ku = (c1 >= G.p || mb(ub, c1)) && (c2 >= G.p || mb(ub, c2));
                 const int par = (G.i - 1) / 2;
                 if (!G.uprel && ku) {
@@ -422,7 +446,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         }
         return false;
     };
-    auto grp_delivered = [&](Group<NW> &G) {
+    auto grp_delivered = [&](Group &G) {
         G.flow_deliv++;
         if (G.tree_cur) {
             if (G.fup) G.upd = true; else G.dnd = true;
@@ -506,9 +530,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     gpu = a.ro[TR.ro_off + r];
                     const uint32_t ntp = tp > 1 ? m * (HS.TF + HS.TB) + HS.TO : 0;
                     const uint32_t ndp = dp > 1 ? HS.ndp : 0;
-                    grp_init(GT, used && tp > 1, tp, tt, (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp);
+                    grp_init(GT, used && tp > 1, tp, tt, (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp, d * S + s);
                     grp_init(GD, used && dp > 1, dp, d, s * tp + tt, S * tp,
-                             (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp);
+                             (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp, s * tp + tt);
                     if (used) {
                         // route checks of every pair this rank's flows will use (R3)
                         auto chk = [&](uint32_t x, uint32_t y) {
@@ -517,7 +541,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             else if (l > MAX_HOPS) rlong = true;
                         };
                         for (int gk = 0; gk < 2; gk++) {
-                            const Group<NW> &G = gk == 0 ? GT : GD;
+                            const Group &G = gk == 0 ? GT : GD;
                             if (!G.member || G.ncoll == 0) continue;
                             if (C->need_ring) chk(gpu, gpu_of_member(G, (G.i + 1) % G.p));
                             if (C->need_tree && G.i >= 1) {
@@ -785,7 +809,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 uD = uD && !iD;
                 uP = uP && !iP;
             }
-            const uint32_t nact = bal(aT).popc() + bal(aD).popc() + bal(aP).popc();
+            const uint32_t nact = scount(aT) + scount(aD) + scount(aP);
             if (segdirty) {
                 nwf++;
                 nrounds += rounds;
@@ -872,13 +896,20 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
 #undef EV
 }
 
+size_t k3h_dyn_smem(int W, uint32_t lmax) { return W <= 32 ? 0 : (size_t)lmax * 16; }
+
 template <int W, int NW>
 static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
-    k3_hybrid<W, NW><<<grid, NW == 1 ? K3_THREADS : 32 * NW, 0, s>>>(a);
+    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, a.lmax);
+    if (NW > 1) {
+        const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+        if (e != cudaSuccess) return e;
+    }
+    k3_hybrid<W, NW><<<grid, NW == 1 ? K3_THREADS : 32 * NW, dyn, s>>>(a);
     return cudaGetLastError();
 }
 
-// W <= 32: W-lane segments in 256-thread CTAs; W = 64..256: one point per CTA of W threads
+// W <= 32: W-lane segments in 256-thread CTAs; W = 64..1024: one point per CTA of W threads
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
     switch (W) {
     case 2: return launch_h<2, 1>(a, grid, s);
@@ -889,20 +920,36 @@ cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
     case 64: return launch_h<32, 2>(a, grid, s);
     case 128: return launch_h<32, 4>(a, grid, s);
     case 256: return launch_h<32, 8>(a, grid, s);
+    case 512: return launch_h<32, 16>(a, grid, s);
+    case 1024: return launch_h<32, 32>(a, grid, s);
     default: return cudaErrorInvalidValue;
     }
 }
 
 template <int W, int NW>
-static int occ_h() {
+static int occ_h(uint32_t lmax) {
+    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, lmax);
+    if (NW > 1 && cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
+        return 0;
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW>, NW == 1 ? K3_THREADS : 32 * NW, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
     return nb;
 }
 
-int k3h_max_blocks_per_sm(int W) {
-    const int nb = W == 2 ? occ_h<2, 1>() : W == 4 ? occ_h<4, 1>() : W == 8 ? occ_h<8, 1>() : W == 16 ? occ_h<16, 1>()
-                 : W == 32 ? occ_h<32, 1>() : W == 64 ? occ_h<32, 2>() : W == 128 ? occ_h<32, 4>() : occ_h<32, 8>();
+int k3h_max_blocks_per_sm(int W, uint32_t lmax) {
+    int nb;
+    switch (W) {
+    case 2: nb = occ_h<2, 1>(lmax); break;
+    case 4: nb = occ_h<4, 1>(lmax); break;
+    case 8: nb = occ_h<8, 1>(lmax); break;
+    case 16: nb = occ_h<16, 1>(lmax); break;
+    case 32: nb = occ_h<32, 1>(lmax); break;
+    case 64: nb = occ_h<32, 2>(lmax); break;
+    case 128: nb = occ_h<32, 4>(lmax); break;
+    case 256: nb = occ_h<32, 8>(lmax); break;
+    case 512: nb = occ_h<32, 16>(lmax); break;
+    default: nb = occ_h<32, 32>(lmax); break;
+    }
     return nb > 0 ? nb : 1;
 }
 

@@ -736,34 +736,51 @@ def sweep_c4(trace=None, seed=4, n_bw=25, n_lat=8) -> Sweep:
     return Sweep("c4_gpt2xl_pp", tr, topos, arr[perm])
 
 
-def sweep_c5(trace=None, seed=5, max_gpus=32, n_bw=4, n_lat=2) -> Sweep:
-    """configs[4] within the warp kernel's 32-GPU limit: GPT-3-class HYBRID DP x TP x PP on 8-32
-    simulated GPUs of a hierarchical topology (2:1 / 4:1 oversubscribed, also with a seeded slow
-    link subset), every (TP, PP, DP) split with TP <= 8 inside a node and TP*PP >= 4, micro-batches
-    8-32, 2 GiB gradient buckets."""
+def sweep_c5(trace=None, seed=5, Ns=(64, 128, 256, 512, 1024), n_bw=25, n_lat=14, oversubs=(1.0, 2.0, 4.0),
+             ms=(8, 16, 32, 64)) -> Sweep:
+    """configs[4]: GPT-3-class HYBRID DP x TP x PP on N in {64..1024} simulated GPUs of a hierarchical
+    topology (8-GPU nodes on a node switch, per-GPU NIC to leaf switches, spine at 1:1 / 2:1 / 4:1
+    oversubscription; each also with a seeded slow link subset).  Every (TP, PP, DP) split with
+    TP <= 8 inside a node, PP | N a power of two <= 64, TP*PP >= 4 (a 175B model needs >= 4-way model
+    parallelism to fit), micro-batches 8..64 (one sample each), 2 GiB gradient buckets, n_bw bandwidth x
+    n_lat latency scales.  Defaults give 2,760 structural combinations x 350 = 966,000 points (the
+    configs[4] ~1M-point sweep); seeded order.  Built with numpy (no per-point Python objects)."""
     tr = trace if trace is not None else gpt3_trace()
-    topos, pts = [], []
-    for N in (8, 16, 32):
-        if N > max_gpus:
-            continue
-        for ov in (2.0, 4.0):
+    topos, rows = [], []
+    for N in Ns:
+        for ov in oversubs:
             base = hierarchical(max(N // 8, 1), 8, intra=1.0, nic=0.125, oversub=ov)
             for asym in (0, 1):
                 ti = len(topos)
                 topos.append(base if asym == 0 else perturb_subset(base, 500 + 10 * N + int(ov)))
-                for tp in (1, 2, 4, 8):
-                    for pp in (1, 2, 4, 8, 16):
-                        if N % (tp * pp) or pp > tr.n_layers or tp * pp < 4:
-                            continue   # a 175B model needs >= 4-way model parallelism to fit
-                        dp = N // (tp * pp)
-                        for m in (8, 16, 32):
-                            if pp == 1 and m > 8:
-                                continue
-                            for bw in np.logspace(np.log10(100e9), np.log10(900e9), n_bw):
-                                for lat in np.logspace(np.log10(1e-6), np.log10(5e-6), n_lat):
-                                    pts.append(make_point(ti, ST_HYBRID, dp=dp, tp=tp, pp=pp, m=m, B=dp * m,
-                                                          bucket=2048 * MiB, bw=float(bw), lat=float(lat)))
-    arr = points_array(pts)
+                for tpd in (1, 2, 4, 8):
+                    for pp in (1, 2, 4, 8, 16, 32, 64):
+                        if N % (tpd * pp) or pp > tr.n_layers or tpd * pp < 4:
+                            continue
+                        for m in ms:
+                            rows.append((ti, N // (tpd * pp), tpd, pp, m))
+    bws = np.logspace(np.log10(100e9), np.log10(900e9), n_bw)
+    lats = np.logspace(np.log10(1e-6), np.log10(5e-6), n_lat)
+    R = np.array(rows, dtype=np.int64).reshape(-1, 5)
+    nbl = n_bw * n_lat
+    arr = np.zeros(len(R) * nbl, POINT_DTYPE)
+    rep = np.repeat(R, nbl, axis=0)
+    arr["topo"] = rep[:, 0]
+    arr["strategy"] = ST_HYBRID
+    arr["tp_mode"] = TPM_MEGATRON
+    arr["coll_algo"] = ALG_RING
+    arr["dp"], arr["tp"], arr["pp"], arr["microbatches"] = rep[:, 1], rep[:, 2], rep[:, 3], rep[:, 4]
+    arr["global_batch"] = rep[:, 1] * rep[:, 4]
+    arr["stage_plan"] = -1
+    arr["bucket_bytes"] = 2048 * MiB
+    arr["bw_scale"] = np.tile(np.repeat(bws, n_lat), len(R))
+    arr["lat_scale"] = np.tile(np.tile(lats, n_bw), len(R))
     perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
     return Sweep("c5_gpt3_hybrid", tr, topos, arr[perm])
+
+
+def sweep_c5_small(trace=None, seed=5) -> Sweep:
+    """configs[4]'s structure on 8-32 simulated GPUs (warp-segment hybrid kernel; m in {8,16,32},
+    4 bandwidths x 2 latencies): the small end used by the sampled parity tests."""
+    return sweep_c5(trace, seed, Ns=(8, 16, 32), n_bw=4, n_lat=2, oversubs=(2.0, 4.0), ms=(8, 16, 32))
 

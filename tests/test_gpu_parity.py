@@ -244,13 +244,34 @@ def test_c4_gpt2xl_pp_sampled(ctx):
 
 
 def test_c5_gpt3_hybrid_sampled(ctx):
-    """configs[4] (GPT-3-class DP x TP x PP on a hierarchical asymmetric topology, 8-32 GPUs): a seeded
-    subset of the lighter points (m = 8; the heaviest points have ~2M instants each) on the GPU, every
-    point must simulate, 16 of them against the oracle."""
-    full = W.sweep_c5()
+    """configs[4]'s structure at 8-32 GPUs (warp-segment hybrid kernel): a seeded subset of the lighter
+    points (m = 8; the heaviest points have ~2M instants each) on the GPU, every point must simulate,
+    16 of them against the oracle."""
+    full = W.sweep_c5_small()
     light = [i for i, p in enumerate(full.points) if p["microbatches"] == 8 and p["tp"] <= 4]
     sub = [light[i] for i in sample(len(light), 120, 55)]
     sw = W.Sweep(full.name, full.trace, full.topos, full.points[sub])
     got = ctx.run_sweep(sw)
     assert (got["status"] == 0).all(), np.unique(got["status"], return_counts=True)
     check(got, sw, sample(len(sw.points), 16, 5))
+
+
+def test_c5_full_scale_sampled(ctx):
+    """configs[4] at full scale: the ~1M-point sweep over 64-1024 simulated GPUs (one point per CTA of up
+    to 1024 threads).  A seeded sample of its lighter points at every N -- m = 8, dp <= 4, the symmetric
+    hierarchical topologies above 64 GPUs (<= ~1.2e5 instants; the oracle finishes each in seconds.  The
+    heaviest points, e.g. dp = 16 x tp = 8 at 128 GPUs or the perturbed topologies at 1024 GPUs, take
+    1e6-1e7 instants and minutes of oracle time) -- in the sweep's launch configuration, all against the
+    oracle."""
+    full = W.sweep_c5()
+    P = full.points
+    N = P["dp"].astype(np.int64) * P["tp"] * P["pp"]
+    sym = (P["topo"] % 2) == 0
+    idx = []
+    for n in (64, 128, 256, 512, 1024):
+        cand = np.flatnonzero((N == n) & (P["microbatches"] == 8) & (P["dp"] <= 4) & (sym | (N == 64)))
+        idx += [int(cand[i]) for i in sample(len(cand), 5, 600 + n)]
+    sw = W.Sweep(full.name, full.trace, full.topos, P[sorted(set(idx))])
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all(), np.unique(got["status"], return_counts=True)
+    check(got, sw, list(range(len(sw.points))))
