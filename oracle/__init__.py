@@ -43,12 +43,12 @@ def lib():
             L = C.CDLL(LIB)
             P = C.c_void_p
             u32, i32, i64, f64 = C.c_uint32, C.c_int32, C.c_int64, C.c_double
-            L.oracle_run_point.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P, P]
+            L.oracle_run_point.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P, P, P]
             L.oracle_run_point.restype = C.c_int
             L.oracle_export_graph.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P,
                                               P, P, P, P, P, P, P, P, P, P, P, P, P]
             L.oracle_export_graph.restype = C.c_int
-            L.oracle_sim_graph.argtypes = [i64, P, P, P, P, P, P, P, P, P, P, i32, f64, u32, u32, P, u32, f64, f64, P, P]
+            L.oracle_sim_graph.argtypes = [i64, P, P, P, P, P, P, P, P, P, P, i32, f64, u32, u32, P, u32, f64, f64, P, P, P]
             L.oracle_sim_graph.restype = C.c_int
             L.oracle_route.argtypes = [u32, u32, P, u32, u32, u32, P, i32]
             L.oracle_route.restype = C.c_int
@@ -80,6 +80,11 @@ def _topo_args(topo: W.Topology):
     return (links, ro), [topo.n_nodes, topo.n_gpus, _p(links), len(links), _p(ro)]
 
 
+def _phot(topo: W.Topology):
+    ph = getattr(topo, "photonic", None)
+    return None if ph is None else np.ascontiguousarray(np.asarray(ph, W.PHOTONIC_DTYPE).reshape(1))
+
+
 class OracleError(RuntimeError):
     pass
 
@@ -91,8 +96,9 @@ def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None):
     pl = None if plan is None else np.ascontiguousarray(plan, np.uint32)
     ptv = np.array(pt, W.POINT_DTYPE).reshape(1)
     out = np.zeros(1, W.RESULT_DTYPE)
+    ph = _phot(topo)
     rc = lib().oracle_run_point(*ta, *tpa, _p(pl), 0 if pl is None else len(pl), 0 if pl is None else 1, _p(ptv),
-                                _p(out))
+                                _p(out), _p(ph))
     if rc != 0:
         raise OracleError(f"oracle_run_point rc={rc}")
     return out[0]
@@ -150,8 +156,9 @@ def sim_graph(g, topo: W.Topology, bw_scale=1.0, lat_scale=1.0, n_coll=0, coll_p
             (("type", np.int32), ("gpu", np.int32), ("dur", np.float64), ("src", np.int32), ("dst", np.int32),
              ("bytes", np.float64), ("code", np.uint64), ("flags", np.int32), ("dep_off", np.int64),
              ("dep_ids", np.int32))]
+    ph = _phot(topo)
     rc = lib().oracle_sim_graph(n, *[_p(a) for a in arrs], int(n_coll), float(coll_payload), *tpa[:4],
-                                float(bw_scale), float(lat_scale), _p(out), _p(td))
+                                float(bw_scale), float(lat_scale), _p(out), _p(td), _p(ph))
     if rc != 0:
         raise OracleError(f"sim_graph rc={rc}")
     return (out[0], td[:n]) if times else out[0]

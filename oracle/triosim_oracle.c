@@ -83,6 +83,16 @@ typedef struct {
     uint32_t max_active_flows;
 } OResult; /* 112 B */
 
+/* Photonic circuit-switched interconnect parameters (R20) */
+typedef struct {
+    uint32_t ports;      /* photonic ports per GPU (logical links it can hold) */
+    uint32_t buf_slots;  /* receive buffers per destination GPU (0 = unlimited) */
+    double link_bw;      /* bandwidth of one logical link, B/s */
+    double setup_s;      /* latency of establishing a logical link */
+    double lat_s;        /* per-transfer latency */
+} OPhot; /* 32 B */
+
+_Static_assert(sizeof(OPhot) == 32, "photonic record");
 _Static_assert(sizeof(OOp) == 40, "op record");
 _Static_assert(sizeof(OTensor) == 16, "tensor record");
 _Static_assert(sizeof(OLink) == 24, "link record");
@@ -377,6 +387,7 @@ typedef struct {
     uint32_t n_nodes, n_gpus, n_links;
     const OLink *links;
     int *adj_off, *adj_link;   /* per node, out-links sorted by dst */
+    const OPhot *ph;           /* non-NULL: photonic circuit-switched network (R20) instead of R12-R15 */
 } Topo;
 
 static const OLink *g_sort_links;
@@ -386,9 +397,13 @@ static int cmp_by_dst(const void *a, const void *b) {
     return (da > db) - (da < db);
 }
 
-static int topo_init(Topo *tp, uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links) {
-    tp->n_nodes = n_nodes; tp->n_gpus = n_gpus; tp->n_links = n_links; tp->links = links;
+static int topo_init(Topo *tp, uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links,
+                     const OPhot *ph) {
+    tp->n_nodes = n_nodes; tp->n_gpus = n_gpus; tp->n_links = n_links; tp->links = links; tp->ph = ph;
     if (n_gpus == 0 || n_gpus > n_nodes) return O_EINVAL;
+    if (ph && (ph->ports == 0 || !(ph->link_bw > 0.0) || isinf(ph->link_bw) || !(ph->setup_s >= 0.0) ||
+               isinf(ph->setup_s) || !(ph->lat_s >= 0.0) || isinf(ph->lat_s)))
+        return O_EINVAL;
     tp->adj_off = (int *)calloc(n_nodes + 1, sizeof(int));
     tp->adj_link = (int *)malloc(sizeof(int) * (n_links ? n_links : 1));
     if (!tp->adj_off || !tp->adj_link) return O_ENOMEM;
@@ -1126,6 +1141,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
         if (G->n[i].type != N_FLOW) continue;
         n_flows++;
         if (G->n[i].flags & NF_P2P) n_p2p++;
+        if (tp->ph) continue;   /* photonic: logical links instead of physical routes (R20) */
         int s = G->n[i].src, d = G->n[i].dst;
         long key = (long)s * n_nodes_topo + d;
         if (pair_len[key] == -9) {
@@ -1175,6 +1191,31 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
         for (long i = 0; i < NN; i++)
             if (pending[i] == 0 && G->n[i].type != N_TASK) { iv_push(&ready, (int)i); state[i] = S_QUEUED; }
 
+        /* R20 photonic circuit-switched network: per source GPU `ports` directed logical
+         * links {dst, state NONE/SETUP/UP, t = ready time (SETUP) or last use (UP)}; per flow a stage
+         * REQ (released, no link) -> LINKQ (queued on a link) -> BUFW (link head, waiting for a receive
+         * buffer at dst) -> XFER (delivered at t_drain).  Requests are ordered by (release time, code). */
+        const OPhot *ph = tp->ph;
+        const int PP_ = ph ? (int)ph->ports : 1;
+        int *lk_dst = NULL, *lk_st = NULL, *ph_st = NULL, *ph_lk = NULL, *tmpf = NULL;
+        double *lk_t = NULL;
+        IVec phl = {0};
+        double ph_setup = 0.0, ph_lat = 0.0, ph_bw = 1.0;
+        if (ph) {
+            lk_dst = (int *)malloc(sizeof(int) * (size_t)n_nodes_topo * PP_);
+            lk_st = (int *)calloc((size_t)n_nodes_topo * PP_, sizeof(int));
+            lk_t = (double *)calloc((size_t)n_nodes_topo * PP_, sizeof(double));
+            ph_st = (int *)calloc((size_t)(NN ? NN : 1), sizeof(int));
+            ph_lk = (int *)calloc((size_t)(NN ? NN : 1), sizeof(int));
+            tmpf = (int *)malloc(sizeof(int) * (size_t)(NN ? NN : 1));
+            for (long q = 0; q < (long)n_nodes_topo * PP_; q++) lk_dst[q] = -1;
+            ph_setup = ph->setup_s * lat_scale;
+            ph_lat = ph->lat_s * lat_scale;
+            ph_bw = ph->link_bw * bw_scale;
+        }
+        enum { PS_NONE = 0, PS_REQ = 1, PS_LINKQ = 2, PS_BUFW = 3, PS_XFER = 4 };
+#define PKEY_LT(a, b) (t_act[a] < t_act[b] || (t_act[a] == t_act[b] && G->n[a].code < G->n[b].code))
+
         long n_done = 0;
         double t = 0.0;
         uint64_t H = 0;
@@ -1204,6 +1245,10 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
             long nev = 0;
             int again;
             int dirty = 0;
+            /* R20: logical links whose setup completes now are up (last use = now) */
+            if (ph)
+                for (long q = 0; q < (long)n_nodes_topo * PP_; q++)
+                    if (lk_st[q] == 1 && lk_t[q] == t) lk_st[q] = 2;
             do {
                 int changed;
                 do {
@@ -1227,6 +1272,21 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                             EVENT(EV_DELIVER, G->n[f].code);
                             inflight--;
                             dirty = 1; changed = 1;
+                        } else {
+                            a++;
+                        }
+                    }
+                    /* (b') photonic deliveries: the logical link was last used now (R20) */
+                    for (long a = 0; a < phl.n;) {
+                        int f = phl.v[a];
+                        if (ph_st[f] == PS_XFER && t_drain[f] == t) {
+                            phl.v[a] = phl.v[--phl.n];
+                            ph_st[f] = PS_NONE;
+                            lk_t[G->n[f].src * PP_ + ph_lk[f]] = t;
+                            COMPLETE(f);
+                            EVENT(EV_DELIVER, G->n[f].code);
+                            inflight--;
+                            changed = 1;
                         } else {
                             a++;
                         }
@@ -1258,6 +1318,21 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         if (G->n[k].type == N_BARRIER) {
                             COMPLETE(k);
                             if (G->n[k].flags & NF_COLL_START) EVENT(EV_COLL_START, G->n[k].code);
+                        } else if (ph) {
+                            /* R20: a send request; t_act holds its release time (the FIFO key) */
+                            EVENT(EV_RELEASE, G->n[k].code);
+                            inflight++;
+                            if (G->n[k].src == G->n[k].dst) {
+                                EVENT(EV_ACTIVATE, G->n[k].code);
+                                COMPLETE(k);
+                                EVENT(EV_DELIVER, G->n[k].code);
+                                inflight--;
+                            } else {
+                                state[k] = S_LATENT;
+                                t_act[k] = t;
+                                ph_st[k] = PS_REQ;
+                                iv_push(&phl, k);
+                            }
                         } else {
                             state[k] = S_LATENT;
                             t_act[k] = t + lat[k];
@@ -1279,9 +1354,91 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         changed = 1;
                     }
                 } while (changed);
-                /* (f) re-allocate bandwidth of every in-transit flow (P:210, P:216) */
                 again = 0;
-                if (dirty) {
+                if (ph) {
+                    /* R20: (i) link per request: an existing link to dst, else a free port,
+                     * else tear down the source's link idle the longest (ties: smaller dst), else wait */
+                    for (int g = 0; g < n_nodes_topo; g++) {
+                        int nr = 0;
+                        for (long a = 0; a < phl.n; a++)
+                            if (ph_st[phl.v[a]] == PS_REQ && G->n[phl.v[a]].src == g) tmpf[nr++] = phl.v[a];
+                        for (int x = 1; x < nr; x++)   /* insertion sort by (release time, code) */
+                            for (int y = x; y > 0 && PKEY_LT(tmpf[y], tmpf[y - 1]); y--) {
+                                int sw = tmpf[y]; tmpf[y] = tmpf[y - 1]; tmpf[y - 1] = sw;
+                            }
+                        for (int x = 0; x < nr; x++) {
+                            int f = tmpf[x], d = G->n[f].dst, k = -1;
+                            for (int q = 0; q < PP_; q++) if (lk_st[g * PP_ + q] != 0 && lk_dst[g * PP_ + q] == d) k = q;
+                            if (k < 0) {
+                                int nk = -1;
+                                for (int q = 0; q < PP_ && nk < 0; q++) if (lk_st[g * PP_ + q] == 0) nk = q;
+                                if (nk < 0) {
+                                    for (int q = 0; q < PP_; q++) {
+                                        if (lk_st[g * PP_ + q] != 2) continue;
+                                        int used = 0;
+                                        for (long a = 0; a < phl.n && !used; a++) {
+                                            int h = phl.v[a];
+                                            if (G->n[h].src == g && ph_st[h] >= PS_LINKQ && ph_lk[h] == q) used = 1;
+                                        }
+                                        if (used) continue;
+                                        if (nk < 0 || lk_t[g * PP_ + q] < lk_t[g * PP_ + nk] ||
+                                            (lk_t[g * PP_ + q] == lk_t[g * PP_ + nk] && lk_dst[g * PP_ + q] < lk_dst[g * PP_ + nk]))
+                                            nk = q;
+                                    }
+                                }
+                                if (nk >= 0) {
+                                    const double tr = t + ph_setup;
+                                    lk_dst[g * PP_ + nk] = d;
+                                    if (tr == t) { lk_st[g * PP_ + nk] = 2; lk_t[g * PP_ + nk] = t; }
+                                    else { lk_st[g * PP_ + nk] = 1; lk_t[g * PP_ + nk] = tr; }
+                                    k = nk;
+                                }
+                            }
+                            if (k >= 0) { ph_st[f] = PS_LINKQ; ph_lk[f] = k; }
+                        }
+                    }
+                    /* (ii) an up link with no transfer waiting or running passes its queue head on */
+                    for (int g = 0; g < n_nodes_topo; g++)
+                        for (int q = 0; q < PP_; q++) {
+                            if (lk_st[g * PP_ + q] != 2) continue;
+                            int busy = 0, head = -1;
+                            for (long a = 0; a < phl.n; a++) {
+                                int h = phl.v[a];
+                                if (G->n[h].src != g || ph_lk[h] != q || ph_st[h] < PS_LINKQ) continue;
+                                if (ph_st[h] >= PS_BUFW) busy = 1;
+                                else if (head < 0 || PKEY_LT(h, head)) head = h;
+                            }
+                            if (!busy && head >= 0) ph_st[head] = PS_BUFW;
+                        }
+                    /* (iii) receive buffers at each destination, granted in (release time, code) order;
+                     * a granted transfer owns the link's dedicated bandwidth: t + lat + bytes / bw */
+                    int nx = 0;
+                    for (int d = 0; d < n_nodes_topo; d++) {
+                        int occ = 0, nc = 0;
+                        for (long a = 0; a < phl.n; a++) {
+                            int h = phl.v[a];
+                            if (G->n[h].dst != d) continue;
+                            if (ph_st[h] == PS_XFER) occ++;
+                            else if (ph_st[h] == PS_BUFW) tmpf[nc++] = h;
+                        }
+                        for (int x = 1; x < nc; x++)
+                            for (int y = x; y > 0 && PKEY_LT(tmpf[y], tmpf[y - 1]); y--) {
+                                int sw = tmpf[y]; tmpf[y] = tmpf[y - 1]; tmpf[y - 1] = sw;
+                            }
+                        int fr = ph->buf_slots ? (int)ph->buf_slots - occ : nc;
+                        for (int x = 0; x < nc && x < fr; x++) {
+                            int f = tmpf[x];
+                            ph_st[f] = PS_XFER;
+                            t_drain[f] = (t + ph_lat) + G->n[f].bytes / ph_bw;
+                            EVENT(EV_ACTIVATE, G->n[f].code);
+                            if (t_drain[f] == t) again = 1;
+                        }
+                    }
+                    for (long a = 0; a < phl.n; a++) if (ph_st[phl.v[a]] == PS_XFER) nx++;
+                    if ((uint32_t)nx > max_act) max_act = (uint32_t)nx;
+                }
+                /* (f) re-allocate bandwidth of every in-transit flow (P:210, P:216) */
+                if (!ph && dirty) {
                     dirty = 0;
                     int nf = (int)active.n;
                     for (int a = 0; a < nf; a++) {
@@ -1313,11 +1470,16 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
             for (int g = 0; g < n_nodes_topo; g++) if (running[g] >= 0 && t_end[running[g]] < tn) tn = t_end[running[g]];
             for (long a = 0; a < latent.n; a++) if (t_act[latent.v[a]] < tn) tn = t_act[latent.v[a]];
             for (long a = 0; a < active.n; a++) if (t_drain[active.v[a]] < tn) tn = t_drain[active.v[a]];
+            if (ph) {
+                for (long a = 0; a < phl.n; a++) if (ph_st[phl.v[a]] == PS_XFER && t_drain[phl.v[a]] < tn) tn = t_drain[phl.v[a]];
+                for (long q = 0; q < (long)n_nodes_topo * PP_; q++) if (lk_st[q] == 1 && lk_t[q] < tn) tn = lk_t[q];
+            }
             if (!(tn < INFINITY)) { status = PT_DEADLOCK; break; }
             t = tn;
         }
 #undef COMPLETE
 #undef EVENT
+#undef PKEY_LT
         if (status == PT_OK) {
             res->iter_time_s = t;
             res->compute_busy_max_s = cbmax;
@@ -1339,6 +1501,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
         free(state); free(t_end); free(t_act); free(rem); free(rate); free(t_upd); free(t_drain); free(has_dependents);
         iv_free(&ready); iv_free(&latent); iv_free(&active);
         free(wf_flows); free(wf_rate); free(wf_unf);
+        free(lk_dst); free(lk_st); free(lk_t); free(ph_st); free(ph_lk); free(tmpf); iv_free(&phl);
     }
 out:
     free(doff); free(roff); free(dlist); free(rlist); free(pending);
@@ -1388,11 +1551,11 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
 int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
                      uint32_t n_io, uint32_t trace_batch, uint32_t n_nodes, uint32_t n_gpus, const OLink *links,
                      uint32_t n_links, const uint32_t *ring_order, const uint32_t *plan, uint32_t plan_len,
-                     int have_plan, const OPoint *pt, OResult *out) {
+                     int have_plan, const OPoint *pt, OResult *out, const OPhot *ph) {
     Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
     Topo tp; memset(&tp, 0, sizeof tp);
     int rc = trace_check(&T);
-    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links, ph);
     if (rc == O_OK && ring_order) {
         for (uint32_t i = 0; i < n_gpus; i++) {
             if (ring_order[i] >= n_gpus) rc = O_EINVAL;
@@ -1421,7 +1584,7 @@ int oracle_export_graph(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint3
     Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
     Topo tp; memset(&tp, 0, sizeof tp);
     int rc = trace_check(&T);
-    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    if (rc == O_OK) rc = topo_init(&tp, n_nodes, n_gpus, links, n_links, NULL);
     if (rc != O_OK) { free(T.prod); topo_free(&tp); return rc; }
     Graph G; memset(&G, 0, sizeof G);
     int st = PT_OK;
@@ -1454,9 +1617,9 @@ int oracle_sim_graph(int64_t n, const int32_t *type, const int32_t *gpu, const d
                      const int32_t *dst, const double *bytes, const uint64_t *code, const int32_t *flags,
                      const int64_t *dep_off, const int32_t *dep_ids, int32_t n_coll, double coll_payload,
                      uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links, double bw_scale,
-                     double lat_scale, OResult *out, double *t_done) {
+                     double lat_scale, OResult *out, double *t_done, const OPhot *ph) {
     Topo tp; memset(&tp, 0, sizeof tp);
-    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links, ph);
     if (rc != O_OK) { topo_free(&tp); return rc; }
     Graph G; memset(&G, 0, sizeof G);
     for (int64_t i = 0; i < n; i++) {
@@ -1483,7 +1646,7 @@ int oracle_sim_graph(int64_t n, const int32_t *type, const int32_t *gpu, const d
 int oracle_route(uint32_t n_nodes, uint32_t n_gpus, const OLink *links, uint32_t n_links, uint32_t src, uint32_t dst,
                  int32_t *out_links, int32_t cap) {
     Topo tp; memset(&tp, 0, sizeof tp);
-    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links);
+    int rc = topo_init(&tp, n_nodes, n_gpus, links, n_links, NULL);
     if (rc != O_OK) { topo_free(&tp); return -100 + rc; }
     int *tmp = (int *)malloc(sizeof(int) * (size_t)(n_nodes + 1));
     int h = bfs_route(&tp, (int)src, (int)dst, tmp, (int)n_nodes);

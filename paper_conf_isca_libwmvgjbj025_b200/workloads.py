@@ -39,6 +39,8 @@ POINT_DTYPE = np.dtype([
     ("dp", "<u2"), ("tp", "<u2"), ("pp", "<u2"), ("pad1", "<u2"),
     ("microbatches", "<u4"), ("global_batch", "<u4"), ("stage_plan", "<i4"), ("pad2", "<u4"),
     ("bucket_bytes", "<u8"), ("bw_scale", "<f8"), ("lat_scale", "<f8")])
+PHOTONIC_DTYPE = np.dtype([("ports", "<u4"), ("buf_slots", "<u4"), ("link_bw_Bps", "<f8"), ("setup_s", "<f8"),
+                           ("lat_s", "<f8")])
 RESULT_DTYPE = np.dtype([
     ("iter_time_s", "<f8"), ("compute_busy_max_s", "<f8"), ("comm_busy_s", "<f8"),
     ("exposed_comm_s", "<f8"), ("coll_payload_bytes", "<f8"),
@@ -491,6 +493,7 @@ class Topology:
     n_gpus: int
     links: np.ndarray       # LINK_DTYPE
     ring_order: np.ndarray  # uint32[n_gpus]
+    photonic: object = None  # PHOTONIC_DTYPE record: circuit-switched photonic network (R20)
 
 
 def _mk(name, n_nodes, n_gpus, edges, ring_order, bidir=True):
@@ -534,6 +537,29 @@ def mesh(r, c, bw=1.0, lat=1.0):
         row = [i * c + j for j in range(c)]
         order += row if i % 2 == 0 else row[::-1]
     return _mk(f"mesh{r}x{c}", r * c, r * c, e, order)
+
+
+def wafer_mesh(rows=12, cols=7, bw=1.0, lat=1.0):
+    """The Passage case study's electrical baseline: a rows x cols wafer of GPUs on a 2D mesh whose
+    ring order is a Hamiltonian cycle of the mesh ("we use the mesh network on the wafer to form a
+    ring"): down column 0, then boustrophedon rows over columns 1..cols-1 back to row 0 (rows even)."""
+    assert rows % 2 == 0
+    t = mesh(rows, cols, bw, lat)
+    order = [r * cols for r in range(rows)]
+    for k, r in enumerate(range(rows - 1, -1, -1)):
+        row = [r * cols + j for j in range(1, cols)]
+        order += row if k % 2 == 0 else row[::-1]
+    return Topology(f"wafer{rows}x{cols}", t.n_nodes, t.n_gpus, t.links, np.asarray(order, np.uint32))
+
+
+def photonic(n_gpus, ports=8, link_bw=484e9 / 8, setup=20e-3, lat=0.0, buf_slots=0, ring_order=None, name=None):
+    """Circuit-switched photonic interconnect (Lightmatter Passage; R20): every GPU
+    can hold `ports` logical links (484 GB/s across 8 links, 20 ms to establish a link); no
+    physical links.  Points carry bw_scale / lat_scale as usual."""
+    ph = np.zeros((), PHOTONIC_DTYPE)
+    ph["ports"], ph["buf_slots"], ph["link_bw_Bps"], ph["setup_s"], ph["lat_s"] = ports, buf_slots, link_bw, setup, lat
+    ro = np.arange(n_gpus, dtype=np.uint32) if ring_order is None else np.asarray(ring_order, np.uint32)
+    return Topology(name or f"photonic{n_gpus}p{ports}", n_gpus, n_gpus, np.zeros(0, LINK_DTYPE), ro, ph)
 
 
 def cube_mesh8(bw=1.0, lat=1.0):
