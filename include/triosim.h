@@ -45,7 +45,7 @@ typedef int32_t triosim_status;
 #define TRIOSIM_PT_BAD_BATCH 1   /* global_batch not divisible by dp * microbatches (Q3, Q12) */
 #define TRIOSIM_PT_BAD_DEGREES 2 /* zero / inconsistent degrees, dp*tp*pp > GPUs, pp > layers or > 64 */
 #define TRIOSIM_PT_NO_ROUTE 3    /* a needed (src, dst) GPU pair has no path */
-#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 32 lanes, > 128 links (256 hybrid), > 8 hops) */
+#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 1024 ranks, > 12288 links, > 8 hops) */
 #define TRIOSIM_PT_DEADLOCK 5    /* the task graph cannot make progress */
 #define TRIOSIM_PT_BAD_PLAN 6    /* explicit stage plan invalid for this point */
 #define TRIOSIM_PT_BAD_CONFIG 7  /* unknown enum, topology index out of range, bw_scale <= 0, lat_scale < 0 */
@@ -107,10 +107,30 @@ typedef struct {
     double lat_s;       /* >= 0 */
 } triosim_link;         /* 24 B */
 
+/* Photonic circuit-switched interconnect (Lightmatter Passage case study; R20).
+ * A send (1) establishes a directed logical link src -> dst if none exists, taking setup_s, on one of
+ * the sender's `ports` photonic ports; with no free port it tears down the sender's link that has been
+ * idle the longest; (2) waits for a receive buffer at the destination (buf_slots per GPU,
+ * 0 = unlimited); (3) moves the data at the link's dedicated bandwidth: delivered lat_s + bytes /
+ * link_bw_Bps after the buffer is granted.  Requests are served in (release time, flow id) order.
+ * The point's bw_scale multiplies link_bw_Bps, lat_scale multiplies setup_s and lat_s. */
 typedef struct {
-    uint32_t n_nodes, n_gpus, n_links, pad;
+    uint32_t ports;       /* 1..8 */
+    uint32_t buf_slots;   /* receive buffers per GPU, 0 = unlimited */
+    double link_bw_Bps;   /* > 0: bandwidth of one logical link (484 GB/s across 8 links) */
+    double setup_s;       /* >= 0: latency of establishing a logical link (20 ms) */
+    double lat_s;         /* >= 0: latency of one transfer */
+} triosim_photonic;       /* 32 B */
+
+#define TRIOSIM_NET_FLOW 0      /* links + routes, max-min fair flow model (R12-R15) */
+#define TRIOSIM_NET_PHOTONIC 1  /* logical links of a circuit-switched photonic interposer (R20) */
+
+typedef struct {
+    uint32_t n_nodes, n_gpus, n_links;
+    uint32_t net_model;             /* TRIOSIM_NET_*; PHOTONIC ignores links (n_links may be 0) */
     const triosim_link *links;      /* at most one link per ordered pair */
     const uint32_t *ring_order;     /* permutation of [0, n_gpus) or NULL (= identity) */
+    const triosim_photonic *photonic;  /* required iff net_model == PHOTONIC, else ignored */
 } triosim_topology;
 
 /* Explicit PP stage plans: plan k has first_layer[off[k] .. off[k+1]) (first must be 0,
@@ -160,6 +180,7 @@ static_assert(sizeof(triosim_op) == 40, "op");
 static_assert(sizeof(triosim_tensor) == 16, "tensor");
 static_assert(sizeof(triosim_link) == 24, "link");
 static_assert(sizeof(triosim_point) == 56, "point");
+static_assert(sizeof(triosim_photonic) == 32, "photonic");
 static_assert(sizeof(triosim_result) == 112, "result");
 #endif
 
@@ -180,7 +201,8 @@ const char *triosim_last_error(const triosim_ctx *ctx);
 triosim_status triosim_load_trace(triosim_ctx *ctx, const triosim_trace_desc *t, int32_t *trace_id);
 
 /* Build a sweep of n_pts design points over trace_id (P:142 inputs).  Validates topologies
- * (EINVAL: bad endpoints, bw <= 0, lat < 0, duplicate ordered pair, bad ring_order), computes
+ * (EINVAL: bad endpoints, bw <= 0, lat < 0, duplicate ordered pair, bad ring_order, unknown net_model,
+ * photonic parameters missing or out of range), computes
  * routes (S5) and stage partitions on the host, groups points into structural classes and
  * stages everything in device memory.  Invalid design points do NOT fail the call: they get a
  * per-point status.  plans may be NULL.  Synchronous.  *sweep_id receives the handle. */

@@ -99,6 +99,7 @@ struct Sweep {
     DevBuf<uint32_t> d_work_tmp[N_GROUPS];
     std::vector<int> mode;                   // per point
     uint32_t lmax[N_GROUPS] = {};            // hybrid CTA groups: largest topology (links) among their points
+    uint32_t pmax[N_GROUPS] = {};            // hybrid groups: most photonic ports among their points (R20)
     int occ[N_GROUPS] = {};                  // hybrid CTA groups: resident CTAs per SM at that smem
     DevBuf<unsigned int> d_counter;
     DevBuf<unsigned long long> d_alg;
@@ -167,7 +168,7 @@ triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
             return TRIOSIM_ECUDA;
         }
         const int Wi = W_OF[i / N_MODES], md = i % N_MODES;
-        ctx->occ[i] = md == MODE_HYBRID ? (Wi <= 32 ? k3h_max_blocks_per_sm(Wi, 0) : 1)
+        ctx->occ[i] = md == MODE_HYBRID ? (Wi <= 32 ? k3h_max_blocks_per_sm(Wi, 0, 0) : 1)
                                         : Wi <= 32 ? k3_max_blocks_per_sm(Wi, md) : 1;
     }
     if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
@@ -329,6 +330,8 @@ static std::vector<uint32_t> auto_partition(const Trace &T, int S) {
 
 struct HostTopo {
     uint32_t n_nodes, n_gpus, n_links, max_hops;
+    bool photonic = false;
+    triosim_photonic ph = {};
     std::vector<uint32_t> ro;
     std::vector<uint32_t> rt_off;   // n_gpus^2
     std::vector<uint8_t> rt_len;
@@ -339,6 +342,17 @@ static triosim_status prep_topology(triosim_ctx *ctx, const triosim_topology &tp
     if (tp.n_gpus == 0 || tp.n_gpus > tp.n_nodes || (tp.n_links && !tp.links))
         return fail(ctx, TRIOSIM_EINVAL, "topology %u: bad sizes", idx);
     H.n_nodes = tp.n_nodes; H.n_gpus = tp.n_gpus; H.n_links = tp.n_links; H.max_hops = 0;
+    if (tp.net_model > TRIOSIM_NET_PHOTONIC) return fail(ctx, TRIOSIM_EINVAL, "topology %u: unknown net_model", idx);
+    H.photonic = tp.net_model == TRIOSIM_NET_PHOTONIC;
+    if (H.photonic) {
+        if (!tp.photonic) return fail(ctx, TRIOSIM_EINVAL, "topology %u: photonic parameters missing", idx);
+        H.ph = *tp.photonic;
+        const triosim_photonic &P = H.ph;
+        if (P.ports == 0 || P.ports > (uint32_t)MAX_PORTS || !(P.link_bw_Bps > 0.0) || std::isinf(P.link_bw_Bps) ||
+            !(P.setup_s >= 0.0) || std::isinf(P.setup_s) || !(P.lat_s >= 0.0) || std::isinf(P.lat_s))
+            return fail(ctx, TRIOSIM_EINVAL, "topology %u: photonic ports must be 1..%d, bw > 0, setup/lat >= 0",
+                        idx, MAX_PORTS);
+    }
     std::vector<std::vector<std::pair<uint32_t, uint32_t>>> adj(tp.n_nodes);
     std::vector<std::vector<uint32_t>> seen(tp.n_nodes);
     for (uint32_t e = 0; e < tp.n_links; e++) {
@@ -484,19 +498,25 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto lm = [&](bool h, int w) { return !h ? lmax_warp(w) : w <= 32 ? lmax_hybrid(w) : LMAX_CTA; };
         int W0 = 2;
         while (W0 < (int)lanes) W0 <<= 1;
+        // photonic points (R20) always run in the HYBRID kernel, whose lanes own their logical links;
+        // DataParallel maps to HYBRID with its buckets triggered after the backward pass
         int W = 0;
-        if (pt.strategy != TRIOSIM_HYBRID)
+        bool dp_after = false;
+        if (pt.strategy != TRIOSIM_HYBRID && !tp.photonic)
             for (int w = W0; w <= 32; w <<= 1)
                 if ((int)tp.n_links <= lm(false, w)) { W = w; break; }
-        if (W == 0 && (pt.strategy == TRIOSIM_HYBRID || pt.strategy == TRIOSIM_DDP || pt.strategy == TRIOSIM_TP ||
-                       pt.strategy == TRIOSIM_PP)) {
+        if (W == 0) {
             if (pt.strategy != TRIOSIM_HYBRID) {
+                dp_after = pt.strategy == TRIOSIM_DP;
                 if (pt.strategy != TRIOSIM_PP) pt.microbatches = 1;
                 pt.strategy = TRIOSIM_HYBRID;
             }
             for (int w = W0; w <= 1024; w <<= 1)
-                if ((int)tp.n_links <= lm(true, w)) { W = w; break; }
+                if (tp.photonic || (int)tp.n_links <= lm(true, w)) { W = w; break; }
         }
+        // photonic tree collectives: a broadcast flow parent -> child lives in the child's lane but needs the
+        // parent's logical links (ports are the sender's, R20); not supported by this kernel
+        if (tp.photonic && pt.coll_algo == TRIOSIM_ALGO_TREE && pt.strategy != TRIOSIM_PP) W = 0;
         if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
         const uint32_t mbe = pt.microbatches;   // after a DDP / TP -> HYBRID mapping this is 1
         // structural class
@@ -509,7 +529,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         int key_algo = mode != MODE_PIPE ? pt.coll_algo : 0;
         uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP || hyb) ? pt.bucket_bytes : 0;
         int key_m = (mode == MODE_PIPE || hyb) ? (int)mbe : 0;
-        auto key = std::make_tuple((int)pt.strategy, (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
+        auto key = std::make_tuple((int)pt.strategy + (dp_after ? 100 : 0), (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
                                    hyb ? (int)tpd : 0, key_algo, key_bucket, key_m,
                                    (mode == MODE_PIPE || hyb) ? plan_key : -2);
         auto ci = cls_of.find(key);
@@ -519,6 +539,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             std::memset(&cd, 0, sizeof cd);
             cd.mode = mode;
             cd.strategy = pt.strategy;
+            cd.dp_after_bwd = dp_after ? 1u : 0u;
             cd.tp_mode = key_mode;
             cd.algo = key_algo;
             cd.p = hyb ? pp : lanes;
@@ -622,7 +643,10 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         d.ro_off = (uint32_t)ro.size();
         ro.insert(ro.end(), HT[i].ro.begin(), HT[i].ro.end());
         d.ring_disjoint_lo = d.ring_disjoint_hi = 0;
-        {
+        d.net = HT[i].photonic ? TRIOSIM_NET_PHOTONIC : TRIOSIM_NET_FLOW;
+        d.ports = HT[i].ph.ports; d.buf_slots = HT[i].ph.buf_slots; d.pad = 0;
+        d.ph_bw = HT[i].ph.link_bw_Bps; d.ph_setup = HT[i].ph.setup_s; d.ph_lat = HT[i].ph.lat_s;
+        if (!HT[i].photonic) {
             const HostTopo &Ht = HT[i];
             const uint32_t G = Ht.n_gpus;
             for (uint32_t pp = 2; pp <= std::min<uint32_t>(G, 32); pp++) {
@@ -684,14 +708,15 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     for (uint64_t i : order) {
         const int g = N_MODES * w_index(S->width[i]) + S->mode[i];
         S->work[g].push_back((uint32_t)i);
-        if (S->width[i] > 32) {
-            const uint32_t nl = HT[pts[i].topo].n_links;
-            const uint32_t r = (nl + 63) / 64 * 64;
+        const HostTopo &ht = HT[pts[i].topo];
+        if (S->width[i] > 32 && !ht.photonic) {
+            const uint32_t r = (ht.n_links + 63) / 64 * 64;
             if (r > S->lmax[g]) S->lmax[g] = r;
         }
+        if (ht.photonic && ht.ph.ports > S->pmax[g]) S->pmax[g] = ht.ph.ports;
     }
     for (int g = 0; g < N_GROUPS; g++)
-        if (S->lmax[g]) S->occ[g] = k3h_max_blocks_per_sm(W_OF[g / N_MODES], S->lmax[g]);
+        if (S->lmax[g] || S->pmax[g]) S->occ[g] = k3h_max_blocks_per_sm(W_OF[g / N_MODES], S->lmax[g], S->pmax[g]);
     for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
         CK(S->d_work_tmp[w].alloc(S->work[w].size()));
@@ -771,6 +796,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         a.out = S.d_res.p;
         a.alg_ops = S.d_alg.p;
         a.lmax = S.lmax[w];
+        a.pmax = S.pmax[w];
         uint64_t blocks;
         if (W <= 32) {
             const int nseg = 32 / W;
@@ -779,7 +805,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         } else {
             blocks = n;   // one point per CTA
         }
-        const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)(S.lmax[w] ? S.occ[w] : ctx->occ[w]);
+        const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)((S.lmax[w] || S.pmax[w]) ? S.occ[w] : ctx->occ[w]);
         if (blocks > cap) blocks = cap;
         CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
         if (mode == MODE_HYBRID) CK(launch_k3_hybrid(W, a, (int)blocks, ctx->side[w]));

@@ -110,7 +110,8 @@ struct ClassDesc {
     uint32_t plan_off, stage_off, ent_off, ent_cap;
     uint32_t send_off, send_cap, recv_off, recv_cap;
     uint32_t scratch_off, dp;            // dp: HYBRID data-parallel degree
-    uint32_t hst_off, tcol_off, tcol_cap, dcol_off, dcol_cap, pad1;   // HYBRID pools
+    uint32_t hst_off, tcol_off, tcol_cap, dcol_off, dcol_cap;   // HYBRID pools
+    uint32_t dp_after_bwd;               // HYBRID form of DataParallel: DP buckets trigger after the backward pass
     // written by K2
     uint32_t n_coll, need_ring, need_tree, n_prog_max;
     double coll_payload;
@@ -123,6 +124,9 @@ struct TopoDev {
     // bit p (p = 2..32 over the two words): the routes ring_order[i] -> ring_order[(i+1) % p] of
     // the first p GPUs are pairwise link-disjoint, so ring flows never share a link (K3 fast path)
     uint32_t ring_disjoint_lo, ring_disjoint_hi;
+    // photonic circuit-switched network (R20); net == TRIOSIM_NET_FLOW: unused
+    uint32_t net, ports, buf_slots, pad;
+    double ph_bw, ph_setup, ph_lat;
 };
 
 struct PointDesc {
@@ -134,6 +138,7 @@ struct K3Args {
     const PointDesc *pts;
     const uint32_t *work;
     uint32_t n_work, lmax;         // lmax: links per segment in dynamic smem (one-point-per-CTA hybrid)
+    uint32_t pmax, pad2;           // pmax: photonic ports per lane in dynamic smem (hybrid, R20)
     unsigned int *counter;
     const ClassDesc *cls;
     const TopoDev *topo;
@@ -169,8 +174,8 @@ cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, c
                              RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s);      // ts_k3h.cu
-int k3h_max_blocks_per_sm(int W, uint32_t lmax);   // lmax: dynamic-smem links (W > 32)
-size_t k3h_dyn_smem(int W, uint32_t lmax);
+int k3h_max_blocks_per_sm(int W, uint32_t lmax, uint32_t pmax);   // dynamic smem: links (W > 32), ports
+size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax);
 int k3_max_blocks_per_sm(int W, int mode);
 // links per segment the K3 kernels keep in shared memory
 __host__ __device__ constexpr int lmax_warp(int W) { return 4 * W < 8 ? 8 : 4 * W; }
@@ -179,5 +184,6 @@ constexpr int LMAX_CTA = 12288;         // links of a one-point-per-CTA hybrid s
 constexpr int N_WIDTHS = 10;            // W = 2, 4, 8, 16, 32 (warp segments), 64 ... 1024 (hybrid CTAs)
 constexpr int N_MODES = 4;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
+constexpr int MAX_PORTS = 8;            // photonic ports per GPU the hybrid kernel holds (R20)
 
 }  // namespace ts

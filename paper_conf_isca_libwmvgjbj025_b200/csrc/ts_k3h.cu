@@ -17,7 +17,8 @@ namespace ts {
 namespace {
 
 enum { CS_IDLE = 0, CS_RUN = 1 };
-enum { FS_NONE = 0, FS_LAT = 1, FS_ACT = 2 };
+enum { FS_NONE = 0, FS_LAT = 1, FS_ACT = 2 };   // FS_ACT: draining (flow network) / transferring (photonic)
+enum { PS_REQ = 3, PS_LINKQ = 4, PS_BUFW = 5 };  // photonic (R20): no link yet, queued on a link, awaiting a buffer
 enum { EV_COLL_START = 1, EV_RELEASE = 2, EV_ACTIVATE = 3, EV_DELIVER = 4, EV_TASK_START = 5, EV_TASK_END = 6 };
 
 __device__ __forceinline__ uint64_t mix64(uint64_t z) {
@@ -55,6 +56,7 @@ __device__ __forceinline__ unsigned long long seg_sum_u64(unsigned long long v) 
 
 struct Topo {
     uint32_t n_gpus, link_off, rt_off, ro_off;
+    bool phot;
 };
 
 struct Flow {
@@ -99,9 +101,26 @@ __device__ __forceinline__ int route_len(const K3Args &a, const Topo &T, uint32_
     return a.rt_len[T.rt_off + s * T.n_gpus + d];
 }
 
-// release flow f along src -> dst: route latency fold (R12), link ids cached (<= 8 hops)
+// release flow f along src -> dst: route latency fold (R12), link ids cached (<= 8 hops).  Photonic
+// (R20): a send request keyed by (release time t_upd, code); hl[0] = destination GPU, hl[1] = link slot
 __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f, uint32_t src, uint32_t dst,
                                         double bytes, uint64_t code, double t, double lats, uint64_t &alg) {
+    if (T.phot) {
+        f.len = 0;
+        f.bytes = bytes;
+        f.code = code;
+        f.hl[0] = dst;
+        f.hl[1] = 0;
+        f.t_upd = t;
+        if (src == dst) {          // nothing to move: activation and delivery now (as an empty route)
+            f.st = FS_LAT;
+            f.t_act = t;
+        } else {
+            f.st = PS_REQ;
+            f.t_act = __longlong_as_double(0x7ff0000000000000ll);
+        }
+        return;
+    }
     const uint32_t k = T.rt_off + src * T.n_gpus + dst;
     const int len = a.rt_len[k];
     const uint32_t off = a.rt_off[k];
@@ -138,6 +157,18 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     __shared__ int s_k[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
     extern __shared__ double s_dyn[];
     const int LMAX = NW == 1 ? LMAXW : (int)a.lmax;
+    // photonic tables (R20) after the CTA link arrays: per lane a.pmax logical links {dst GPU, state
+    // 0 none / 1 setup / 2 up, t = ready time or last use} and per flow slot its buffer request
+    constexpr int NTHR = NW == 1 ? K3_THREADS : 32 * NW;
+    const int PM = (int)a.pmax;
+    double *p_t = s_dyn + (NW == 1 ? 0 : 2 * LMAX);
+    int *p_dst = (int *)(p_t + NTHR * PM);
+    int *p_st = p_dst + NTHR * PM;
+    double *q_t = (double *)(p_st + NTHR * PM);               // [3 * NTHR] request key time
+    unsigned long long *q_code = (unsigned long long *)(q_t + 3 * NTHR);
+    int *q_dst = (int *)(q_code + 3 * NTHR);                   // destination GPU or -1
+    uint8_t *q_st = (uint8_t *)(q_dst + 3 * NTHR);             // 1 waiting for a buffer, 2 transferring
+    uint8_t *q_g = q_st + 3 * NTHR;                            // granted
     __shared__ uint32_t s_cnt[NSLOT][NW == 1 ? 32 : SL];
     __shared__ double s_red[2][NW];
     __shared__ unsigned long long s_red64[2][NW];
@@ -162,6 +193,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     }
     if constexpr (NW > 1) {
         s_gc[0][threadIdx.x] = s_gc[1][threadIdx.x] = s_gc[2][threadIdx.x] = 0;
+    }
+    if (PM > 0) {
+        for (int k = 0; k < PM; k++) p_st[k * NTHR + threadIdx.x] = 0;
+        for (int k = 0; k < 3; k++) q_g[threadIdx.x * 3 + k] = 0;
     }
     int bb = 0;   // double-buffer toggle of the block-level exchanges (NW > 1)
     int fb = 0;   // double-buffer toggle of the tree-flag exchange (NW > 1)
@@ -273,11 +308,13 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     bool have = false, exhausted = false;
     uint32_t pidx = 0;
     double t = 0.0, bws = 1.0, lats = 1.0;
+    double ph_bw = 1.0, ph_set = 0.0, ph_lat = 0.0;   // photonic (R20), scaled by the point
+    int ports = 0, bufs = 0;
     int R = 1, S = 1, tp = 1, dp = 1;
     uint32_t m = 1;
     bool tree_algo = false;
     const ClassDesc *C = nullptr;
-    Topo TR = {0, 0, 0, 0};
+    Topo TR = {0, 0, 0, 0, false};
     uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
     bool bon = false;
     double bstart = 0.0, cbusy = 0.0;
@@ -427,7 +464,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         if (F.st == FS_ACT && F.t_drain == t) {
             F.st = FS_NONE;
             EV(EV_DELIVER, F.code);
-            dirty = true;
+            if (TR.phot) p_t[F.hl[1] * NTHR + threadIdx.x] = t;   // R20: the logical link was last used now
+            else dirty = true;
             return true;
         }
         if (F.st == FS_LAT && F.t_act == t) {
@@ -498,6 +536,12 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     {
                         const TopoDev td = a.topo[pd.topo];
                         TR.n_gpus = td.n_gpus; TR.link_off = td.link_off; TR.rt_off = td.rt_off; TR.ro_off = td.ro_off;
+                        TR.phot = td.net == TRIOSIM_NET_PHOTONIC;
+                        ports = (int)td.ports;
+                        bufs = (int)td.buf_slots;
+                        ph_bw = td.ph_bw * bws;
+                        ph_set = td.ph_setup * lats;
+                        ph_lat = td.ph_lat * lats;
                     }
                     S = (int)C->p;
                     tp = (int)C->tpdeg;
@@ -533,7 +577,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     grp_init(GT, used && tp > 1, tp, tt, (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp, d * S + s);
                     grp_init(GD, used && dp > 1, dp, d, s * tp + tt, S * tp,
                              (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp, s * tp + tt);
-                    if (used) {
+                    if (TR.phot)
+                        for (int k = 0; k < ports; k++) p_st[k * NTHR + threadIdx.x] = 0;
+                    if (used && !TR.phot) {
                         // route checks of every pair this rank's flows will use (R3)
                         auto chk = [&](uint32_t x, uint32_t y) {
                             const int l = route_len(a, TR, x, y);
@@ -577,6 +623,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
 
         // ------------------------------ one instant ------------------------------
         bool dirty = false;
+        if (TR.phot && used)   // R20: logical links whose setup completes now are up (last use = now)
+            for (int k = 0; k < ports; k++)
+                if (p_st[k * NTHR + threadIdx.x] == 1 && p_t[k * NTHR + threadIdx.x] == t) p_st[k * NTHR + threadIdx.x] = 2;
         for (;;) {
             for (;;) {
                 bool more = false;
@@ -674,8 +723,133 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 if (!vany(more)) break;
             }
 
+            bool again = false;
+            // (f') R20 photonic network: (i) a logical link per request, (ii) link heads ask for a
+            // receive buffer, (iii) destinations grant buffers in (release time, code) order
+            const bool phw = TR.phot && used && (FT.st >= PS_REQ || FD.st >= PS_REQ || FP.st >= PS_REQ);
+            if (vany(phw)) {
+                const int me = (int)threadIdx.x;
+                auto onlink = [&](int k) -> bool {   // a transfer of this lane is queued on / using link k
+                    auto u = [&](const Flow &F) { return (F.st >= PS_LINKQ || F.st == FS_ACT) && (int)F.hl[1] == k; };
+                    return u(FT) || u(FD) || u(FP);
+                };
+                auto klt = [](double ta, uint64_t ca, double tb, uint64_t cb) { return ta < tb || (ta == tb && ca < cb); };
+                if (phw) {
+                    // (i) requests in key order: existing link, free port, else tear down the link idle longest
+                    for (int r = 0; r < 3; r++) {
+                        Flow *best = nullptr;
+                        auto pick = [&](Flow &F) {
+                            if (F.st == PS_REQ && F.len == 0 && (!best || klt(F.t_upd, F.code, best->t_upd, best->code))) best = &F;
+                        };
+                        pick(FT); pick(FD); pick(FP);
+                        if (!best) break;
+                        Flow &F = *best;
+                        F.len = 1;   // visited in this pass
+                        const int dg = (int)F.hl[0];
+                        int k = -1;
+                        for (int q = 0; q < ports; q++)
+                            if (p_st[q * NTHR + me] != 0 && p_dst[q * NTHR + me] == dg) k = q;
+                        if (k < 0) {
+                            int nk = -1;
+                            for (int q = 0; q < ports && nk < 0; q++) if (p_st[q * NTHR + me] == 0) nk = q;
+                            if (nk < 0)
+                                for (int q = 0; q < ports; q++) {
+                                    if (p_st[q * NTHR + me] != 2 || onlink(q)) continue;
+                                    if (nk < 0 || p_t[q * NTHR + me] < p_t[nk * NTHR + me] ||
+                                        (p_t[q * NTHR + me] == p_t[nk * NTHR + me] && p_dst[q * NTHR + me] < p_dst[nk * NTHR + me]))
+                                        nk = q;
+                                }
+                            if (nk >= 0) {
+                                const double tr = t + ph_set;
+                                p_dst[nk * NTHR + me] = dg;
+                                p_st[nk * NTHR + me] = tr == t ? 2 : 1;
+                                p_t[nk * NTHR + me] = tr;
+                                k = nk;
+                                alg += 1;
+                            }
+                        }
+                        if (k >= 0) { F.st = PS_LINKQ; F.hl[1] = (uint32_t)k; }
+                    }
+                    FT.len = FT.st == PS_REQ ? 0 : FT.len;
+                    FD.len = FD.st == PS_REQ ? 0 : FD.len;
+                    FP.len = FP.st == PS_REQ ? 0 : FP.len;
+                    // (ii) an up link with nothing waiting for a buffer or moving passes its queue head on
+                    for (int r = 0; r < 3; r++) {
+                        Flow *head = nullptr;
+                        auto hd = [&](Flow &F) {
+                            if (F.st != PS_LINKQ) return;
+                            const int k = (int)F.hl[1];
+                            if (p_st[k * NTHR + me] != 2) return;
+                            auto busy = [&](const Flow &G) { return (G.st == PS_BUFW || G.st == FS_ACT) && (int)G.hl[1] == k; };
+                            if (busy(FT) || busy(FD) || busy(FP)) return;
+                            if (!head || klt(F.t_upd, F.code, head->t_upd, head->code)) head = &F;
+                        };
+                        hd(FT); hd(FD); hd(FP);
+                        if (!head) break;
+                        head->st = PS_BUFW;
+                    }
+                }
+                // (iii) publish buffer requests and transfers, each destination grants in key order
+                auto pub = [&](const Flow &F, int k) {
+                    const int e = me * 3 + k;
+                    const bool w = TR.phot && used && (F.st == PS_BUFW || (F.st == FS_ACT && F.len == 0));
+                    q_dst[e] = w ? (int)F.hl[0] : -1;
+                    q_st[e] = F.st == PS_BUFW ? 1 : 2;
+                    q_t[e] = F.t_upd;
+                    q_code[e] = F.code;
+                };
+                pub(FT, 0);
+                pub(FD, 1);
+                pub(FP, 2);
+                ssync();
+                if (TR.phot && used) {
+                    const int e0 = NW == 1 ? (wid * 32 + sbase) * 3 : 0, e1 = e0 + 3 * SL;
+                    const int g = (int)gpu;
+                    int occ = 0, nc = 0;
+                    for (int e = e0; e < e1; e++)
+                        if (q_dst[e] == g) { if (q_st[e] == 2) occ++; else nc++; }
+                    if (nc > 0) {
+                        const int fr = bufs > 0 ? bufs - occ : nc;
+                        if (fr >= nc) {
+                            for (int e = e0; e < e1; e++) if (q_dst[e] == g && q_st[e] == 1) q_g[e] = 1;
+                        } else {
+                            for (int r = 0; r < fr; r++) {
+                                int be = -1;
+                                for (int e = e0; e < e1; e++)
+                                    if (q_dst[e] == g && q_st[e] == 1 && !q_g[e] &&
+                                        (be < 0 || klt(q_t[e], q_code[e], q_t[be], q_code[be])))
+                                        be = e;
+                                q_g[be] = 1;
+                            }
+                        }
+                    }
+                }
+                ssync();
+                auto take = [&](Flow &F, int k) {
+                    const int e = me * 3 + k;
+                    if (q_g[e]) {
+                        q_g[e] = 0;
+                        F.st = FS_ACT;
+                        F.len = 0;
+                        F.t_drain = (t + ph_lat) + F.bytes / ph_bw;
+                        alg += 3;
+                        EV(EV_ACTIVATE, F.code);
+                        if (F.t_drain == t) again = true;
+                    }
+                };
+                take(FT, 0);
+                take(FD, 1);
+                take(FP, 2);
+                const uint32_t nx = scount(TR.phot && used && FT.st == FS_ACT) + scount(TR.phot && used && FD.st == FS_ACT) +
+                                    scount(TR.phot && used && FP.st == FS_ACT);
+                if (TR.phot && have && nx > maxact) maxact = nx;
+            }
+
             // (f) R14 over every in-transit flow of the segment (up to three per lane)
-            if (!vany(dirty)) break;
+            if (!vany(dirty)) {
+                if (!vany(again)) break;
+                continue;
+            }
             const bool segdirty = sany(dirty);
             dirty = false;
             const bool aT = segdirty && used && FT.st == FS_ACT;
@@ -815,7 +989,6 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 nrounds += rounds;
                 if (nact > maxact) maxact = nact;
             }
-            bool again = false;
             auto drain = [&](Flow &F, bool on) {
                 if (on) {
                     F.t_drain = (F.rem == 0.0) ? t : t + F.rem / F.rate;
@@ -853,6 +1026,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             cf(FT);
             cf(FD);
             cf(FP);
+            if (TR.phot)
+                for (int k = 0; k < ports; k++)
+                    if (p_st[k * NTHR + threadIdx.x] == 1 && p_t[k * NTHR + threadIdx.x] < cand) cand = p_t[k * NTHR + threadIdx.x];
         }
         const double tn = smin(cand);
         const bool stuck = have && !fin && !(tn < dinf());
@@ -896,12 +1072,16 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
 #undef EV
 }
 
-size_t k3h_dyn_smem(int W, uint32_t lmax) { return W <= 32 ? 0 : (size_t)lmax * 16; }
+size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
+    const size_t nthr = W <= 32 ? K3_THREADS : (size_t)W;
+    const size_t ph = pmax ? nthr * pmax * 16 + nthr * 3 * (8 + 8 + 4 + 1 + 1) : 0;
+    return (W <= 32 ? 0 : (size_t)lmax * 16) + ph;
+}
 
 template <int W, int NW>
 static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
-    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, a.lmax);
-    if (NW > 1) {
+    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, a.lmax, a.pmax);
+    if (dyn > 0) {
         const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
         if (e != cudaSuccess) return e;
     }
@@ -927,28 +1107,28 @@ cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
 }
 
 template <int W, int NW>
-static int occ_h(uint32_t lmax) {
-    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, lmax);
-    if (NW > 1 && cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
+static int occ_h(uint32_t lmax, uint32_t pmax) {
+    const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, lmax, pmax);
+    if (dyn > 0 && cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
         return 0;
     int nb = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
     return nb;
 }
 
-int k3h_max_blocks_per_sm(int W, uint32_t lmax) {
+int k3h_max_blocks_per_sm(int W, uint32_t lmax, uint32_t pmax) {
     int nb;
     switch (W) {
-    case 2: nb = occ_h<2, 1>(lmax); break;
-    case 4: nb = occ_h<4, 1>(lmax); break;
-    case 8: nb = occ_h<8, 1>(lmax); break;
-    case 16: nb = occ_h<16, 1>(lmax); break;
-    case 32: nb = occ_h<32, 1>(lmax); break;
-    case 64: nb = occ_h<32, 2>(lmax); break;
-    case 128: nb = occ_h<32, 4>(lmax); break;
-    case 256: nb = occ_h<32, 8>(lmax); break;
-    case 512: nb = occ_h<32, 16>(lmax); break;
-    default: nb = occ_h<32, 32>(lmax); break;
+    case 2: nb = occ_h<2, 1>(lmax, pmax); break;
+    case 4: nb = occ_h<4, 1>(lmax, pmax); break;
+    case 8: nb = occ_h<8, 1>(lmax, pmax); break;
+    case 16: nb = occ_h<16, 1>(lmax, pmax); break;
+    case 32: nb = occ_h<32, 1>(lmax, pmax); break;
+    case 64: nb = occ_h<32, 2>(lmax, pmax); break;
+    case 128: nb = occ_h<32, 4>(lmax, pmax); break;
+    case 256: nb = occ_h<32, 8>(lmax, pmax); break;
+    case 512: nb = occ_h<32, 16>(lmax, pmax); break;
+    default: nb = occ_h<32, 32>(lmax, pmax); break;
     }
     return nb > 0 ? nb : 1;
 }

@@ -586,11 +586,16 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     ce.kind = CK_AR;
                     ce.pad = 0;
                     colls[hs.dcol_off + b++] = ce;
-                    // trigger: (producer of the bucket's last gradient, micro-batch 0)
-                    const int P = (int)(T.info[last_prod] & INFO_PHASE_MASK);
-                    const uint32_t cntP = P == 0 ? si.nF : P == 1 ? si.nB : si.nO;
-                    for (uint32_t q = 0; q < cntP; q++)
-                        if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig++; break; }
+                    // trigger: (producer of the bucket's last gradient, micro-batch 0); the HYBRID form
+                    // of DataParallel (R6) triggers every bucket after the stage's last non-OPT op
+                    if (C.dp_after_bwd && (si.nB > 0 || si.nF > 0)) {
+                        ents[si.nB > 0 ? eoff[1] + si.nB - 1 : eoff[0] + si.nF - 1].dp_nsig++;
+                    } else {
+                        const int P = (int)(T.info[last_prod] & INFO_PHASE_MASK);
+                        const uint32_t cntP = P == 0 ? si.nF : P == 1 ? si.nB : si.nO;
+                        for (uint32_t q = 0; q < cntP; q++)
+                            if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig++; break; }
+                    }
                     sum = 0;
                     Sb = 0.0;
                     open = false;

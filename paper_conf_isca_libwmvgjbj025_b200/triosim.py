@@ -36,8 +36,11 @@ class _TraceDesc(C.Structure):
 
 
 class _Topology(C.Structure):
-    _fields_ = [("n_nodes", C.c_uint32), ("n_gpus", C.c_uint32), ("n_links", C.c_uint32), ("pad", C.c_uint32),
-                ("links", C.c_void_p), ("ring_order", C.c_void_p)]
+    _fields_ = [("n_nodes", C.c_uint32), ("n_gpus", C.c_uint32), ("n_links", C.c_uint32), ("net_model", C.c_uint32),
+                ("links", C.c_void_p), ("ring_order", C.c_void_p), ("photonic", C.c_void_p)]
+
+
+NET_FLOW, NET_PHOTONIC = 0, 1
 
 
 class _Plans(C.Structure):
@@ -124,8 +127,11 @@ class Context:
         for i, tp in enumerate(topos):
             links = np.ascontiguousarray(tp.links, W.LINK_DTYPE)
             ro = None if tp.ring_order is None else np.ascontiguousarray(tp.ring_order, np.uint32)
-            keep += [links, ro]
-            tarr[i] = _Topology(tp.n_nodes, tp.n_gpus, len(links), 0, _ptr(links), _ptr(ro))
+            ph = getattr(tp, "photonic", None)
+            ph = None if ph is None else np.ascontiguousarray(np.asarray(ph, W.PHOTONIC_DTYPE).reshape(1))
+            keep += [links, ro, ph]
+            tarr[i] = _Topology(tp.n_nodes, tp.n_gpus, len(links), NET_FLOW if ph is None else NET_PHOTONIC,
+                                _ptr(links), _ptr(ro), _ptr(ph))
         pl = None
         if plans:
             off = np.zeros(len(plans) + 1, np.uint32)

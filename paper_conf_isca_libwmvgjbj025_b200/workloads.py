@@ -805,6 +805,30 @@ def sweep_c5(trace=None, seed=5, Ns=(64, 128, 256, 512, 1024), n_bw=25, n_lat=14
     return Sweep("c5_gpt3_hybrid", tr, topos, arr[perm])
 
 
+def sweep_wafer(trace=None, seed=6, n_bw=10, n_lat=5) -> Sweep:
+    """NEXT 1: the Passage case study (Fig. 15).  84 GPUs on a 12 x 7 wafer,
+    DDP over all of them, ring AllReduce along a Hamiltonian cycle of the electrical mesh vs the
+    same ring over photonic logical links (8 ports, 484 GB/s across 8 links, 20 ms link setup).  Axes:
+    network x per-GPU batch {16, 32, 64, 128} x bucket {per tensor, 25 MiB} x bandwidth x latency scales."""
+    tr = trace if trace is not None else resnet50_trace()
+    elec = wafer_mesh(12, 7, bw=50e9, lat=1e-6)
+    opt = photonic(84, ports=8, link_bw=484e9 / 8, setup=20e-3, lat=1e-6, ring_order=elec.ring_order,
+                   name="passage84")
+    topos = [elec, opt]
+    bws = np.logspace(np.log10(0.5), np.log10(2.0), n_bw)
+    lats = np.logspace(np.log10(0.5), np.log10(2.0), n_lat)
+    pts = []
+    for ti in range(2):
+        for b in (16, 32, 64, 128):
+            for bucket in (0, 25 * MiB):
+                for bw in bws:
+                    for lat in lats:
+                        pts.append(make_point(ti, ST_DDP, dp=84, B=84 * b, bucket=bucket, bw=float(bw), lat=float(lat)))
+    arr = points_array(pts)
+    perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
+    return Sweep("wafer84_passage_dp", tr, topos, arr[perm])
+
+
 def sweep_c5_small(trace=None, seed=5) -> Sweep:
     """configs[4]'s structure on 8-32 simulated GPUs (warp-segment hybrid kernel; m in {8,16,32},
     4 bandwidths x 2 latencies): the small end used by the sampled parity tests."""

@@ -160,11 +160,14 @@ def test_statuses_and_edge_cases(ctx):
     got = ctx.run_sweep(sw)
     check(got, sw, list(range(len(pts))))
     assert list(got["status"][:11]) == [1, 2, 1, 0, 6, 6, 7, 7, 0, 7, 3]
-    # beyond the kernels' limits -- DataParallel (after-backward) with more than 32 GPUs, a route longer
-    # than 8 hops (tree edges across a 32-GPU ring) -- is reported, never silently wrong
+    # DataParallel (after-backward) with more than 32 GPUs runs in its HYBRID form; beyond the kernels'
+    # limits -- a route longer than 8 hops (tree edges across a 32-GPU ring) -- is reported, never
+    # silently wrong
     big = W.Sweep("big", tr, topos, W.points_array([P(2, W.ST_DP, dp=40, B=40 * 64),
                                                     P(1, W.ST_DDP, dp=32, B=32 * 64, algo=W.ALG_TREE)]))
-    assert list(ctx.run_sweep(big)["status"]) == [W.PT_TOO_LARGE, W.PT_TOO_LARGE]
+    gb = ctx.run_sweep(big)
+    assert list(gb["status"]) == [W.PT_OK, W.PT_TOO_LARGE]
+    check(gb, big, [0])
     # empty sweep
     empty = W.Sweep("empty", tr, topos, np.zeros(0, W.POINT_DTYPE))
     assert len(ctx.run_sweep(empty)) == 0
@@ -275,3 +278,69 @@ def test_c5_full_scale_sampled(ctx):
     got = ctx.run_sweep(sw)
     assert (got["status"] == 0).all(), np.unique(got["status"], return_counts=True)
     check(got, sw, list(range(len(sw.points))))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_random_photonic(ctx, seed):
+    """Photonic circuit-switched network (R20) on random traces: every strategy (all run in
+    the hybrid kernel, whose lanes own their logical links), 1-4 ports (LRU teardown), 0-2 receive
+    buffers, with and without setup latency; mixed in one sweep with flow-network points so warp
+    segments of both models share a warp.  Compared point by point with the oracle."""
+    rng = np.random.Generator(np.random.PCG64(1700 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=2)
+    topos = []
+    for g in (2, 3, 4, 8, 12, 16, 40):
+        topos.append(W.photonic(g, ports=int(rng.integers(1, 5)), link_bw=float(rng.uniform(5e9, 80e9)),
+                                setup=float(rng.choice([0.0, 1e-5, 2e-4])), lat=float(rng.choice([0.0, 1e-6])),
+                                buf_slots=int(rng.integers(0, 3)),
+                                ring_order=rng.permutation(g).astype(np.uint32)))
+    topos += [W.ring(8, 40e9, 1e-6), W.mesh(2, 4, 60e9, 1e-6)]
+    pts = []
+    P = W.make_point
+    for _ in range(300):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        st = int(rng.integers(0, 5))
+        bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
+        algo = int(rng.integers(0, 2))
+        if st in (W.ST_DP, W.ST_DDP):
+            dp = int(rng.integers(1, G + 1))
+            pts.append(P(ti, st, dp=dp, B=dp * int(rng.integers(1, 5)), algo=algo, bw=bw, lat=lat,
+                         bucket=int(rng.choice([0, 1 << 12, 1 << 30]))))
+        elif st == W.ST_TP:
+            pts.append(P(ti, st, tp=int(rng.integers(1, G + 1)), B=int(rng.integers(1, 5)), algo=algo, bw=bw,
+                         lat=lat, tp_mode=int(rng.integers(0, 2))))
+        elif st == W.ST_PP:
+            m = int(rng.integers(1, 5))
+            pts.append(P(ti, st, pp=int(rng.integers(1, min(G, tr.n_layers) + 1)), m=m, B=m * int(rng.integers(1, 3)),
+                         bw=bw, lat=lat))
+        else:
+            while True:
+                dp, tpd, pp = int(rng.integers(1, 4)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 4))
+                if dp * tpd * pp <= G and pp <= tr.n_layers:
+                    break
+            m = int(rng.integers(1, 3))
+            pts.append(P(ti, W.ST_HYBRID, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m, algo=algo, bw=bw, lat=lat,
+                         tp_mode=int(rng.integers(0, 2)), bucket=int(rng.choice([0, 1 << 30]))))
+    sw = W.Sweep("phot", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    check(got, sw, list(range(len(pts))), allow_too_large=True)
+    phot = np.array([sw.topos[int(p["topo"])].photonic is not None for p in sw.points])
+    # the one kernel limit: tree collectives over photonic links (the broadcast flow's sender is another lane)
+    tl = got["status"] == W.PT_TOO_LARGE
+    assert (phot[tl] & (sw.points["coll_algo"][tl] == W.ALG_TREE) & (sw.points["strategy"][tl] != W.ST_PP)).all()
+    assert ((got["status"] == 0) & phot).sum() > 120
+
+
+def test_wafer_passage_case_study(ctx):
+    """NEXT 1 at full size: the 84-GPU wafer sweep (electrical mesh ring vs Passage photonic links, DDP
+    ResNet-50), the bench workload of `bench.py --config wafer`; every point simulates, a seeded sample
+    of both networks against the oracle, and the photonic ring pays one 20 ms link setup."""
+    sw = W.sweep_wafer()
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all()
+    phot = sw.points["topo"] == 1
+    assert (got["n_wf_calls"][phot] == 0).all() and (got["n_wf_calls"][~phot] > 0).all()
+    assert (got["comm_busy_s"][phot] >= 20e-3 * sw.points["lat_scale"][phot]).all()
+    idx = sample(len(sw.points), 24, 66)
+    check(got, sw, idx)
