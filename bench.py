@@ -31,15 +31,19 @@ from paper_conf_isca_libwmvgjbj025_b200 import workloads as W  # noqa: E402
 
 METRIC = "simulated design points/sec"
 UNIT = "points/s"
-CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1, "c5": W.sweep_c5}
+CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1, "c5": W.sweep_c5,
+           "wafer": W.sweep_wafer}
+DEFAULT_POINTS = {"c5": 296}   # configs[4]'s 966k-point sweep: a seeded prefix (two waves of 1024-thread CTAs)
 WORKLOAD = {"c2": "configs[1]: ResNet-50 DP/DDP, 2-16 simulated GPUs on an NVLink-style ring, 10k-point "
                   "bandwidth x latency x batch x bucket sweep",
             "c3": "configs[2]: BERT-large Megatron/paper TP 2/4/8, ring/star/mesh/cube-mesh/ring-graph/"
                   "double-ring topologies incl. asymmetric",
             "c4": "configs[3]: GPT-2 XL GPipe 4-16 stages x 8-64 micro-batches on 2D meshes",
             "c1": "configs[0]: 4-layer MLP DDP on 2 GPUs, one uniform link",
-            "c5": "configs[4] (<= 32 simulated GPUs): GPT-3-class DP x TP x PP, hierarchical 2:1 / 4:1 "
-                  "topology incl. a seeded slow-link subset"}
+            "c5": "configs[4]: GPT-3-class DP x TP x PP on 64-1024 simulated GPUs, hierarchical 1:1 / 2:1 / 4:1 "
+                  "topology incl. a seeded slow-link subset (966k-point sweep, seeded prefix)",
+            "wafer": "NEXT 1: 84-GPU 12x7 wafer, DDP ResNet-50, ring over the electrical mesh vs Passage photonic "
+                     "logical links (P:330-342)"}
 FP64_LANES_PER_SM = 64     # B200 FP64 pipe: 64 DFMA/DADD/DMUL lanes per SM per clock
 N_SMS = 148
 
@@ -207,6 +211,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--points", type=int, default=0,
+                    help="simulate a seeded prefix of this many points of the sweep (0 = config default)")
     ap.add_argument("--shard", action="store_true",
                     help="strong scaling: deal one sweep to the ranks by cost instead of a full sweep per rank")
     args = ap.parse_args()
@@ -226,6 +232,9 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     sw = CONFIGS[args.config]()
+    npts = args.points or DEFAULT_POINTS.get(args.config, 0)
+    if npts and npts < len(sw.points):
+        sw = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[:npts], sw.plans)
     n_sweep = len(sw.points)
     if args.shard and world > 1:
         tr = sw.trace
@@ -333,6 +342,7 @@ def main():
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "scaling": "strong" if (args.shard and world > 1) else "weak",
             "config": {"workload": WORKLOAD[args.config], "points": n, "points_ok": n_ok,
+                       "sweep_points": len(CONFIGS[args.config]().points) if npts else n_sweep,
                        "trace": sw.trace.name, "ops": int(len(sw.trace.ops)),
                        "parallelism": (f"one sweep dealt to {world} ranks by cost; records all-gathered over NCCL"
                                        if (args.shard and world > 1) else
