@@ -43,7 +43,8 @@ def lib():
             L = C.CDLL(LIB)
             P = C.c_void_p
             u32, i32, i64, f64 = C.c_uint32, C.c_int32, C.c_int64, C.c_double
-            L.oracle_run_point.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P, P, P]
+            L.oracle_run_point.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P, P, P,
+                                           P, P]
             L.oracle_run_point.restype = C.c_int
             L.oracle_export_graph.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P,
                                               P, P, P, P, P, P, P, P, P, P, P, P, P]
@@ -89,26 +90,36 @@ class OracleError(RuntimeError):
     pass
 
 
-def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None):
-    """Simulate one design point; returns a RESULT_DTYPE record."""
+def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None, breakdown=False):
+    """Simulate one design point; returns a RESULT_DTYPE record (and, with breakdown=True, the
+    per-layer compute and communication times of DESIGN.md R22)."""
     k1, ta = _trace_args(tr)
     k2, tpa = _topo_args(topo)
     pl = None if plan is None else np.ascontiguousarray(plan, np.uint32)
     ptv = np.array(pt, W.POINT_DTYPE).reshape(1)
     out = np.zeros(1, W.RESULT_DTYPE)
     ph = _phot(topo)
+    lc = lm = None
+    if breakdown:
+        lc, lm = np.zeros(max(tr.n_layers, 1)), np.zeros(max(tr.n_layers, 1))
     rc = lib().oracle_run_point(*ta, *tpa, _p(pl), 0 if pl is None else len(pl), 0 if pl is None else 1, _p(ptv),
-                                _p(out), _p(ph))
+                                _p(out), _p(ph), _p(lc), _p(lm))
     if rc != 0:
         raise OracleError(f"oracle_run_point rc={rc}")
+    if breakdown:
+        return out[0], lc[:tr.n_layers], lm[:tr.n_layers]
     return out[0]
 
 
-def run_sweep(sw: W.Sweep, idx=None):
+def run_sweep(sw: W.Sweep, idx=None, breakdown=False):
     """Oracle results for points idx of a sweep; topology index and plan index are resolved
-    here in DESIGN.md R3 order (topology first, the plan inside the point checks)."""
+    here in DESIGN.md R3 order (topology first, the plan inside the point checks).  With
+    breakdown=True also returns per-layer compute / comm arrays [len(idx), n_layers] (R22)."""
     idx = range(len(sw.points)) if idx is None else idx
     res = np.zeros(len(idx), W.RESULT_DTYPE)
+    if breakdown:
+        L = sw.trace.n_layers
+        bc, bm = np.zeros((len(idx), L)), np.zeros((len(idx), L))
     for q, i in enumerate(idx):
         pt = sw.points[i]
         if pt["topo"] >= len(sw.topos):
@@ -117,7 +128,12 @@ def run_sweep(sw: W.Sweep, idx=None):
         plan = None
         if pt["stage_plan"] >= 0:
             plan = sw.plans[pt["stage_plan"]] if pt["stage_plan"] < len(sw.plans) else []
-        res[q] = run_point(sw.trace, sw.topos[pt["topo"]], pt, plan)
+        if breakdown:
+            res[q], bc[q], bm[q] = run_point(sw.trace, sw.topos[pt["topo"]], pt, plan, breakdown=True)
+        else:
+            res[q] = run_point(sw.trace, sw.topos[pt["topo"]], pt, plan)
+    if breakdown:
+        return res, bc, bm
     return res
 
 

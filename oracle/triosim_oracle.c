@@ -238,6 +238,7 @@ typedef struct {
     double bytes;     /* flow size */
     uint64_t code;    /* canonical id for the order hash */
     int flags;
+    int layer;        /* task: its operator's layer (R22 breakdown); -1 otherwise */
 } GNode;
 
 typedef struct {
@@ -245,6 +246,12 @@ typedef struct {
     IVec dep_from, dep_to;   /* edge list: node dep_from[i] waits for node dep_to[i] */
     int n_coll;
     double coll_payload;     /* left fold of collective payloads in creation order */
+    /* R22 per-layer breakdown: the representative rank of each layer, and the communications it
+     * takes part in, attributed to the layer of the operator that triggers / produces them */
+    int want_bd, n_layers;
+    int *rep;                /* per layer: GPU of the representative rank */
+    int cur_layer, cur_cat;  /* attribution of the next collective: layer, 0 = TP / 1 = DP group */
+    IVec rc_s, rc_e, rc_l, rc_c;   /* records: start node, end node, layer, category (2 = P2P) */
 } Graph;
 
 static int g_add(Graph *G, GNode nd) {
@@ -264,21 +271,26 @@ static int g_dep(Graph *G, int node, int on) {
 static void g_free(Graph *G) {
     free(G->n); G->n = NULL; G->count = G->cap = 0;
     iv_free(&G->dep_from); iv_free(&G->dep_to);
+    free(G->rep); G->rep = NULL;
+    iv_free(&G->rc_s); iv_free(&G->rc_e); iv_free(&G->rc_l); iv_free(&G->rc_c);
 }
-static int add_task(Graph *G, int gpu, long prog, double dur) {
+static void g_record(Graph *G, int start, int end, int layer, int cat) {
+    iv_push(&G->rc_s, start); iv_push(&G->rc_e, end); iv_push(&G->rc_l, layer); iv_push(&G->rc_c, cat);
+}
+static int add_task(Graph *G, int gpu, long prog, double dur, int layer) {
     GNode n; memset(&n, 0, sizeof n);
-    n.type = N_TASK; n.gpu = gpu; n.dur = dur;
+    n.type = N_TASK; n.gpu = gpu; n.dur = dur; n.layer = layer;
     n.code = ((uint64_t)(uint32_t)gpu << 40) | (uint64_t)prog;
     return g_add(G, n);
 }
 static int add_barrier(Graph *G, int flags, uint64_t code) {
     GNode n; memset(&n, 0, sizeof n);
-    n.type = N_BARRIER; n.flags = flags; n.code = code;
+    n.type = N_BARRIER; n.flags = flags; n.code = code; n.layer = -1;
     return g_add(G, n);
 }
 static int add_flow(Graph *G, int src, int dst, double bytes, uint64_t code, int flags) {
     GNode n; memset(&n, 0, sizeof n);
-    n.type = N_FLOW; n.src = src; n.dst = dst; n.bytes = bytes; n.code = code; n.flags = flags;
+    n.type = N_FLOW; n.src = src; n.dst = dst; n.bytes = bytes; n.code = code; n.flags = flags; n.layer = -1;
     return g_add(G, n);
 }
 static uint64_t coll_flow_code(uint64_t c, int step, int member) {
@@ -369,6 +381,10 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
         if (!any) g_dep(G, done[i], sb);
     }
     iv_free(&fl);
+    /* R22: the layer's representative rank times this collective from its start to "done" on it */
+    if (G->want_bd && G->cur_layer >= 0)
+        for (int i = 0; i < p; i++)
+            if (members[i] == G->rep[G->cur_layer]) { g_record(G, sb, done[i], G->cur_layer, G->cur_cat); break; }
     return 0;
 }
 
@@ -565,7 +581,7 @@ static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
     /* every rank duplicates every operator */
     for (int r = 0; r < dp; r++)
         for (uint32_t o = 0; o < N; o++)
-            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, 1, pt->tp_mode));
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer);
     if (dp > 1) {
         /* weight gradients in production order (reading Q4: produced by the backward pass) */
         WEnt *w = (WEnt *)malloc(sizeof(WEnt) * (T->n_ts ? T->n_ts : 1));
@@ -599,6 +615,8 @@ static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
              * last gradient; DP (DataParallel): after the backward pass (reading Q6) */
             int trig_op = (pt->strategy == ST_DDP) ? w[j - 1].prod : last_nonopt;
             for (int r = 0; r < dp; r++) trig[r] = task[(size_t)r * N + trig_op];
+            G->cur_layer = (int)T->ops[trig_op].layer;
+            G->cur_cat = 1;
             if (build_collective(G, ro, dp, CK_AR, pt->coll_algo, S, trig, have_prev ? prev : NULL, done)) return -1;
             memcpy(prev, done, sizeof(int) * (size_t)dp);
             have_prev = 1;
@@ -624,7 +642,7 @@ static int expand_tp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
     if (!task) return -1;
     for (int r = 0; r < tp; r++)
         for (uint32_t o = 0; o < N; o++)
-            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, tp, pt->tp_mode));
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, tp, pt->tp_mode), (int)T->ops[o].layer);
     if (tp > 1) {
         int *done_of = (int *)malloc(sizeof(int) * (size_t)(T->n_ts ? T->n_ts : 1) * (size_t)tp);
         char *has = (char *)calloc(T->n_ts ? T->n_ts : 1, 1);
@@ -648,6 +666,8 @@ static int expand_tp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
                 double S = (double)T->ts[x].bytes_b0;
                 if (T->ts[x].batch_scaled) S = S * r_b;
                 for (int r = 0; r < tp; r++) trig[r] = task[(size_t)r * N + o];
+                G->cur_layer = (int)op->layer;
+                G->cur_cat = 0;
                 if (build_collective(G, ro, tp, kind, pt->coll_algo, S, trig, have_prev ? prev : NULL,
                                      done_of + (size_t)x * tp)) return -1;
                 memcpy(prev, done_of + (size_t)x * tp, sizeof(int) * (size_t)tp);
@@ -720,7 +740,7 @@ static int expand_pp(const Trace *T, const OPoint *pt, const int *ro, const uint
         int prev_send = -1;
         for (long q = 0; q < np; q++) {
             int o = prog_op[q], j = prog_mb[q];
-            int t = add_task(G, ro[s], q, op_time(T, (uint32_t)o, r_b, 1, pt->tp_mode));
+            int t = add_task(G, ro[s], q, op_time(T, (uint32_t)o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer);
             inst[(size_t)o * m + j] = t;
             /* "send its output data to the next GPU. Simultaneously ... the next micro-batch"
              * (P:190): push every produced tensor to each other stage that reads it, FIFO per
@@ -734,6 +754,7 @@ static int expand_pp(const Trace *T, const OPoint *pt, const int *ro, const uint
                     double b = tensor_bytes(T, x, r_b, 1, pt->tp_mode);
                     int f = add_flow(G, ro[s], ro[d], b, p2p_flow_code(x, j, ro[d]), NF_P2P);
                     g_dep(G, f, t);
+                    if (G->want_bd && ro[s] == G->rep[op->layer]) g_record(G, f, f, (int)op->layer, 2);
                     if (prev_send >= 0) g_dep(G, f, prev_send);
                     prev_send = f;
                     p2p[((size_t)xidx[x] * m + j) * S + d] = f;
@@ -857,7 +878,8 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
         task[r] = (int *)malloc(sizeof(int) * ((size_t)plen[s] + 1));
         if (!task[r]) goto out;
         for (long q = 0; q < plen[s]; q++)
-            task[r][q] = add_task(G, ro[r], q, op_time(T, (uint32_t)pop[s][q], r_b, tp, pt->tp_mode));
+            task[r][q] = add_task(G, ro[r], q, op_time(T, (uint32_t)pop[s][q], r_b, tp, pt->tp_mode),
+                                  (int)T->ops[pop[s][q]].layer);
     }
     /* TP collectives: per group (d, s), one per (op, output, micro-batch) instance in program order */
     if (tp > 1) {
@@ -877,6 +899,8 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                         double Sb = (double)T->ts[x].bytes_b0;      /* full tensor (Q8) */
                         if (T->ts[x].batch_scaled) Sb = Sb * r_b;
                         for (int t = 0; t < tp; t++) trig[t] = task[base + t][q];
+                        G->cur_layer = (int)op->layer;
+                        G->cur_cat = 0;
                         if (build_collective_code(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, Sb, trig,
                                                   have_prev ? prev : NULL, done)) goto out;
                         seq++;
@@ -921,6 +945,7 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                     const int f = add_flow(G, ro[r], dg, tensor_bytes(T, x, r_b, tp, pt->tp_mode),
                                            p2p_flow_code(x, j, dg), NF_P2P);
                     g_dep(G, f, task[r][q]);
+                    if (G->want_bd && ro[r] == G->rep[op->layer]) g_record(G, f, f, (int)op->layer, 2);
                     if (prev_send >= 0) g_dep(G, f, prev_send);
                     if (tp > 1) {
                         const int di = hm_get(&tpc, (gid << 40) | ((uint64_t)x << 16) | (uint64_t)j);
@@ -985,6 +1010,8 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                         if (pop[s][q] == w[j - 1].prod && pmb[s][q] == 0) { qt = q; break; }
                     if (qt < 0) { free(w); goto out; }
                     for (int d = 0; d < dp; d++) trig[d] = task[(d * S + s) * tp + t][qt];
+                    G->cur_layer = (int)T->ops[pop[s][qt]].layer;
+                    G->cur_cat = 1;
                     if (build_collective_code(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, Sb, trig,
                                               have_prev ? prev : NULL, done)) { free(w); goto out; }
                     seq++;
@@ -1083,8 +1110,16 @@ static uint64_t dbits(double d) { uint64_t u; memcpy(&u, &d, 8); return u; }
 /* ------------------------------------------------------------------ */
 enum { S_WAIT = 0, S_QUEUED = 1, S_RUN = 2, S_LATENT = 3, S_ACTIVE = 4, S_DONE = 5 };
 
-static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale, OResult *res, double *t_done) {
+static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale, OResult *res, double *t_done,
+                    double *l_comp, double *l_comm) {
     long NN = G->count;
+    const int bd = l_comp != NULL && G->want_bd;
+    double *td_own = NULL, *t_rel = NULL;
+    if (bd) {
+        t_rel = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        if (!t_done) t_done = td_own = (double *)calloc((size_t)(NN ? NN : 1), sizeof(double));
+        if (!t_rel || !t_done) { free(t_rel); free(td_own); return -1; }
+    }
     int n_nodes_topo = (int)tp->n_nodes;
     /* dependency CSR (forward) and dependents CSR (reverse) */
     long NE = G->dep_from.n;
@@ -1320,6 +1355,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                             if (G->n[k].flags & NF_COLL_START) EVENT(EV_COLL_START, G->n[k].code);
                         } else if (ph) {
                             /* R20: a send request; t_act holds its release time (the FIFO key) */
+                            if (t_rel) t_rel[k] = t;
                             EVENT(EV_RELEASE, G->n[k].code);
                             inflight++;
                             if (G->n[k].src == G->n[k].dst) {
@@ -1336,6 +1372,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         } else {
                             state[k] = S_LATENT;
                             t_act[k] = t + lat[k];
+                            if (t_rel) t_rel[k] = t;
                             EVENT(EV_RELEASE, G->n[k].code);
                             iv_push(&latent, k);
                             inflight++;
@@ -1495,6 +1532,24 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
             res->n_wf_rounds = n_rounds;
             res->order_hash = H;
             res->max_active_flows = max_act;
+            if (bd) {
+                /* R22: compute = left fold of t' over the representative rank's op instances of the layer
+                 * in program order; comm = (TP-group + DP-group collective time) + P2P time, each a left
+                 * fold in creation order of (done on the rank - start) / (delivery - release) */
+                int L = G->n_layers;
+                double *acc3 = (double *)calloc((size_t)(3 * (L ? L : 1)), sizeof(double));
+                for (int l = 0; l < L; l++) l_comp[l] = 0.0;
+                for (long i = 0; i < NN; i++)
+                    if (G->n[i].type == N_TASK && G->n[i].gpu == G->rep[G->n[i].layer])
+                        l_comp[G->n[i].layer] = l_comp[G->n[i].layer] + G->n[i].dur;
+                for (long r = 0; r < G->rc_s.n; r++) {
+                    const int c = G->rc_c.v[r], l = G->rc_l.v[r], a0 = G->rc_s.v[r], a1 = G->rc_e.v[r];
+                    const double d = t_done[a1] - (c == 2 ? t_rel[a0] : t_done[a0]);
+                    acc3[c * L + l] = acc3[c * L + l] + d;
+                }
+                for (int l = 0; l < L; l++) l_comm[l] = (acc3[l] + acc3[L + l]) + acc3[2 * L + l];
+                free(acc3);
+            }
         }
         res->status = status;
         free(w.bw); free(w.n_e); free(w.k_e); free(w.res); free(w.share);
@@ -1507,6 +1562,7 @@ out:
     free(doff); free(roff); free(dlist); free(rlist); free(pending);
     free(qoff); free(qlist); free(head); free(running);
     free(froff); free(frlen); iv_free(&rpool); free(pair_off); free(pair_len); free(tmp); free(lat);
+    free(t_rel); free(td_own);
     return 0;
 }
 
@@ -1521,22 +1577,26 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
     if (!ro) return -1;
     ring_order_of(ring_order, tp->n_gpus, ro);
     int rc = 0;
+    /* R22: the representative rank of layer l = the lowest rank running it: rank 0 (DP/DDP/TP), the
+     * stage's GPU (PP), rank (d=0, s(l), t=0) (HYBRID) */
+    G->n_layers = (int)T->n_layers;
+    G->rep = (int *)malloc(sizeof(int) * (T->n_layers ? T->n_layers : 1));
+    if (!G->rep) { free(ro); return -1; }
+    for (uint32_t l = 0; l < T->n_layers; l++) G->rep[l] = ro[0];
+    G->cur_layer = -1;
     switch (pt->strategy) {
     case ST_DP: case ST_DDP: rc = expand_dp(T, pt, ro, G); break;
     case ST_TP: rc = expand_tp(T, pt, ro, G); break;
-    case ST_PP: {
+    case ST_PP: case ST_HYBRID: {
         uint32_t *fl = (uint32_t *)malloc(sizeof(uint32_t) * pt->pp);
         if (have_plan) memcpy(fl, plan, sizeof(uint32_t) * pt->pp);
         else if (auto_partition(T, pt->pp, fl)) { free(fl); free(ro); return -1; }
-        rc = expand_pp(T, pt, ro, fl, G);
-        free(fl);
-        break;
-    }
-    case ST_HYBRID: {
-        uint32_t *fl = (uint32_t *)malloc(sizeof(uint32_t) * pt->pp);
-        if (have_plan) memcpy(fl, plan, sizeof(uint32_t) * pt->pp);
-        else if (auto_partition(T, pt->pp, fl)) { free(fl); free(ro); return -1; }
-        rc = expand_hybrid(T, pt, ro, fl, G);
+        for (uint32_t l = 0; l < T->n_layers; l++) {
+            uint32_t st = 0;
+            while (st + 1 < pt->pp && fl[st + 1] <= l) st++;
+            G->rep[l] = ro[pt->strategy == ST_PP ? st : st * pt->tp];
+        }
+        rc = pt->strategy == ST_PP ? expand_pp(T, pt, ro, fl, G) : expand_hybrid(T, pt, ro, fl, G);
         free(fl);
         break;
     }
@@ -1551,7 +1611,8 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
 int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
                      uint32_t n_io, uint32_t trace_batch, uint32_t n_nodes, uint32_t n_gpus, const OLink *links,
                      uint32_t n_links, const uint32_t *ring_order, const uint32_t *plan, uint32_t plan_len,
-                     int have_plan, const OPoint *pt, OResult *out, const OPhot *ph) {
+                     int have_plan, const OPoint *pt, OResult *out, const OPhot *ph, double *l_comp,
+                     double *l_comm) {
     Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
     Topo tp; memset(&tp, 0, sizeof tp);
     int rc = trace_check(&T);
@@ -1564,11 +1625,13 @@ int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t
     }
     if (rc != O_OK) { free(T.prod); topo_free(&tp); return rc; }
     Graph G; memset(&G, 0, sizeof G);
+    G.want_bd = l_comp != NULL && l_comm != NULL;
     int status = PT_OK;
     memset(out, 0, sizeof *out);
+    if (l_comp) for (uint32_t l = 0; l < T.n_layers; l++) l_comp[l] = l_comm[l] = 0.0;
     if (build_graph(&T, &tp, ring_order, plan, plan_len, have_plan, pt, &G, &status)) rc = O_ENOMEM;
     else if (status != PT_OK) out->status = status;
-    else if (simulate(&G, &tp, pt->bw_scale, pt->lat_scale, out, NULL)) rc = O_ENOMEM;
+    else if (simulate(&G, &tp, pt->bw_scale, pt->lat_scale, out, NULL, l_comp, l_comm)) rc = O_ENOMEM;
     g_free(&G); free(T.prod); topo_free(&tp);
     return rc;
 }
@@ -1637,7 +1700,7 @@ int oracle_sim_graph(int64_t n, const int32_t *type, const int32_t *gpu, const d
     }
     G.n_coll = n_coll;
     G.coll_payload = coll_payload;
-    if (rc == O_OK && simulate(&G, &tp, bw_scale, lat_scale, out, t_done)) rc = O_ENOMEM;
+    if (rc == O_OK && simulate(&G, &tp, bw_scale, lat_scale, out, t_done, NULL, NULL)) rc = O_ENOMEM;
     g_free(&G); topo_free(&tp);
     return rc;
 }
