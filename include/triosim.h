@@ -226,6 +226,33 @@ triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t firs
 /* Free a trace or sweep handle (a trace must outlive its sweeps). */
 triosim_status triosim_release(triosim_ctx *ctx, int32_t handle);
 
+/* Per-layer breakdown ("the communication time and computation time of each layer or stage";
+ * Fig. 13; R22).  enable != 0 allocates, for the sweep, per-class layer tables and
+ * 3 x n_layers f64 accumulators per point (24 B x n_layers x n_pts of device memory; ENOMEM if that
+ * fails) and makes every later triosim_simulate_batch on the sweep also record the breakdown (a
+ * separate instantiation of the timeline kernels; the plain path is unchanged).  enable == 0 frees
+ * them.  Synchronises the device.  Errors: ENOTFOUND, ENOMEM, ECUDA. */
+triosim_status triosim_set_breakdown(triosim_ctx *ctx, int32_t sweep_id, int enable);
+
+/* Per-layer times of points [first, first+count) as two row-major [count][n_layers] f64 arrays
+ * (layer ids as in the trace, R1), of the layer's representative rank -- the lowest rank that runs
+ * it: rank 0 for DP / DDP / TP, the stage's GPU for PP, rank (d = 0, its stage, t = 0) for HYBRID:
+ *   layer_compute_s[l] = left fold, in that rank's program order, of t' over its operator instances
+ *                        of layer l (R4);
+ *   layer_comm_s[l]    = (TP-group + DP-group collective time) + P2P time, where a collective counts
+ *                        (done on the rank - start) and is attributed to the layer of the operator
+ *                        that triggers it (R6, R7, R9), and a P2P send of the rank counts
+ *                        (delivery - release) attributed to the producing operator's layer (R11);
+ *                        each term a left fold in creation order.
+ * Points whose status is not OK get zeros.  Values are those of the most recent simulate_batch that
+ * covered the point after the breakdown was enabled.  Either output may be NULL.  out_is_device == 0:
+ * host memory, the call runs the finalising kernel on `cuda_stream` and synchronises it;
+ * out_is_device != 0: device pointers on the context's GPU, stream-ordered and asynchronous.
+ * Errors: EINVAL (breakdown not enabled), ENOTFOUND, ERANGE, ENOMEM, ECUDA. */
+triosim_status triosim_breakdown(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
+                                 double *layer_compute_s, double *layer_comm_s, int out_is_device,
+                                 void *cuda_stream);
+
 /* Kernel launch counters since the context was created (K1, K2, K3 launches), for the bench. */
 triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3);
 

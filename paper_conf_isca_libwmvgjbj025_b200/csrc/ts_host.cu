@@ -104,6 +104,10 @@ struct Sweep {
     DevBuf<unsigned int> d_counter;
     DevBuf<unsigned long long> d_alg;
     cudaStream_t last_stream = nullptr;
+    // R22 per-layer breakdown (triosim_set_breakdown): per-class layer compute, per-point [3][L]
+    // communication accumulators, staging for host-bound copies
+    bool bd = false;
+    DevBuf<double> d_lcomp, d_bd_acc, d_bd_stage;
 };
 
 int w_index(int W) { int i = 0; while ((2 << i) < W) i++; return i; }
@@ -764,6 +768,12 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     CK(launch_k2_hybrid(S.d_cls.p, S.d_hyb_list.p, (uint32_t)S.hyb_list.size(), T.dev, S.d_plans.p, S.d_stages.p,
                         S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, st));
     if (!S.hyb_list.empty()) ctx->n_k2++;
+    const uint32_t L = T.n_layers;
+    if (S.bd) {
+        CK(launch_k4_layer_compute(S.d_cls.p, ncls, T.dev, S.d_dur.p, S.d_stages.p, S.d_ents.p, S.d_hents.p,
+                                   S.d_lcomp.p, st));
+        CK(cudaMemsetAsync(S.d_bd_acc.p + first * 3 * L, 0, count * 3 * L * sizeof(double), st));
+    }
     // K3 per segment width, forked onto side streams so the widths run concurrently
     const bool full = first == 0 && count == S.n_pts;
     CK(cudaMemsetAsync(S.d_counter.p, 0, N_GROUPS * sizeof(unsigned int), st));
@@ -797,6 +807,11 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         a.alg_ops = S.d_alg.p;
         a.lmax = S.lmax[w];
         a.pmax = S.pmax[w];
+        if (S.bd) {
+            a.bd = S.d_bd_acc.p;
+            a.layer = T.d_layer.p;
+            a.n_layers = L;
+        }
         uint64_t blocks;
         if (W <= 32) {
             const int nseg = 32 / W;
@@ -865,6 +880,62 @@ triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t firs
         CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
     }
+    return TRIOSIM_OK;
+}
+
+triosim_status triosim_set_breakdown(triosim_ctx *ctx, int32_t sweep_id, int enable) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    CK(cudaSetDevice(ctx->device));
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    const uint64_t L = ctx->traces.at(S.trace_handle)->n_layers;
+    CK(cudaDeviceSynchronize());   // no launch of this sweep may still use the buffers
+    S.bd = false;
+    S.d_lcomp.alloc(0);
+    S.d_bd_acc.alloc(0);
+    S.d_bd_stage.alloc(0);
+    if (!enable) return TRIOSIM_OK;
+    if (S.d_lcomp.alloc(S.classes.size() * L) != cudaSuccess || S.d_bd_acc.alloc(S.n_pts * 3 * L) != cudaSuccess) {
+        cudaGetLastError();
+        S.d_lcomp.alloc(0);
+        S.d_bd_acc.alloc(0);
+        return fail(ctx, TRIOSIM_ENOMEM, "breakdown buffers: %llu points x %llu layers",
+                    (unsigned long long)S.n_pts, (unsigned long long)L);
+    }
+    CK(cudaMemset(S.d_lcomp.p, 0, S.d_lcomp.n * sizeof(double) + (S.d_lcomp.n ? 0 : sizeof(double))));
+    CK(cudaMemset(S.d_bd_acc.p, 0, S.d_bd_acc.n * sizeof(double) + (S.d_bd_acc.n ? 0 : sizeof(double))));
+    S.bd = true;
+    return TRIOSIM_OK;
+}
+
+triosim_status triosim_breakdown(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
+                                 double *layer_compute_s, double *layer_comm_s, int out_is_device, void *cuda_stream) {
+    if (!ctx) return TRIOSIM_EINVAL;
+    CK(cudaSetDevice(ctx->device));
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    if (!S.bd) return fail(ctx, TRIOSIM_EINVAL, "breakdown not enabled on sweep %d (triosim_set_breakdown)", sweep_id);
+    if (first > S.n_pts || count > S.n_pts - first) return fail(ctx, TRIOSIM_ERANGE, "range outside sweep");
+    const uint64_t L = ctx->traces.at(S.trace_handle)->n_layers;
+    if (count == 0 || L == 0) return TRIOSIM_OK;
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    if (out_is_device) {
+        CK(launch_k4_breakdown(S.d_pts.p, S.d_res.p, first, count, (uint32_t)L, S.d_lcomp.p, S.d_bd_acc.p,
+                               layer_compute_s, layer_comm_s, st));
+        return TRIOSIM_OK;
+    }
+    const uint64_t n = count * L;
+    if (S.d_bd_stage.n < 2 * n && S.d_bd_stage.alloc(2 * n) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ctx, TRIOSIM_ENOMEM, "breakdown staging buffer");
+    }
+    CK(launch_k4_breakdown(S.d_pts.p, S.d_res.p, first, count, (uint32_t)L, S.d_lcomp.p, S.d_bd_acc.p,
+                           S.d_bd_stage.p, S.d_bd_stage.p + n, st));
+    if (layer_compute_s) CK(cudaMemcpyAsync(layer_compute_s, S.d_bd_stage.p, n * sizeof(double), cudaMemcpyDeviceToHost, st));
+    if (layer_comm_s) CK(cudaMemcpyAsync(layer_comm_s, S.d_bd_stage.p + n, n * sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
     return TRIOSIM_OK;
 }
 

@@ -44,7 +44,9 @@ struct OpHook {
 struct CollEnt {
     double S;         // payload bytes
     uint32_t kind;    // CK_*
-    uint32_t pad;
+    uint32_t pad;     // HYBRID K2: the communicated tensor
+    uint32_t layer;   // layer of the triggering operator (R22 per-layer breakdown)
+    uint32_t pad2;
 };
 
 // PIPE mode (GPipe): per stage of a class
@@ -159,6 +161,12 @@ struct K3Args {
     const HSend *hsends;
     triosim_result *out;
     unsigned long long *alg_ops;   // method fp64 operations performed
+    // R22 per-layer breakdown (kernel variant BD only): per point [3][n_layers] communication
+    // accumulators (TP-group collectives, DP-group collectives, P2P sends of the layer's
+    // representative rank), zeroed by the host before the launch
+    double *bd;
+    const uint32_t *layer;         // trace: layer of each operator
+    uint32_t n_layers, pad3;
 };
 
 // launchers (ts_kernels.cu)
@@ -172,8 +180,17 @@ cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
                              const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
                              RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
+// K3 variants: a.bd != nullptr selects the breakdown-recording (BD) instantiation
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s);      // ts_k3h.cu
+// R22: per-class layer compute (left fold of t' over the representative rank's program) and the
+// per-point finalisation into caller buffers (ts_kernels.cu)
+cudaError_t launch_k4_layer_compute(const ClassDesc *cls, uint32_t n_cls, const TraceDev &T, const double *dur,
+                                    const StageInfo *stages, const StageEnt *ents, const HEnt *hents,
+                                    double *lcomp, cudaStream_t s);
+cudaError_t launch_k4_breakdown(const PointDesc *pts, const triosim_result *res, uint64_t first, uint64_t count,
+                                uint32_t n_layers, const double *lcomp, const double *acc, double *out_comp,
+                                double *out_comm, cudaStream_t s);
 int k3h_max_blocks_per_sm(int W, uint32_t lmax, uint32_t pmax);   // dynamic smem: links (W > 32), ports
 size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax);
 int k3_max_blocks_per_sm(int W, int mode);

@@ -113,7 +113,9 @@ __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[
 #ifndef TS_K3_MINB
 #define TS_K3_MINB 1
 #endif
-template <int W, int MODE>
+// BD: also record the per-layer communication breakdown (R22) into a.bd (a separate instantiation,
+// so the plain timeline carries none of its state)
+template <int W, int MODE, bool BD>
 __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Args a) {
     constexpr int NSEG = 32 / W;
     constexpr int LMAX = lmax_warp(W);
@@ -176,6 +178,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     uint32_t alg = 0;            // fp64 operations of the method performed by this lane (wraps per point only beyond 4e9)
     uint64_t tmix = 0;           // mix64(bits(t)) of the current instant
     bool nev = false;            // this lane recorded an event at the current instant
+    // R22 (BD): the representative rank's current collective (rank 0) / P2P send (every stage):
+    // start or release time and the layer it is attributed to; category 0 TP / 1 DP / 2 P2P
+    double bd_t0 = 0.0;
+    uint32_t bd_l = 0, bd_cat = 0;
 
 #define EV(kind, code)                                                  \
     do {                                                                \
@@ -210,6 +216,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 ncoll = C->n_coll;
                 m = C->m;
                 tree_algo = TREE && C->algo == TRIOSIM_ALGO_TREE;
+                if constexpr (BD) bd_cat = !COLL ? 2u : C->strategy == TRIOSIM_TP ? 0u : 1u;
                 t = 0.0;
                 tmix = mix64(0ull);
                 ninst = nwf = nrounds = maxact = 0;
@@ -360,6 +367,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         }
                     } else {
                         dcnt++;
+                        if constexpr (BD) {   // R22: P2P time of the sending (representative) stage
+                            double *q = a.bd + ((size_t)pidx * 3 + 2) * a.n_layers + bd_l;
+                            *q = *q + (t - bd_t0);
+                        }
                     }
                 }
                 if constexpr (COLL) {
@@ -385,6 +396,11 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         if (dn) {
                             ldone = true;
                             donec = cur + 1;
+                            if constexpr (BD)
+                                if (li == 0) {   // R22: collective time on the representative rank
+                                    double *q = a.bd + ((size_t)pidx * 3 + bd_cat) * a.n_layers + bd_l;
+                                    *q = *q + (t - bd_t0);
+                                }
                         }
                     }
                     const bool allfin = (__ballot_sync(FULL, !used || ldone) & smask) == smask;
@@ -405,6 +421,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         D = 0;
                         ldone = uprel = upd = dnrel = dnd = false;
                         if (li == 0) { EV(EV_COLL_START, cur); alg += 1; }
+                        if constexpr (BD) { bd_t0 = t; bd_l = ce.layer; }
                     }
                     if (used && running && fst == FS_NONE) {
                         bool rel = false;
@@ -477,6 +494,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             alg += 2 * flen + 1;
                             fcode = (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg;
                             EV(EV_RELEASE, fcode);
+                            if constexpr (BD) {
+                                bd_t0 = t;
+                                bd_l = a.layer[a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + se.pidx].op];
+                            }
                             sq++;
                             if (t_act == t) more = true;
                         }
@@ -716,7 +737,8 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 
 template <int W, int MODE>
 static cudaError_t launch_wm(const K3Args &a, int grid, cudaStream_t s) {
-    k3_timeline<W, MODE><<<grid, K3_THREADS, 0, s>>>(a);
+    if (a.bd) k3_timeline<W, MODE, true><<<grid, K3_THREADS, 0, s>>>(a);
+    else k3_timeline<W, MODE, false><<<grid, K3_THREADS, 0, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -743,9 +765,9 @@ cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s
 template <int W>
 static int occ_w(int mode) {
     int nb = 0;
-    if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL>, K3_THREADS, 0);
-    else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE>, K3_THREADS, 0);
-    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE>, K3_THREADS, 0);
+    if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL, false>, K3_THREADS, 0);
+    else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE, false>, K3_THREADS, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE, false>, K3_THREADS, 0);
     return nb;
 }
 

@@ -93,6 +93,8 @@ struct Group {
     int K, D;
     double cS, chunk;
     uint32_t flow_deliv;      // deliveries of this group's flows (for counts)
+    double bd_t0;             // R22 (BD): start time of the running collective
+    uint32_t bd_l;            // ... and the layer it is attributed to
 };
 
 __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[h >> 1] >> (16 * (h & 1))) & 0xffff; }
@@ -144,7 +146,8 @@ __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f,
 }  // namespace
 
 
-template <int W, int NW>
+// BD: also record the per-layer communication breakdown (R22) into a.bd (separate instantiation)
+template <int W, int NW, bool BD>
 __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(const K3Args a) {
     constexpr int SL = NW == 1 ? W : 32 * NW;           // lanes per segment
     constexpr int NSEG = NW == 1 ? 32 / W : 1;          // segments per warp (NW = 1)
@@ -338,6 +341,14 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     FT.st = FD.st = FP.st = FS_NONE;
     uint64_t acc = 0, alg = 0, tmix = 0;
     bool nev = false;
+    // R22 (BD): this lane is its layers' representative rank (d = 0, t = 0); its P2P send in flight
+    bool bd_rep = false;
+    double bd_p_t0 = 0.0;
+    uint32_t bd_p_l = 0;
+    auto bd_add = [&](uint32_t cat, uint32_t l, double dt) {
+        double *q = a.bd + ((size_t)pidx * 3 + cat) * a.n_layers + l;
+        *q = *q + dt;
+    };
 
 #define EV(kind, code)                                                        \
     do {                                                                      \
@@ -368,6 +379,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         G.K = G.D = 0;
         G.cS = G.chunk = 0.0;
         G.flow_deliv = 0;
+        G.bd_t0 = 0.0;
+        G.bd_l = 0;
     };
     auto gpu_of_member = [&](const Group &G, int k) -> uint32_t { return a.ro[TR.ro_off + G.lane0 + k * G.stride]; };
     auto tp_seq = [&](uint32_t P, uint32_t j, uint32_t e) -> uint32_t {
@@ -396,6 +409,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             if (dn) {
                 G.ldone = true;
                 G.donec = G.cur + 1;
+                if constexpr (BD)
+                    if (bd_rep) bd_add(is_tp ? 0u : 1u, G.bd_l, t - G.bd_t0);
             }
         }
         const bool allfin = gall(G, G.ldone);
@@ -427,6 +442,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             if (G.i == 0) {
                 EV(EV_COLL_START, (G.gid << 20) | G.cur);
                 alg += 1;
+            }
+            if constexpr (BD) {
+                G.bd_t0 = t;
+                G.bd_l = ce.layer;
             }
         }
         if (G.member && G.running && F.st == FS_NONE) {
@@ -567,6 +586,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     d = r / (S * tp);
                     s = (r / tp) % S;
                     tt = r % tp;
+                    bd_rep = used && d == 0 && tt == 0;
                     SI = a.stages[C->stage_off + s];
                     HS = a.hst[C->hst_off + s];
                     nprog = used ? m * (SI.nF + SI.nB) + SI.nO : 0;
@@ -644,7 +664,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 if (used) {
                     if (flow_step(FT, dirty)) { nflow++; grp_delivered(GT); }
                     if (flow_step(FD, dirty)) { nflow++; grp_delivered(GD); }
-                    if (flow_step(FP, dirty)) { nflow++; np2p++; dcnt++; }
+                    if (flow_step(FP, dirty)) {
+                        nflow++; np2p++; dcnt++;
+                        if constexpr (BD)
+                            if (bd_rep) bd_add(2u, bd_p_l, t - bd_p_t0);
+                    }
                 }
                 cnt[li] = dcnt;
                 ssync();
@@ -668,6 +692,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         release(a, TR, FP, gpu, dg, se.bytes,
                                 (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg, t, lats, alg);
                         EV(EV_RELEASE, FP.code);
+                        if constexpr (BD) {
+                            bd_p_t0 = t;
+                            bd_p_l = a.layer[ent_at(P, se.pidx).op];
+                        }
                         sq++;
                         if (FP.t_act == t) more = true;
                     }
@@ -1078,15 +1106,19 @@ size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
     return (W <= 32 ? 0 : (size_t)lmax * 16) + ph;
 }
 
-template <int W, int NW>
-static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
+template <int W, int NW, bool BD>
+static cudaError_t launch_hb(const K3Args &a, int grid, cudaStream_t s) {
     const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, a.lmax, a.pmax);
     if (dyn > 0) {
-        const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+        const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW, BD>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
         if (e != cudaSuccess) return e;
     }
-    k3_hybrid<W, NW><<<grid, NW == 1 ? K3_THREADS : 32 * NW, dyn, s>>>(a);
+    k3_hybrid<W, NW, BD><<<grid, NW == 1 ? K3_THREADS : 32 * NW, dyn, s>>>(a);
     return cudaGetLastError();
+}
+template <int W, int NW>
+static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
+    return a.bd ? launch_hb<W, NW, true>(a, grid, s) : launch_hb<W, NW, false>(a, grid, s);
 }
 
 // W <= 32: W-lane segments in 256-thread CTAs; W = 64..1024: one point per CTA of W threads
@@ -1109,10 +1141,10 @@ cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
 template <int W, int NW>
 static int occ_h(uint32_t lmax, uint32_t pmax) {
     const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, lmax, pmax);
-    if (dyn > 0 && cudaFuncSetAttribute(k3_hybrid<W, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
+    if (dyn > 0 && cudaFuncSetAttribute(k3_hybrid<W, NW, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
         return 0;
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW, false>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
     return nb;
 }
 

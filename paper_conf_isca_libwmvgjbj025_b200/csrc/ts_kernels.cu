@@ -7,6 +7,7 @@
 //       k2_pipe        GPipe stage programs, P2P send / receive lists
 //  K3   k3_timeline    (ts_k3.cu) event-driven timeline + max-min progressive filling, one point
 //                      per W-lane warp segment (W = 2..32 simulated GPUs)
+//  K4   k4_layer_compute, k4_breakdown   per-layer compute / comm breakdown (R22; Fig. 13)
 //
 // Numerics: compiled with --fmad=false (no FMA contraction), IEEE division; every sum is a
 // left fold in the order DESIGN.md states, so results match the oracle bit for bit.
@@ -166,6 +167,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                     int trig = (C.strategy == TRIOSIM_DDP) ? T.prod[T.wgrad[j - 1]] : last_nonopt;
                     CE[nc].S = S;
                     CE[nc].kind = CK_AR;
+                    CE[nc].layer = T.layer[trig];
                     H[trig].nsig += 1;
                     payload = payload + S;
                     nc++;
@@ -207,6 +209,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         if (T.ts[x].batch_scaled) S = S * C.r_b;
                         CE[nc].S = S;
                         CE[nc].kind = (uint32_t)kind;
+                        CE[nc].layer = T.layer[o];
                         H[o].nsig += 1;
                         coll_of[x] = (int32_t)nc;
                         payload = payload + S;
@@ -547,6 +550,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                         if (T.ts[x].batch_scaled) ce.S = ce.S * C.r_b;
                         ce.kind = (uint32_t)kind;
                         ce.pad = x;
+                        ce.layer = op.layer;
+                        ce.pad2 = 0;
                         colls[toff[P] + tj[P]++] = ce;
                         ntp++;
                     }
@@ -585,17 +590,21 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     ce.S = Sb;
                     ce.kind = CK_AR;
                     ce.pad = 0;
-                    colls[hs.dcol_off + b++] = ce;
+                    ce.layer = T.layer[last_prod];
+                    ce.pad2 = 0;
                     // trigger: (producer of the bucket's last gradient, micro-batch 0); the HYBRID form
                     // of DataParallel (R6) triggers every bucket after the stage's last non-OPT op
                     if (C.dp_after_bwd && (si.nB > 0 || si.nF > 0)) {
-                        ents[si.nB > 0 ? eoff[1] + si.nB - 1 : eoff[0] + si.nF - 1].dp_nsig++;
+                        HEnt &te = ents[si.nB > 0 ? eoff[1] + si.nB - 1 : eoff[0] + si.nF - 1];
+                        te.dp_nsig++;
+                        ce.layer = T.layer[te.op];
                     } else {
                         const int P = (int)(T.info[last_prod] & INFO_PHASE_MASK);
                         const uint32_t cntP = P == 0 ? si.nF : P == 1 ? si.nB : si.nO;
                         for (uint32_t q = 0; q < cntP; q++)
                             if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig++; break; }
                     }
+                    colls[hs.dcol_off + b++] = ce;
                     sum = 0;
                     Sb = 0.0;
                     open = false;
@@ -717,6 +726,93 @@ cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, c
                              RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch, cudaStream_t s) {
     if (n == 0) return cudaSuccess;
     k2_hybrid<<<n, K2P_THREADS, 0, s>>>(cls, list, T, plan_pool, stages, hst, ents, sends, recvs, colls, scratch);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------
+// K4 (R22): per-layer breakdown.  k4_layer_compute: per class, one thread per layer, the left fold
+// of t' over the representative rank's program instances of that layer in program order (rank 0
+// runs every operator in DP / DDP / TP; in GPipe / HYBRID the layer's stage runs FWD of
+// micro-batches 0..m-1, BWD of m-1..0, OPT once).  k4_breakdown: per (point, layer), the class's
+// compute and comm = (TP-group + DP-group collective time) + P2P time from K3's accumulators.
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(128) k4_layer_compute(const ClassDesc *cls, TraceDev T, const double *dur,
+                                                        const StageInfo *stages, const StageEnt *ents,
+                                                        const HEnt *hents, double *lcomp) {
+    const ClassDesc &C = cls[blockIdx.x];
+    const uint32_t L = T.n_layers;
+    const double *du = dur + C.dur_off;
+    for (uint32_t l = threadIdx.x; l < L; l += blockDim.x) {
+        double acc = 0.0;
+        if (C.mode == MODE_COLL || C.mode == MODE_TREE) {
+            for (uint32_t o = 0; o < T.n_ops; o++)
+                if (T.layer[o] == l) acc = acc + du[o];
+        } else {
+            const bool hyb = C.mode == MODE_HYBRID;
+            auto op_at = [&](uint32_t e) -> uint32_t { return hyb ? hents[e].op : ents[e].op; };
+            // the stage that runs layer l (stages hold contiguous layers, every op of l in one stage)
+            int st = -1;
+            for (uint32_t s = 0; s < C.p && st < 0; s++) {
+                const StageInfo SI = stages[C.stage_off + s];
+                const uint32_t n = SI.nF + SI.nB + SI.nO;
+                for (uint32_t e = 0; e < n; e++)
+                    if (T.layer[op_at(SI.ent_off + e)] == l) { st = (int)s; break; }
+            }
+            if (st >= 0) {
+                const StageInfo SI = stages[C.stage_off + st];
+                for (uint32_t j = 0; j < C.m; j++)
+                    for (uint32_t e = 0; e < SI.nF; e++) {
+                        const uint32_t o = op_at(SI.ent_off + e);
+                        if (T.layer[o] == l) acc = acc + du[o];
+                    }
+                for (uint32_t j = 0; j < C.m; j++)
+                    for (uint32_t e = 0; e < SI.nB; e++) {
+                        const uint32_t o = op_at(SI.ent_off + SI.nF + e);
+                        if (T.layer[o] == l) acc = acc + du[o];
+                    }
+                for (uint32_t e = 0; e < SI.nO; e++) {
+                    const uint32_t o = op_at(SI.ent_off + SI.nF + SI.nB + e);
+                    if (T.layer[o] == l) acc = acc + du[o];
+                }
+            }
+        }
+        lcomp[(size_t)blockIdx.x * L + l] = acc;
+    }
+}
+
+cudaError_t launch_k4_layer_compute(const ClassDesc *cls, uint32_t n_cls, const TraceDev &T, const double *dur,
+                                    const StageInfo *stages, const StageEnt *ents, const HEnt *hents,
+                                    double *lcomp, cudaStream_t s) {
+    if (n_cls == 0 || T.n_layers == 0) return cudaSuccess;
+    k4_layer_compute<<<n_cls, 128, 0, s>>>(cls, T, dur, stages, ents, hents, lcomp);
+    return cudaGetLastError();
+}
+
+__global__ void k4_breakdown(const PointDesc *pts, const triosim_result *res, uint64_t first, uint64_t count,
+                             uint32_t L, const double *lcomp, const double *acc, double *out_comp, double *out_comm) {
+    const uint64_t n = count * L;
+    for (uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < n; q += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = first + q / L;
+        const uint32_t l = (uint32_t)(q % L);
+        double c = 0.0, m = 0.0;
+        if (res[i].status == TRIOSIM_PT_OK) {
+            const double *A = acc + i * 3ull * L;
+            c = lcomp[(size_t)pts[i].cls * L + l];
+            m = (A[l] + A[L + l]) + A[2 * L + l];
+        }
+        if (out_comp) out_comp[q] = c;
+        if (out_comm) out_comm[q] = m;
+    }
+}
+
+cudaError_t launch_k4_breakdown(const PointDesc *pts, const triosim_result *res, uint64_t first, uint64_t count,
+                                uint32_t n_layers, const double *lcomp, const double *acc, double *out_comp,
+                                double *out_comm, cudaStream_t s) {
+    const uint64_t n = count * n_layers;
+    if (n == 0) return cudaSuccess;
+    uint64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    k4_breakdown<<<(unsigned)blocks, 256, 0, s>>>(pts, res, first, count, n_layers, lcomp, acc, out_comp, out_comm);
     return cudaGetLastError();
 }
 

@@ -19,7 +19,8 @@ LIB_PATH = os.environ.get("TRIOSIM_LIB", os.path.join(HERE, "libtriosim.so"))
 
 EXPORTS = ["triosim_create", "triosim_destroy", "triosim_last_error", "triosim_load_trace", "triosim_build_sweep",
            "triosim_simulate_batch", "triosim_results", "triosim_release", "triosim_launch_counts",
-           "triosim_results_device_ptr", "triosim_work_counters", "triosim_timing", "triosim_timings"]
+           "triosim_results_device_ptr", "triosim_work_counters", "triosim_timing", "triosim_timings",
+           "triosim_set_breakdown", "triosim_breakdown"]
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENOTFOUND", -5: "ERANGE", -6: "EUNSUPPORTED"}
 
@@ -72,6 +73,8 @@ def load_library(path=LIB_PATH):
         L.triosim_work_counters.argtypes = [P, i32, C.POINTER(u64)]
         L.triosim_timing.argtypes = [P, C.c_int]
         L.triosim_timings.argtypes = [P, P, P, i32]
+        L.triosim_set_breakdown.argtypes = [P, i32, C.c_int]
+        L.triosim_breakdown.argtypes = [P, i32, u64, u64, P, P, C.c_int, P]
         L.triosim_results_device_ptr.argtypes = [P, i32]
         L.triosim_results_device_ptr.restype = P
         for f in EXPORTS:
@@ -170,6 +173,25 @@ class Context:
         self._check("triosim_results", st)
         return out
 
+    def triosim_set_breakdown(self, sweep_id: int, enable=True):
+        """Record the per-layer breakdown (R22) in later simulate_batch calls."""
+        self._check("triosim_set_breakdown", self.L.triosim_set_breakdown(self.h, int(sweep_id), 1 if enable else 0))
+
+    def triosim_breakdown(self, sweep_id: int, first: int, count: int, n_layers: int, device_ptrs=None, stream=0):
+        """Per-layer (compute, comm) times [count, n_layers] as numpy arrays, or, with device_ptrs =
+        (compute_ptr, comm_ptr), a stream-ordered write into device memory."""
+        sp = C.c_void_p(int(stream)) if stream else None
+        if device_ptrs is not None:
+            cp, mp = (None if v is None else C.c_void_p(int(v)) for v in device_ptrs)
+            self._check("triosim_breakdown", self.L.triosim_breakdown(self.h, int(sweep_id), int(first), int(count),
+                                                                      cp, mp, 1, sp))
+            return None
+        comp = np.zeros((count, n_layers))
+        comm = np.zeros((count, n_layers))
+        self._check("triosim_breakdown", self.L.triosim_breakdown(self.h, int(sweep_id), int(first), int(count),
+                                                                  _ptr(comp), _ptr(comm), 0, sp))
+        return comp, comm
+
     def triosim_release(self, handle: int):
         self._check("triosim_release", self.L.triosim_release(self.h, int(handle)))
 
@@ -198,11 +220,16 @@ class Context:
         return self.L.triosim_results_device_ptr(self.h, int(sweep_id)) or 0
 
     # -- convenience --
-    def run_sweep(self, sw: W.Sweep, stream=0):
+    def run_sweep(self, sw: W.Sweep, stream=0, breakdown=False):
+        """Results of every point; with breakdown=True also the per-layer (compute, comm) arrays (R22)."""
         tid = self.triosim_load_trace(sw.trace)
         sid = self.triosim_build_sweep(tid, sw.topos, sw.points, sw.plans or None)
+        if breakdown:
+            self.triosim_set_breakdown(sid, True)
         self.triosim_simulate_batch(sid, 0, len(sw.points), stream)
         res = self.triosim_results(sid, 0, len(sw.points), stream=stream)
+        if breakdown:
+            bd = self.triosim_breakdown(sid, 0, len(sw.points), sw.trace.n_layers, stream=stream)
         self.triosim_release(sid)
         self.triosim_release(tid)
-        return res
+        return (res, *bd) if breakdown else res

@@ -1,0 +1,117 @@
+"""GPU parity of the per-layer compute / communication breakdown ("the communication time and
+computation time of each layer or stage"; Fig. 13; R22) against the oracle, through the C ABI
+(triosim_set_breakdown / triosim_breakdown).  Every point of seeded random sweeps over every strategy,
+collective algorithm, the one-point-per-CTA kernel and the photonic network; the C2 bench sweep on a
+sample; and the invariant that recording the breakdown does not change any result bit."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_isca_libwmvgjbj025_b200 import workloads as W
+from tests import sweeps as S
+
+pytestmark = pytest.mark.gpu
+RTOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_isca_libwmvgjbj025_b200 import triosim
+    c = triosim.Context(0)
+    yield c
+    c.close()
+
+
+def _check(ctx, sw, idx=None):
+    plain = ctx.run_sweep(sw)
+    got, comp, comm = ctx.run_sweep(sw, breakdown=True)
+    # the BD kernel variant computes the same timeline: every result bit identical
+    assert got.tobytes() == plain.tobytes()
+    idx = list(range(len(sw.points))) if idx is None else idx
+    ref, rc, rm = oracle.run_sweep(sw, idx, breakdown=True)
+    bad = []
+    for q, i in enumerate(idx):
+        if got[i]["status"] != ref[q]["status"]:
+            bad.append(f"point {i}: status {got[i]['status']} vs {ref[q]['status']}")
+            continue
+        if got[i]["status"] != 0:
+            if np.any(comp[i] != 0) or np.any(comm[i] != 0):
+                bad.append(f"point {i}: failed point with a non-zero breakdown")
+            continue
+        for name, g, r in (("compute", comp[i], rc[q]), ("comm", comm[i], rm[q])):
+            err = np.abs(g - r) > RTOL * np.abs(r)
+            if err.any():
+                l = int(np.argmax(err))
+                bad.append(f"point {i}: layer {l} {name} gpu={g[l]!r} oracle={r[l]!r}")
+    assert not bad, "\n".join(bad[:20])
+    return got, comp, comm
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_breakdown_random_small_all_strategies(ctx, seed):
+    got, comp, comm = _check(ctx, S.random_small(seed))
+    assert (got["status"] == 0).sum() > 300
+    ok = got["status"] == 0
+    assert (comm[ok].sum(axis=1) > 0).any()
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_breakdown_random_hybrid(ctx, seed):
+    _check(ctx, S.random_hybrid(seed))
+
+
+def test_breakdown_large_points_cta_kernel(ctx):
+    _check(ctx, S.large_points(0))
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_breakdown_random_photonic(ctx, seed):
+    _check(ctx, S.random_photonic(seed))
+
+
+def test_breakdown_c1_partitions_compute_busy(ctx):
+    """DDP on the C1 MLP: rank 0 runs every operator, so the layers partition compute_busy_max; the
+    trace has dyadic times, so the identity is exact."""
+    sw = W.sweep_c1()
+    got, comp, comm = _check(ctx, sw)
+    for i in range(len(sw.points)):
+        acc = 0.0
+        for v in comp[i]:
+            acc = acc + float(v)
+        assert acc == got[i]["compute_busy_max_s"]
+
+
+def test_breakdown_c2_sampled_and_ranges(ctx):
+    """The bench workload (configs[1], 10,000 points) with the breakdown on: a seeded sample against the
+    oracle; partial ranges and device-pointer outputs equal the full host copy."""
+    import torch
+    sw = W.sweep_c2()
+    rng = np.random.Generator(np.random.PCG64(22))
+    idx = sorted(rng.choice(len(sw.points), size=60, replace=False).tolist())
+    _check(ctx, sw, idx)
+    tid = ctx.triosim_load_trace(sw.trace)
+    sid = ctx.triosim_build_sweep(tid, sw.topos, sw.points)
+    with pytest.raises(Exception):
+        ctx.triosim_breakdown(sid, 0, 1, sw.trace.n_layers)   # not enabled
+    ctx.triosim_set_breakdown(sid, True)
+    ctx.triosim_simulate_batch(sid, 0, len(sw.points))
+    L = sw.trace.n_layers
+    comp, comm = ctx.triosim_breakdown(sid, 0, len(sw.points), L)
+    for first, count in ((0, 1), (4321, 777), (9999, 1)):
+        ctx.triosim_simulate_batch(sid, first, count)
+        c2, m2 = ctx.triosim_breakdown(sid, first, count, L)
+        assert c2.tobytes() == comp[first:first + count].tobytes()
+        assert m2.tobytes() == comm[first:first + count].tobytes()
+    dc = torch.zeros((len(sw.points), L), dtype=torch.float64, device="cuda")
+    dm = torch.zeros_like(dc)
+    s = torch.cuda.current_stream()
+    ctx.triosim_breakdown(sid, 0, len(sw.points), L, device_ptrs=(dc.data_ptr(), dm.data_ptr()), stream=s.cuda_stream)
+    torch.cuda.synchronize()
+    assert dc.cpu().numpy().tobytes() == comp.tobytes() and dm.cpu().numpy().tobytes() == comm.tobytes()
+    with pytest.raises(Exception):
+        ctx.triosim_breakdown(sid, 9990, 20, L)
+    ctx.triosim_set_breakdown(sid, False)
+    ctx.triosim_release(sid)
+    ctx.triosim_release(tid)

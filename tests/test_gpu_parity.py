@@ -9,6 +9,7 @@ import pytest
 
 import oracle
 from paper_conf_isca_libwmvgjbj025_b200 import workloads as W
+from tests import sweeps as S
 from tests.parity import compare
 
 pytestmark = pytest.mark.gpu
@@ -50,34 +51,9 @@ def test_c1_mlp_dp2_exact(ctx):
 def test_random_small_all_strategies(ctx, seed):
     """Random traces x random topologies x every strategy / collective, several hundred points
     so each launch spans many warps, segments and a ragged tail."""
-    rng = np.random.Generator(np.random.PCG64(500 + seed))
-    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=4)
-    topos = [W.random_topology(rng, n_gpus=g, n_switch=int(rng.integers(0, 3)), p_edge=0.25)
-             for g in (2, 3, 4, 5, 8, 12)]
-    topos += [W.ring(16, 40e9, 1e-6), W.star(8, 80e9, 2e-6), W.mesh(2, 4, 60e9, 1e-6), W.cube_mesh8(50e9, 1e-6),
-              W.double_ring(8, 30e9, 3e-6), W.perturb(W.ring_graph(8, 90e9, 1e-6), seed)]
-    pts = []
-    for _ in range(400):
-        ti = int(rng.integers(len(topos)))
-        G = topos[ti].n_gpus
-        st = int(rng.integers(0, 4))
-        bw, lat = float(rng.uniform(0.2, 3.0)), float(rng.uniform(0.0, 2.0))
-        algo = int(rng.integers(0, 2))
-        if st in (W.ST_DP, W.ST_DDP):
-            dp = int(rng.integers(1, G + 1))
-            pts.append(W.make_point(ti, st, dp=dp, B=dp * int(rng.integers(1, 9)), algo=algo, bw=bw, lat=lat,
-                                    bucket=int(rng.choice([0, 1 << 10, 1 << 14, 1 << 30]))))
-        elif st == W.ST_TP:
-            tpd = int(rng.integers(1, G + 1))
-            pts.append(W.make_point(ti, st, tp=tpd, B=int(rng.integers(1, 9)), algo=algo, bw=bw, lat=lat,
-                                    tp_mode=int(rng.integers(0, 2))))
-        else:
-            pp = int(rng.integers(1, min(G, tr.n_layers) + 1))
-            m = int(rng.integers(1, 6))
-            pts.append(W.make_point(ti, st, pp=pp, m=m, B=m * int(rng.integers(1, 4)), bw=bw, lat=lat))
-    sw = W.Sweep("rand", tr, topos, W.points_array(pts))
+    sw = S.random_small(seed)
     got = ctx.run_sweep(sw)
-    check(got, sw, list(range(len(pts))))
+    check(got, sw, list(range(len(sw.points))))
     assert (got["status"] == 0).sum() > 300
 
 
@@ -85,25 +61,9 @@ def test_random_small_all_strategies(ctx, seed):
 def test_random_hybrid(ctx, seed):
     """HYBRID DP x TP x PP (R9) on random traces / topologies: every degree split, both TP modes,
     ring and tree, buckets, micro-batches; compared point by point with the oracle."""
-    rng = np.random.Generator(np.random.PCG64(900 + seed))
-    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=2)
-    topos = [W.random_topology(rng, n_gpus=g, n_switch=int(rng.integers(0, 3)), p_edge=0.2) for g in (4, 8, 12)]
-    topos += [W.star(16, 50e9, 1e-6), W.mesh(4, 4, 40e9, 2e-6), W.perturb(W.cube_mesh8(60e9, 1e-6), seed)]
-    pts = []
-    for _ in range(250):
-        ti = int(rng.integers(len(topos)))
-        G = topos[ti].n_gpus
-        while True:
-            dp, tp, pp = (int(rng.integers(1, 5)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 4)))
-            if dp * tp * pp <= G and pp <= tr.n_layers:
-                break
-        m = int(rng.integers(1, 4))
-        pts.append(W.make_point(ti, W.ST_HYBRID, dp=dp, tp=tp, pp=pp, m=m, B=dp * m * int(rng.integers(1, 3)),
-                                bucket=int(rng.choice([0, 1 << 12, 1 << 30])), tp_mode=int(rng.integers(0, 2)),
-                                algo=int(rng.integers(0, 2)), bw=float(rng.uniform(0.3, 3)), lat=float(rng.uniform(0, 2))))
-    sw = W.Sweep("hyb", tr, topos, W.points_array(pts))
+    sw = S.random_hybrid(seed)
     got = ctx.run_sweep(sw)
-    check(got, sw, list(range(len(pts))))
+    check(got, sw, list(range(len(sw.points))))
     assert (got["status"] == 0).sum() > 200
 
 
@@ -111,24 +71,10 @@ def test_random_hybrid(ctx, seed):
 def test_large_points_cta_kernel(ctx, seed):
     """More than 32 simulated GPUs (configs[4] scale): DDP / TP / PP points map to their exactly
     equivalent HYBRID form and run one point per CTA (64-256 ranks); compared with the oracle."""
-    rng = np.random.Generator(np.random.PCG64(1300 + seed))
-    tr = W.transformer_trace("tiny-gpt", 8, 64, 4, 256, 16, 100, 2, 11 + seed)
-    topos = [W.ring(64, 50e9, 1e-6), W.star(64, 80e9, 1e-6), W.hierarchical(8, 8, 1.0, 0.125, 2.0),
-             W.perturb_subset(W.hierarchical(32, 8, 1.0, 0.125, 4.0), 7 + seed)]
-    P = W.make_point
-    pts = [P(0, W.ST_DDP, dp=64, B=128, bucket=1 << 14, bw=2e9, lat=1e-6),
-           P(1, W.ST_DDP, dp=48, B=96, bucket=0, bw=5e9, lat=2e-6, algo=W.ALG_TREE),
-           P(1, W.ST_TP, tp=64, B=4, tp_mode=W.TPM_MEGATRON),
-           P(1, W.ST_TP, tp=48, B=4, tp_mode=W.TPM_PAPER, algo=W.ALG_TREE),
-           P(2, W.ST_HYBRID, dp=4, tp=8, pp=2, m=4, B=16, bucket=1 << 16, bw=100e9, lat=1e-6),
-           P(2, W.ST_HYBRID, dp=8, tp=4, pp=2, m=2, B=16, bucket=0, bw=100e9, lat=2e-6, tp_mode=W.TPM_PAPER),
-           P(3, W.ST_HYBRID, dp=8, tp=8, pp=4, m=4, B=32, bucket=1 << 18, bw=300e9, lat=1e-6),
-           P(3, W.ST_HYBRID, dp=16, tp=4, pp=4, m=2, B=32, bucket=1 << 18, bw=300e9, lat=1e-6, algo=W.ALG_TREE),
-           P(3, W.ST_PP, pp=8, m=4, B=8, bw=300e9, lat=1e-6)]
-    sw = W.Sweep("large", tr, topos, W.points_array(pts))
+    sw = S.large_points(seed)
     got = ctx.run_sweep(sw)
     assert (got["status"] == 0).all(), got["status"]
-    check(got, sw, list(range(len(pts))))
+    check(got, sw, list(range(len(sw.points))))
 
 
 def test_statuses_and_edge_cases(ctx):
@@ -286,45 +232,9 @@ def test_random_photonic(ctx, seed):
     the hybrid kernel, whose lanes own their logical links), 1-4 ports (LRU teardown), 0-2 receive
     buffers, with and without setup latency; mixed in one sweep with flow-network points so warp
     segments of both models share a warp.  Compared point by point with the oracle."""
-    rng = np.random.Generator(np.random.PCG64(1700 + seed))
-    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 7)), max_ops_per_layer=4, b0=2)
-    topos = []
-    for g in (2, 3, 4, 8, 12, 16, 40):
-        topos.append(W.photonic(g, ports=int(rng.integers(1, 5)), link_bw=float(rng.uniform(5e9, 80e9)),
-                                setup=float(rng.choice([0.0, 1e-5, 2e-4])), lat=float(rng.choice([0.0, 1e-6])),
-                                buf_slots=int(rng.integers(0, 3)),
-                                ring_order=rng.permutation(g).astype(np.uint32)))
-    topos += [W.ring(8, 40e9, 1e-6), W.mesh(2, 4, 60e9, 1e-6)]
-    pts = []
-    P = W.make_point
-    for _ in range(300):
-        ti = int(rng.integers(len(topos)))
-        G = topos[ti].n_gpus
-        st = int(rng.integers(0, 5))
-        bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
-        algo = int(rng.integers(0, 2))
-        if st in (W.ST_DP, W.ST_DDP):
-            dp = int(rng.integers(1, G + 1))
-            pts.append(P(ti, st, dp=dp, B=dp * int(rng.integers(1, 5)), algo=algo, bw=bw, lat=lat,
-                         bucket=int(rng.choice([0, 1 << 12, 1 << 30]))))
-        elif st == W.ST_TP:
-            pts.append(P(ti, st, tp=int(rng.integers(1, G + 1)), B=int(rng.integers(1, 5)), algo=algo, bw=bw,
-                         lat=lat, tp_mode=int(rng.integers(0, 2))))
-        elif st == W.ST_PP:
-            m = int(rng.integers(1, 5))
-            pts.append(P(ti, st, pp=int(rng.integers(1, min(G, tr.n_layers) + 1)), m=m, B=m * int(rng.integers(1, 3)),
-                         bw=bw, lat=lat))
-        else:
-            while True:
-                dp, tpd, pp = int(rng.integers(1, 4)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 4))
-                if dp * tpd * pp <= G and pp <= tr.n_layers:
-                    break
-            m = int(rng.integers(1, 3))
-            pts.append(P(ti, W.ST_HYBRID, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m, algo=algo, bw=bw, lat=lat,
-                         tp_mode=int(rng.integers(0, 2)), bucket=int(rng.choice([0, 1 << 30]))))
-    sw = W.Sweep("phot", tr, topos, W.points_array(pts))
+    sw = S.random_photonic(seed)
     got = ctx.run_sweep(sw)
-    check(got, sw, list(range(len(pts))), allow_too_large=True)
+    check(got, sw, list(range(len(sw.points))), allow_too_large=True)
     phot = np.array([sw.topos[int(p["topo"])].photonic is not None for p in sw.points])
     # the one kernel limit: tree collectives over photonic links (the broadcast flow's sender is another lane)
     tl = got["status"] == W.PT_TOO_LARGE
