@@ -245,8 +245,13 @@ def main():
     n = len(sw.points)
     maxc = maxc if (args.shard and world > 1) else n
     ctx = triosim.Context(local)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
     tid = ctx.triosim_load_trace(sw.trace)
+    t1 = time.perf_counter()
     sid = ctx.triosim_build_sweep(tid, sw.topos, sw.points, sw.plans or None)
+    t2 = time.perf_counter()
+    setup_ms = {"load_trace": round((t1 - t0) * 1e3, 3), "build_sweep": round((t2 - t1) * 1e3, 3)}
     stream = torch.cuda.Stream()
     rec = W.RESULT_DTYPE.itemsize
     res_local = torch.zeros(n * rec, dtype=torch.uint8, device="cuda")
@@ -323,6 +328,33 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
 
+    # the p = 8 slice of C2 timed on its own, per-tensor and 25 MiB buckets
+    slices = {}
+    if args.config == "c2" and rank == 0 and not args.shard:
+        for name, bucket in (("p8_per_tensor", 0), ("p8_bucket_25MiB", 25 << 20)):
+            sel = (sw.points["dp"] == 8) & (sw.points["bucket_bytes"] == bucket)
+            if not sel.any():
+                continue
+            t3 = ctx.triosim_load_trace(sw.trace)
+            s3 = ctx.triosim_build_sweep(t3, sw.topos, sw.points[sel], sw.plans or None)
+            k = int(sel.sum())
+            times = []
+            for r in range(6):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                with torch.cuda.stream(stream):
+                    flush.zero_()
+                    e0.record(stream)
+                ctx.triosim_simulate_batch(s3, 0, k, stream.cuda_stream)
+                e1.record(stream)
+                torch.cuda.synchronize()
+                if r > 0:
+                    times.append(e0.elapsed_time(e1))
+            ctx.triosim_release(s3)
+            ctx.triosim_release(t3)
+            med = float(np.median(times))
+            slices[name] = {"points": k, "value": round(k / (med / 1e3), 1), "unit": UNIT, "ms": round(med, 4),
+                            "timing": "median of 5 device-timed simulate_batch calls, L2 flushed before each"}
+
     if rank == 0:
         pk, src = peaks()
         k3 = float(np.mean(k3_ms)) if len(k3_ms) else float("nan")
@@ -362,12 +394,18 @@ def main():
             "e2e": {"value": round(e2e_points / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(n * rec), "ms_per_step": round(e2e_ms, 3)},
             "gpu_launches": int(gpu_launches),
+            "setup_ms": setup_ms,
             "clocks": clk.summary(),
             "paper_context": "TrioSim (Go/Akita, 1 CPU process): 'within seconds' per simulation, host not "
                              "stated (P:29, P:306)",
         }
+        if slices:
+            out["slices"] = slices
         if not args.no_cpu_baseline and world == 1:
-            out["cpu_baseline"] = oracle_rate(args.config, seconds=args.cpu_seconds)
+            cb = oracle_rate(args.config, seconds=args.cpu_seconds)
+            out["cpu_baseline"] = cb
+            out["speedup_vs_oracle"] = {"one_core": round(value / cb["single_core_value"], 1),
+                                        f"{cb['cores']}_cores": round(value / cb["value"], 1)}
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.barrier()

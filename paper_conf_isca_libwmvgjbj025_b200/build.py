@@ -10,12 +10,12 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = [os.path.join(HERE, "csrc", f) for f in ("ts_host.cu", "ts_kernels.cu", "ts_k3.cu", "ts_k3h.cu")]
 HDR = [os.path.join(HERE, "csrc", "ts_internal.h"), os.path.join(ROOT, "include", "triosim.h")]
-OUT = os.path.join(HERE, "libtriosim.so")
+OUT = os.environ.get("TS_BUILD_OUT", os.path.join(HERE, "libtriosim.so"))   # override: A/B variants
 OBJ = os.path.join(HERE, "csrc", "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = [*ARCH, "-lineinfo", "-O3", "--fmad=false", "-std=c++17", "-Xcompiler", "-fPIC",
-         "-I" + os.path.join(ROOT, "include")]
+         "-I" + os.path.join(ROOT, "include")] + os.environ.get("TS_NVCC_EXTRA", "").split()
 
 
 def stale() -> bool:

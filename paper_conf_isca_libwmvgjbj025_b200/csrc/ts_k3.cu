@@ -14,6 +14,7 @@
 // changed, and the instant repeats if that made a flow drain now.
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdio>
 #include "ts_internal.h"
 
 namespace ts {
@@ -150,6 +151,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     double bstart = 0.0, cbusy = 0.0;
     uint32_t cur = 0;
     bool running = false, tree_cur = false, tree_algo = false, ring_fast = false, ring_uni = false;
+    bool ring_ff = false;   // uniform ring whose lanes also share one route latency: ring fast-forward
+#ifdef TS_WATCHDOG
+    unsigned int wd_iter = 0;
+#endif
     int K = 0;
     double cS = 0.0, chunk = 0.0;
     // ---- per-lane state ----
@@ -202,6 +207,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 exhausted = true;
             } else {
                 fresh = have = true;
+#ifdef TS_WATCHDOG
+                wd_iter = 0;
+#endif
                 const PointDesc pd = a.pts[a.work[it]];
                 pidx = pd.idx;
                 bws = pd.bw_scale;
@@ -289,7 +297,12 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
               // water-filling call is a single round at that rate (R14)
               const double lo = seg_min_shfl<W>(used ? rbw : dinf());
               const double hi = seg_max<W>(used ? rbw : 0.0);
-              if (fresh) ring_uni = ring_fast && lo == hi;
+              const double llo = seg_min_shfl<W>(used ? Lring : dinf());
+              const double lhi = seg_max<W>(used ? Lring : 0.0);
+              if (fresh) {
+                  ring_uni = ring_fast && lo == hi;
+                  ring_ff = ring_uni && llo == lhi && llo > 0.0;
+              }
           }
           if (__any_sync(FULL, fresh && (rbad || rlong))) {
               // a needed (src, dst) pair without a path (R3) / beyond this kernel's hop limit
@@ -309,6 +322,83 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
         // done when every segment has drained the work list (a segment whose point was just
         // rejected refills on the next iteration)
         if (__all_sync(FULL, !have && exhausted)) break;
+#ifdef TS_WATCHDOG
+        {
+            static __device__ unsigned int wd_printed = 0;
+            if (have && ++wd_iter > 2000000u) {
+                if (atomicAdd(&wd_printed, 1u) < 16u)
+                    printf("WD pidx=%u li=%d used=%d t=%.17g t_end=%.17g cst=%d fst=%d t_act=%.17g t_drain=%.17g D=%d K=%d cur=%u running=%d ring_ff=%d ldone=%d pos=%u nprog=%u\n",
+                           pidx, li, (int)used, t, t_end, cst, fst, t_act, t_drain, D, K, cur, (int)running, (int)ring_ff, (int)ldone, pos, nprog);
+                if (wd_iter > 2000010u) { have = false; exhausted = true; used = false; }
+            }
+        }
+#endif
+
+        // ------------------------- exact fast-forward of a uniform ring -------------------------
+        // While a ring collective runs on a link-disjoint ring with one bandwidth and one route
+        // latency, every lane releases, activates and delivers its step at the same instants:
+        // activation at t_a (rate = rbw after one progressive-filling round, drain t_a + chunk/rbw)
+        // and delivery + release of the next step at t_d (activation t_d + L).  Until the first
+        // compute completion t_c (the only other pending event: the lanes' flows are all in this
+        // collective and no operator can start before it is done), those instants are processed
+        // here lane-locally, with exactly the arithmetic, events, hash terms and counters of the
+        // general pass below (R13-R19) -- only without its warp-wide votes.  The collective's last
+        // delivery, a zero-length drain / latency and any instant at or after t_c go to the
+        // general pass.
+        if constexpr (COLL) {
+            if (__any_sync(FULL, have && running && ring_ff && !tree_cur)) {
+                const double tc = seg_min_shfl<W>(used && cst == CS_RUN ? t_end : dinf());
+                const int Dseg = __shfl_sync(FULL, D, sbase);
+                // segment-uniform copies (every used lane holds the same values; unused lanes follow them)
+                const double rbw0 = __shfl_sync(FULL, rbw, sbase), L0 = __shfl_sync(FULL, Lring, sbase);
+                const bool okl = !used || (fst == FS_LAT && t_act == t && D == Dseg && flen > 0);
+                const bool allok = (__ballot_sync(FULL, okl) & smask) == smask;   // (every lane votes)
+                const bool ok = allok && have && running && ring_ff && !tree_cur && chunk > 0.0 && Dseg < K && t < tc;
+                if (ok) {
+                    const double x = chunk / rbw0;  // = rem / rate at activation (rem = chunk, rate = rbw)
+                    bool actv = true;               // the instant at t activates step D
+                    int Dseg_l = Dseg;              // steps delivered so far (segment-uniform)
+                    for (;;) {
+                        if (actv) {
+                            const double td = t + x;
+                            if (!(t < tc) || !(td > t)) break;
+                            if (used) {
+                                EV(EV_ACTIVATE, fcode);
+                                fst = FS_ACT;
+                                rem = chunk;
+                                t_upd = t;
+                                rate = rbw;
+                                t_drain = td;
+                                alg += 2;
+                            }
+                            nrounds++;
+                            if ((uint32_t)p > maxact) maxact = (uint32_t)p;
+                            t = tc < td ? tc : td;   // next instant: the drain, or a compute completion first
+                        } else {
+                            const double ta = t + L0;
+                            if (!(t < tc) || Dseg_l + 1 >= K || !(ta > t)) break;
+                            if (used) {
+                                EV(EV_DELIVER, fcode);
+                                nflow++;
+                                D = Dseg_l + 1;
+                                fcode = ((uint64_t)cur << 32) | ((uint64_t)D << 16) | (uint64_t)li;
+                                EV(EV_RELEASE, fcode);
+                                fst = FS_LAT;
+                                t_act = ta;
+                                alg += 1;
+                            }
+                            Dseg_l++;
+                            t = tc < ta ? tc : ta;
+                        }
+                        actv = !actv;
+                        nwf++;
+                        ninst++;
+                        nev = false;
+                        tmix = mix64((uint64_t)__double_as_longlong(t));
+                    }
+                }
+            }
+        }
 
         // ------------------------------ one instant at time t ------------------------------
         bool dirty = false;

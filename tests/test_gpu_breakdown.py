@@ -33,6 +33,8 @@ def _check(ctx, sw, idx=None):
     ref, rc, rm = oracle.run_sweep(sw, idx, breakdown=True)
     bad = []
     for q, i in enumerate(idx):
+        if got[i]["status"] == W.PT_TOO_LARGE and ref[q]["status"] == 0:
+            continue   # a documented kernel limit (tree collectives over photonic links, R20)
         if got[i]["status"] != ref[q]["status"]:
             bad.append(f"point {i}: status {got[i]['status']} vs {ref[q]['status']}")
             continue
