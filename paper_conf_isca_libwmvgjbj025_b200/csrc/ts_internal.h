@@ -13,7 +13,7 @@ enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 constexpr int MAX_HOPS = 8;
 constexpr uint8_t NO_ROUTE = 0xFF;
 #ifndef TS_K3_THREADS
-#define TS_K3_THREADS 256
+#define TS_K3_THREADS 128
 #endif
 constexpr int K3_THREADS = TS_K3_THREADS;   // threads per CTA of the warp-segment K3 kernels
 constexpr int K3_WARPS = K3_THREADS / 32;

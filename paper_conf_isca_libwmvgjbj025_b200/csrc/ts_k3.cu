@@ -155,6 +155,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 #ifdef TS_WATCHDOG
     unsigned int wd_iter = 0;
 #endif
+#ifdef TS_PROF
+    long long pf_ff = 0, pf_t0 = 0;
+    unsigned int pf_gen = 0, pf_entries = 0;
+#endif
     int K = 0;
     double cS = 0.0, chunk = 0.0;
     // ---- per-lane state ----
@@ -207,6 +211,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 exhausted = true;
             } else {
                 fresh = have = true;
+#ifdef TS_PROF
+                pf_ff = 0; pf_gen = 0; pf_entries = 0; pf_t0 = clock64();
+#endif
 #ifdef TS_WATCHDOG
                 wd_iter = 0;
 #endif
@@ -345,6 +352,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
         // general pass below (R13-R19) -- only without its warp-wide votes.  The collective's last
         // delivery, a zero-length drain / latency and any instant at or after t_c go to the
         // general pass.
+#ifdef TS_PROF
+        const long long pf_a = clock64();
+#endif
         if constexpr (COLL) {
             if (__any_sync(FULL, have && running && ring_ff && !tree_cur)) {
                 const double tc = seg_min_shfl<W>(used && cst == CS_RUN ? t_end : dinf());
@@ -355,51 +365,97 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 const bool allok = (__ballot_sync(FULL, okl) & smask) == smask;   // (every lane votes)
                 const bool ok = allok && have && running && ring_ff && !tree_cur && chunk > 0.0 && Dseg < K && t < tc;
                 if (ok) {
+#ifdef TS_PROF
+                    pf_entries++;
+#endif
                     const double x = chunk / rbw0;  // = rem / rate at activation (rem = chunk, rate = rbw)
-                    bool actv = true;               // the instant at t activates step D
-                    int Dseg_l = Dseg;              // steps delivered so far (segment-uniform)
-                    for (;;) {
-                        if (actv) {
-                            const double td = t + x;
-                            if (!(t < tc) || !(td > t)) break;
-                            if (used) {
-                                EV(EV_ACTIVATE, fcode);
+                    const uint64_t cbase = ((uint64_t)cur << 32) | (uint64_t)li;
+                    int Dl = Dseg;                  // steps delivered so far; the flow in flight is step Dl
+                    int lastk = -1;                 // kind of the last processed instant: 0 activation, 1 delivery
+                    double tl = t;                  // ... and its time
+                    bool go = true;
+                    // blocks of up to four steps (eight instants): first the instant times (a short
+                    // dependent chain of adds), then their hash terms, which are independent of each other
+                    while (go) {
+                        double ti[8];
+                        int n = 0;
+                        const int D0 = Dl;
+#pragma unroll
+                        for (int i = 0; i < 8; i++) {
+                            if (go) {
+                                if ((i & 1) == 0) {   // activation of step Dl: drain at t + x
+                                    const double td = t + x;
+                                    if (t < tc && td > t) {
+                                        ti[i] = tl = t;
+                                        lastk = 0;
+                                        n = i + 1;
+                                        t = tc < td ? tc : td;   // next instant: the drain, or a compute completion first
+                                    } else {
+                                        go = false;
+                                    }
+                                } else {              // delivery of step Dl, release of step Dl + 1 (not the last)
+                                    const double ta = t + L0;
+                                    if (t < tc && Dl + 1 < K && ta > t) {
+                                        ti[i] = tl = t;
+                                        lastk = 1;
+                                        n = i + 1;
+                                        Dl++;
+                                        t = tc < ta ? tc : ta;
+                                    } else {
+                                        go = false;
+                                    }
+                                }
+                            }
+                        }
+                        if (used) {
+#pragma unroll
+                            for (int i = 0; i < 8; i++)
+                                if (i < n) {
+                                    const uint64_t m = mix64((uint64_t)__double_as_longlong(ti[i]));
+                                    const uint64_t k = (uint64_t)(D0 + (i >> 1));
+                                    if ((i & 1) == 0) {
+                                        acc += emix(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
+                                    } else {
+                                        acc += emix(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16)));
+                                        acc += emix(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
+                                    }
+                                }
+                            alg += 2u * (uint32_t)((n + 1) >> 1) + (uint32_t)(n >> 1);
+                            nflow += (uint32_t)(n >> 1);
+                        }
+                        nrounds += (uint32_t)((n + 1) >> 1);
+                        nwf += (uint32_t)n;
+                        ninst += (uint32_t)n;
+                        go = go && n == 8;
+                    }
+                    if (lastk >= 0) {
+                        maxact = (uint32_t)p > maxact ? (uint32_t)p : maxact;
+                        if (used) {
+                            if (Dl != Dseg) {
+                                D = Dl;
+                                fcode = cbase | ((uint64_t)Dl << 16);
+                            }
+                            if (lastk == 0) {   // the step in flight is active, draining
                                 fst = FS_ACT;
                                 rem = chunk;
-                                t_upd = t;
+                                t_upd = tl;
                                 rate = rbw;
-                                t_drain = td;
-                                alg += 2;
-                            }
-                            nrounds++;
-                            if ((uint32_t)p > maxact) maxact = (uint32_t)p;
-                            t = tc < td ? tc : td;   // next instant: the drain, or a compute completion first
-                        } else {
-                            const double ta = t + L0;
-                            if (!(t < tc) || Dseg_l + 1 >= K || !(ta > t)) break;
-                            if (used) {
-                                EV(EV_DELIVER, fcode);
-                                nflow++;
-                                D = Dseg_l + 1;
-                                fcode = ((uint64_t)cur << 32) | ((uint64_t)D << 16) | (uint64_t)li;
-                                EV(EV_RELEASE, fcode);
+                                t_drain = tl + x;
+                            } else {            // the next step was released and is latent
                                 fst = FS_LAT;
-                                t_act = ta;
-                                alg += 1;
+                                t_act = tl + L0;
                             }
-                            Dseg_l++;
-                            t = tc < ta ? tc : ta;
                         }
-                        actv = !actv;
-                        nwf++;
-                        ninst++;
-                        nev = false;
                         tmix = mix64((uint64_t)__double_as_longlong(t));
                     }
                 }
             }
         }
 
+#ifdef TS_PROF
+        pf_ff += clock64() - pf_a;
+        if (have) pf_gen++;
+#endif
         // ------------------------------ one instant at time t ------------------------------
         bool dirty = false;
         for (;;) {
@@ -814,6 +870,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 r.max_active_flows = fin ? maxact : 0;
                 a.out[pidx] = r;
                 if (a.alg_ops) atomicAdd(a.alg_ops, alg_s);
+#ifdef TS_PROF
+                if (pidx < 4) printf("PROF pidx=%u W=%d inst=%u general=%u ff_entries=%u ff_cycles=%lld total_cycles=%lld\n",
+                                     pidx, W, ninst, pf_gen, pf_entries, pf_ff, clock64() - pf_t0);
+#endif
             }
             if (fin || stuck) have = used = false;
         }
