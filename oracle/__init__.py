@@ -44,7 +44,7 @@ def lib():
             P = C.c_void_p
             u32, i32, i64, f64 = C.c_uint32, C.c_int32, C.c_int64, C.c_double
             L.oracle_run_point.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P, P, P,
-                                           P, P]
+                                           P, P, P, i64, P, i64, P, P]
             L.oracle_run_point.restype = C.c_int
             L.oracle_export_graph.argtypes = [P, u32, P, u32, P, u32, u32, u32, u32, P, u32, P, P, u32, C.c_int, P,
                                               P, P, P, P, P, P, P, P, P, P, P, P, P]
@@ -90,9 +90,12 @@ class OracleError(RuntimeError):
     pass
 
 
-def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None, breakdown=False):
+def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None, breakdown=False, timeline=False):
     """Simulate one design point; returns a RESULT_DTYPE record (and, with breakdown=True, the
-    per-layer compute and communication times of DESIGN.md R22)."""
+    per-layer compute and communication times of DESIGN.md R22; with timeline=True, the R23 task
+    and flow records, TASK_REC_DTYPE ordered by (gpu, prog) and FLOW_REC_DTYPE by (release, code))."""
+    if timeline:
+        return _run_point_timeline(tr, topo, pt, plan)
     k1, ta = _trace_args(tr)
     k2, tpa = _topo_args(topo)
     pl = None if plan is None else np.ascontiguousarray(plan, np.uint32)
@@ -103,12 +106,35 @@ def run_point(tr: W.Trace, topo: W.Topology, pt, plan=None, breakdown=False):
     if breakdown:
         lc, lm = np.zeros(max(tr.n_layers, 1)), np.zeros(max(tr.n_layers, 1))
     rc = lib().oracle_run_point(*ta, *tpa, _p(pl), 0 if pl is None else len(pl), 0 if pl is None else 1, _p(ptv),
-                                _p(out), _p(ph), _p(lc), _p(lm))
+                                _p(out), _p(ph), _p(lc), _p(lm), None, 0, None, 0, None, None)
     if rc != 0:
         raise OracleError(f"oracle_run_point rc={rc}")
     if breakdown:
         return out[0], lc[:tr.n_layers], lm[:tr.n_layers]
     return out[0]
+
+
+def _run_point_timeline(tr, topo, pt, plan):
+    k1, ta = _trace_args(tr)
+    k2, tpa = _topo_args(topo)
+    pl = None if plan is None else np.ascontiguousarray(plan, np.uint32)
+    ptv = np.array(pt, W.POINT_DTYPE).reshape(1)
+    ph = _phot(topo)
+    nt, nf = C.c_int64(), C.c_int64()
+    tasks = np.zeros(0, W.TASK_REC_DTYPE)
+    flows = np.zeros(0, W.FLOW_REC_DTYPE)
+    for _ in range(2):   # first call sizes the record arrays, the second fills them
+        out = np.zeros(1, W.RESULT_DTYPE)
+        rc = lib().oracle_run_point(*ta, *tpa, _p(pl), 0 if pl is None else len(pl), 0 if pl is None else 1, _p(ptv),
+                                    _p(out), _p(ph), None, None, _p(tasks), len(tasks), _p(flows), len(flows),
+                                    C.byref(nt), C.byref(nf))
+        if rc != 0:
+            raise OracleError(f"oracle_run_point rc={rc}")
+        if nt.value <= len(tasks) and nf.value <= len(flows):
+            return out[0], tasks[:nt.value], flows[:nf.value]
+        tasks = np.zeros(nt.value, W.TASK_REC_DTYPE)
+        flows = np.zeros(nf.value, W.FLOW_REC_DTYPE)
+    raise OracleError("timeline sizes changed between calls")
 
 
 def run_sweep(sw: W.Sweep, idx=None, breakdown=False):

@@ -239,6 +239,7 @@ typedef struct {
     uint64_t code;    /* canonical id for the order hash */
     int flags;
     int layer;        /* task: its operator's layer (R22 breakdown); -1 otherwise */
+    int op, mb;       /* task: trace operator and micro-batch (R23 timeline) */
 } GNode;
 
 typedef struct {
@@ -277,9 +278,9 @@ static void g_free(Graph *G) {
 static void g_record(Graph *G, int start, int end, int layer, int cat) {
     iv_push(&G->rc_s, start); iv_push(&G->rc_e, end); iv_push(&G->rc_l, layer); iv_push(&G->rc_c, cat);
 }
-static int add_task(Graph *G, int gpu, long prog, double dur, int layer) {
+static int add_task(Graph *G, int gpu, long prog, double dur, int layer, int op, int mb) {
     GNode n; memset(&n, 0, sizeof n);
-    n.type = N_TASK; n.gpu = gpu; n.dur = dur; n.layer = layer;
+    n.type = N_TASK; n.gpu = gpu; n.dur = dur; n.layer = layer; n.op = op; n.mb = mb;
     n.code = ((uint64_t)(uint32_t)gpu << 40) | (uint64_t)prog;
     return g_add(G, n);
 }
@@ -581,7 +582,7 @@ static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
     /* every rank duplicates every operator */
     for (int r = 0; r < dp; r++)
         for (uint32_t o = 0; o < N; o++)
-            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer);
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer, (int)o, 0);
     if (dp > 1) {
         /* weight gradients in production order (reading Q4: produced by the backward pass) */
         WEnt *w = (WEnt *)malloc(sizeof(WEnt) * (T->n_ts ? T->n_ts : 1));
@@ -642,7 +643,7 @@ static int expand_tp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
     if (!task) return -1;
     for (int r = 0; r < tp; r++)
         for (uint32_t o = 0; o < N; o++)
-            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, tp, pt->tp_mode), (int)T->ops[o].layer);
+            task[(size_t)r * N + o] = add_task(G, ro[r], o, op_time(T, o, r_b, tp, pt->tp_mode), (int)T->ops[o].layer, (int)o, 0);
     if (tp > 1) {
         int *done_of = (int *)malloc(sizeof(int) * (size_t)(T->n_ts ? T->n_ts : 1) * (size_t)tp);
         char *has = (char *)calloc(T->n_ts ? T->n_ts : 1, 1);
@@ -740,7 +741,7 @@ static int expand_pp(const Trace *T, const OPoint *pt, const int *ro, const uint
         int prev_send = -1;
         for (long q = 0; q < np; q++) {
             int o = prog_op[q], j = prog_mb[q];
-            int t = add_task(G, ro[s], q, op_time(T, (uint32_t)o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer);
+            int t = add_task(G, ro[s], q, op_time(T, (uint32_t)o, r_b, 1, pt->tp_mode), (int)T->ops[o].layer, o, j);
             inst[(size_t)o * m + j] = t;
             /* "send its output data to the next GPU. Simultaneously ... the next micro-batch"
              * (P:190): push every produced tensor to each other stage that reads it, FIFO per
@@ -879,7 +880,7 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
         if (!task[r]) goto out;
         for (long q = 0; q < plen[s]; q++)
             task[r][q] = add_task(G, ro[r], q, op_time(T, (uint32_t)pop[s][q], r_b, tp, pt->tp_mode),
-                                  (int)T->ops[pop[s][q]].layer);
+                                  (int)T->ops[pop[s][q]].layer, pop[s][q], pmb[s][q]);
     }
     /* TP collectives: per group (d, s), one per (op, output, micro-batch) instance in program order */
     if (tp > 1) {
@@ -1111,7 +1112,7 @@ static uint64_t dbits(double d) { uint64_t u; memcpy(&u, &d, 8); return u; }
 enum { S_WAIT = 0, S_QUEUED = 1, S_RUN = 2, S_LATENT = 3, S_ACTIVE = 4, S_DONE = 5 };
 
 static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale, OResult *res, double *t_done,
-                    double *l_comp, double *l_comm) {
+                    double *l_comp, double *l_comm, double *tl_s, double *tl_a) {
     long NN = G->count;
     const int bd = l_comp != NULL && G->want_bd;
     double *td_own = NULL, *t_rel = NULL;
@@ -1332,6 +1333,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         if (t_act[f] == t) {
                             latent.v[a] = latent.v[--latent.n];
                             EVENT(EV_ACTIVATE, G->n[f].code);
+                            if (tl_a) tl_a[f] = t;
                             if (G->n[f].bytes == 0.0 || frlen[f] == 0) {
                                 COMPLETE(f);
                                 EVENT(EV_DELIVER, G->n[f].code);
@@ -1356,10 +1358,12 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         } else if (ph) {
                             /* R20: a send request; t_act holds its release time (the FIFO key) */
                             if (t_rel) t_rel[k] = t;
+                            if (tl_s) tl_s[k] = t;
                             EVENT(EV_RELEASE, G->n[k].code);
                             inflight++;
                             if (G->n[k].src == G->n[k].dst) {
                                 EVENT(EV_ACTIVATE, G->n[k].code);
+                                if (tl_a) tl_a[k] = t;
                                 COMPLETE(k);
                                 EVENT(EV_DELIVER, G->n[k].code);
                                 inflight--;
@@ -1373,6 +1377,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                             state[k] = S_LATENT;
                             t_act[k] = t + lat[k];
                             if (t_rel) t_rel[k] = t;
+                            if (tl_s) tl_s[k] = t;
                             EVENT(EV_RELEASE, G->n[k].code);
                             iv_push(&latent, k);
                             inflight++;
@@ -1387,6 +1392,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                         running[g] = k; head[g]++;
                         state[k] = S_RUN;
                         t_end[k] = t + G->n[k].dur;
+                        if (tl_s) tl_s[k] = t;
                         if (doff[k + 1] > doff[k]) EVENT(EV_TASK_START, G->n[k].code);
                         changed = 1;
                     }
@@ -1468,6 +1474,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                             ph_st[f] = PS_XFER;
                             t_drain[f] = (t + ph_lat) + G->n[f].bytes / ph_bw;
                             EVENT(EV_ACTIVATE, G->n[f].code);
+                            if (tl_a) tl_a[f] = t;
                             if (t_drain[f] == t) again = 1;
                         }
                     }
@@ -1608,11 +1615,29 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
     return rc;
 }
 
+/* R23 timeline records: every compute task (its simulated GPU, program position, trace operator,
+ * micro-batch, start and end) and every flow (code, endpoints, bytes, release, activation -- the
+ * photonic grant --, delivery), tasks ordered by (gpu, prog), flows by (release, code) */
+typedef struct { uint32_t gpu, prog, op, mb; double start, end; } OTaskRec;
+typedef struct { uint64_t code; uint32_t src, dst; double bytes, release, start, delivered; } OFlowRec;
+
+static int task_cmp(const void *a, const void *b) {
+    const OTaskRec *x = (const OTaskRec *)a, *y = (const OTaskRec *)b;
+    if (x->gpu != y->gpu) return x->gpu < y->gpu ? -1 : 1;
+    return x->prog < y->prog ? -1 : x->prog > y->prog;
+}
+static int flow_cmp(const void *a, const void *b) {
+    const OFlowRec *x = (const OFlowRec *)a, *y = (const OFlowRec *)b;
+    if (x->release != y->release) return x->release < y->release ? -1 : 1;
+    return x->code < y->code ? -1 : x->code > y->code;
+}
+
 int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t n_ts, const uint32_t *io,
                      uint32_t n_io, uint32_t trace_batch, uint32_t n_nodes, uint32_t n_gpus, const OLink *links,
                      uint32_t n_links, const uint32_t *ring_order, const uint32_t *plan, uint32_t plan_len,
                      int have_plan, const OPoint *pt, OResult *out, const OPhot *ph, double *l_comp,
-                     double *l_comm) {
+                     double *l_comm, OTaskRec *tasks, int64_t task_cap, OFlowRec *flows, int64_t flow_cap,
+                     int64_t *n_tasks, int64_t *n_flows) {
     Trace T = {ops, n_ops, ts, n_ts, io, n_io, trace_batch, NULL, 0};
     Topo tp; memset(&tp, 0, sizeof tp);
     int rc = trace_check(&T);
@@ -1629,9 +1654,49 @@ int oracle_run_point(const OOp *ops, uint32_t n_ops, const OTensor *ts, uint32_t
     int status = PT_OK;
     memset(out, 0, sizeof *out);
     if (l_comp) for (uint32_t l = 0; l < T.n_layers; l++) l_comp[l] = l_comm[l] = 0.0;
+    if (n_tasks && n_flows) *n_tasks = *n_flows = 0;
     if (build_graph(&T, &tp, ring_order, plan, plan_len, have_plan, pt, &G, &status)) rc = O_ENOMEM;
     else if (status != PT_OK) out->status = status;
-    else if (simulate(&G, &tp, pt->bw_scale, pt->lat_scale, out, NULL, l_comp, l_comm)) rc = O_ENOMEM;
+    else {
+        double *t_done = NULL, *tl_s = NULL, *tl_a = NULL;
+        const int tl = n_tasks != NULL && n_flows != NULL;
+        if (tl) {
+            const size_t nn = (size_t)(G.count ? G.count : 1);
+            t_done = (double *)calloc(nn, sizeof(double));
+            tl_s = (double *)calloc(nn, sizeof(double));
+            tl_a = (double *)calloc(nn, sizeof(double));
+            if (!t_done || !tl_s || !tl_a) rc = O_ENOMEM;
+        }
+        if (rc == O_OK && simulate(&G, &tp, pt->bw_scale, pt->lat_scale, out, t_done, l_comp, l_comm, tl_s, tl_a))
+            rc = O_ENOMEM;
+        if (rc == O_OK && tl && out->status == PT_OK) {
+            int64_t nt = 0, nf = 0;
+            for (long i = 0; i < G.count; i++) {
+                const GNode *nd = &G.n[i];
+                if (nd->type == N_TASK) {
+                    if (tasks && nt < task_cap) {
+                        OTaskRec r = {(uint32_t)nd->gpu, (uint32_t)(nd->code & ((1ull << 40) - 1)), (uint32_t)nd->op,
+                                      (uint32_t)nd->mb, tl_s[i], t_done[i]};
+                        tasks[nt] = r;
+                    }
+                    nt++;
+                } else if (nd->type == N_FLOW) {
+                    if (flows && nf < flow_cap) {
+                        OFlowRec r = {nd->code, (uint32_t)nd->src, (uint32_t)nd->dst, nd->bytes, tl_s[i], tl_a[i], t_done[i]};
+                        flows[nf] = r;
+                    }
+                    nf++;
+                }
+            }
+            if (tasks && nt <= task_cap) qsort(tasks, (size_t)nt, sizeof(OTaskRec), task_cmp);
+            if (flows && nf <= flow_cap) qsort(flows, (size_t)nf, sizeof(OFlowRec), flow_cmp);
+            *n_tasks = nt;
+            *n_flows = nf;
+        } else if (tl) {
+            *n_tasks = *n_flows = 0;
+        }
+        free(t_done); free(tl_s); free(tl_a);
+    }
     g_free(&G); free(T.prod); topo_free(&tp);
     return rc;
 }
@@ -1700,7 +1765,7 @@ int oracle_sim_graph(int64_t n, const int32_t *type, const int32_t *gpu, const d
     }
     G.n_coll = n_coll;
     G.coll_payload = coll_payload;
-    if (rc == O_OK && simulate(&G, &tp, bw_scale, lat_scale, out, t_done, NULL, NULL)) rc = O_ENOMEM;
+    if (rc == O_OK && simulate(&G, &tp, bw_scale, lat_scale, out, t_done, NULL, NULL, NULL, NULL)) rc = O_ENOMEM;
     g_free(&G); topo_free(&tp);
     return rc;
 }

@@ -47,6 +47,12 @@ RESULT_DTYPE = np.dtype([
     ("n_compute", "<u8"), ("n_flows", "<u8"), ("n_collectives", "<u8"), ("n_p2p", "<u8"),
     ("n_instants", "<u8"), ("n_wf_calls", "<u8"), ("n_wf_rounds", "<u8"), ("order_hash", "<u8"),
     ("status", "<i4"), ("max_active_flows", "<u4")])
+# R23 timeline records (include/triosim.h triosim_task_rec / triosim_flow_rec)
+TASK_REC_DTYPE = np.dtype([("gpu", "<u4"), ("prog", "<u4"), ("op", "<u4"), ("mb", "<u4"), ("start_s", "<f8"),
+                           ("end_s", "<f8")])
+FLOW_REC_DTYPE = np.dtype([("code", "<u8"), ("src", "<u4"), ("dst", "<u4"), ("bytes", "<f8"), ("release_s", "<f8"),
+                           ("start_s", "<f8"), ("delivered_s", "<f8")])
+assert TASK_REC_DTYPE.itemsize == 32 and FLOW_REC_DTYPE.itemsize == 48
 assert OP_DTYPE.itemsize == 40 and TENSOR_DTYPE.itemsize == 16 and LINK_DTYPE.itemsize == 24
 assert POINT_DTYPE.itemsize == 56 and RESULT_DTYPE.itemsize == 112
 
