@@ -71,10 +71,18 @@ typedef struct {
     uint16_t dp, tp, pp, pad1;
     uint32_t microbatches, global_batch;
     int32_t stage_plan;
-    uint32_t pad2;
+    uint32_t first_bucket_bytes;   /* R24: cap of a group's first gradient bucket, 0 = bucket_bytes */
     uint64_t bucket_bytes;
     double bw_scale, lat_scale;
 } OPoint; /* 56 B */
+
+/* R24 (PyTorch DDP's first-bucket rule): the cap of bucket number k of a gradient group -- the first
+ * bucket closes at first_bucket_bytes when that is set, every later one at bucket_bytes; bucket_bytes
+ * == 0 keeps one tensor per AllReduce (the paper-literal reading of Q5) */
+static uint64_t bucket_cap(const OPoint *pt, int k) {
+    if (pt->bucket_bytes == 0) return 0;
+    return (k == 0 && pt->first_bucket_bytes != 0) ? (uint64_t)pt->first_bucket_bytes : pt->bucket_bytes;
+}
 
 typedef struct {
     double iter_time_s, compute_busy_max_s, comm_busy_s, exposed_comm_s, coll_payload_bytes;
@@ -599,10 +607,11 @@ static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
         int *trig = (int *)malloc(sizeof(int) * (size_t)dp), *prev = (int *)malloc(sizeof(int) * (size_t)dp),
             *done = (int *)malloc(sizeof(int) * (size_t)dp);
         int have_prev = 0;
-        int i = 0;
+        int i = 0, nb = 0;
         while (i < nw) {
             /* bucket (reading Q5): bucket_bytes == 0 -> one tensor per AllReduce (paper-literal);
-             * else greedy: close the bucket once its u64 byte sum reaches bucket_bytes */
+             * else greedy: close the bucket once its u64 byte sum reaches its cap (R24) */
+            const uint64_t cap = bucket_cap(pt, nb++);
             int j = i;
             uint64_t sum = 0;
             double S = 0.0;
@@ -610,7 +619,7 @@ static int expand_dp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
                 sum += T->ts[w[j].x].bytes_b0;
                 S = S + tensor_bytes(T, w[j].x, r_b, 1, pt->tp_mode);
                 j++;
-                if (pt->bucket_bytes == 0 || sum >= pt->bucket_bytes || j == nw) break;
+                if (cap == 0 || sum >= cap || j == nw) break;
             }
             /* DDP: AllReduce parallel with backward, triggered by the op producing the bucket's
              * last gradient; DP (DataParallel): after the backward pass (reading Q6) */
@@ -994,8 +1003,9 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                 for (int d = 0; d < dp; d++) members[d] = ro[(d * S + s) * tp + t];
                 int have_prev = 0;
                 uint64_t seq = 0;
-                int i = 0;
+                int i = 0, nb = 0;
                 while (i < nw) {
+                    const uint64_t cap = bucket_cap(pt, nb++);   /* R24, per stage's DP group */
                     int j = i;
                     uint64_t sum = 0;
                     double Sb = 0.0;
@@ -1003,7 +1013,7 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                         sum += T->ts[w[j].x].bytes_b0;
                         Sb = Sb + tensor_bytes(T, w[j].x, r_b, tp, pt->tp_mode);
                         j++;
-                        if (pt->bucket_bytes == 0 || sum >= pt->bucket_bytes || j == nw) break;
+                        if (cap == 0 || sum >= cap || j == nw) break;
                     }
                     /* program position of (producer of the bucket's last gradient, micro-batch 0) */
                     long qt = -1;

@@ -342,3 +342,70 @@ def test_cf13_comm_bound_is_not_the_formula():
     r = oracle.run_point(tr, W.ring(3, bw=B, lat=a), W.make_point(0, W.ST_PP, pp=3, m=4, B=4))
     c = a + A / B
     assert r["iter_time_s"] > (4 + 2) * (t_f + t_b) + 2 * 2 * c + 1e-9
+
+
+# ---------------- R24: DDP first-bucket rule ----------------
+def _buckets(sizes, first, cap):
+    """Plain greedy bucketing of gradient sizes in production order (R24 restated)."""
+    out, cur, tot = [], [], 0
+    for s in sizes:
+        cur.append(s)
+        tot += s
+        lim = first if (not out and first) else cap
+        if tot >= lim:
+            out.append(cur)
+            cur, tot = [], 0
+    if cur:
+        out.append(cur)
+    return out
+
+
+def _wgrad_sizes(tr):
+    prod = {}
+    for o, op in enumerate(tr.ops):
+        for k in range(int(op["n_out"])):
+            prod[int(tr.io[op["io_off"] + op["n_in"] + k])] = o
+    xs = [x for x in range(len(tr.tensors)) if tr.tensors[x]["category"] == W.CAT_WGRAD and x in prod
+          and tr.ops[prod[x]]["phase"] != W.PH_OPT]
+    xs.sort(key=lambda x: (prod[x], x))
+    return [int(tr.tensors[x]["bytes_b0"]) for x in xs]
+
+
+@pytest.mark.parametrize("first,cap", [(1, 25 << 20), (1 << 20, 25 << 20), (4 << 20, 1 << 20), (1, 1)])
+def test_r24_first_bucket_counts_and_payload(first, cap):
+    """PyTorch DDP caps the first gradient bucket separately (1 MiB by default, later ones 25 MiB): the
+    number of AllReduces is the greedy bucket count with the first cap, and the payload is unchanged."""
+    tr = W.resnet50_trace()
+    sizes = _wgrad_sizes(tr)
+    exp = _buckets(sizes, first, cap)
+    r = oracle.run_point(tr, W.ring(4), W.make_point(0, W.ST_DDP, dp=4, B=4 * tr.trace_batch, bucket=cap,
+                                                     first_bucket=first))
+    assert r["status"] == 0 and r["n_collectives"] == len(exp)
+    assert r["coll_payload_bytes"] == float(sum(sizes))
+    if first == 1:
+        assert len(exp[0]) == 1
+
+
+@pytest.mark.parametrize("st", [W.ST_DP, W.ST_DDP, W.ST_HYBRID])
+def test_r24_first_bucket_equal_to_cap_or_per_tensor_is_the_plain_rule(st):
+    """first_bucket_bytes == bucket_bytes, or bucket_bytes == 0 (one tensor per AllReduce), reproduce the
+    rule without a first cap bit for bit, order hash included."""
+    tr = W.resnet50_trace()
+    topo = W.ring(8, 50e9, 2e-6)
+    kw = dict(dp=4, B=4 * tr.trace_batch) if st != W.ST_HYBRID else dict(dp=2, tp=2, pp=2, m=2, B=4 * tr.trace_batch)
+    for cap, first in ((25 << 20, 25 << 20), (0, 1 << 20)):
+        a = oracle.run_point(tr, topo, W.make_point(0, st, bucket=cap, **kw))
+        b = oracle.run_point(tr, topo, W.make_point(0, st, bucket=cap, first_bucket=first, **kw))
+        assert a.tobytes() == b.tobytes()
+
+
+def test_r24_small_first_bucket_starts_communication_earlier():
+    """A small first bucket launches its AllReduce as soon as its few gradients exist, so on a fast link
+    the iteration is not slower and the first collective starts before the 25 MiB-only case's."""
+    tr = W.resnet50_trace()
+    topo = W.ring(4, 100e9, 1e-6)
+    a, ta, fa = oracle.run_point(tr, topo, W.make_point(0, W.ST_DDP, dp=4, B=256, bucket=25 << 20), timeline=True)
+    b, tb, fb = oracle.run_point(tr, topo, W.make_point(0, W.ST_DDP, dp=4, B=256, bucket=25 << 20,
+                                                        first_bucket=1 << 20), timeline=True)
+    assert fb["release_s"].min() < fa["release_s"].min()
+    assert b["n_collectives"] >= a["n_collectives"]
