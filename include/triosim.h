@@ -157,8 +157,9 @@ typedef struct {
     uint16_t dp, tp, pp, pad1;
     uint32_t microbatches, global_batch;
     int32_t stage_plan;      /* -1 = automatic balanced partition */
-    uint32_t pad2;
-    uint64_t bucket_bytes;   /* DP/DDP gradient bucket; 0 = one AllReduce per tensor */
+    uint32_t first_bucket_bytes;  /* cap of each gradient group's first bucket (PyTorch DDP's first-bucket
+                                     rule, R24); 0 = bucket_bytes; ignored when bucket_bytes == 0 */
+    uint64_t bucket_bytes;   /* DP/DDP/HYBRID gradient bucket; 0 = one AllReduce per tensor */
     double bw_scale;         /* multiplies every link bandwidth (> 0) */
     double lat_scale;        /* multiplies every link latency (>= 0) */
 } triosim_point;             /* 56 B */
@@ -175,6 +176,26 @@ typedef struct {
     uint32_t max_active_flows;
 } triosim_result;                /* 112 B */
 
+/* Timeline records (R23; "the timeline of the communication process among GPUs or the
+ * computation process on each GPU").  A task is one operator instance on one simulated GPU; a
+ * flow is one ring / tree step, P2P send or photonic transfer. */
+typedef struct {
+    uint32_t gpu;        /* simulated GPU (topology node id) */
+    uint32_t prog;       /* position in that GPU's program (micro-batch instances included) */
+    uint32_t op;         /* trace operator */
+    uint32_t mb;         /* micro-batch (0 outside GPipe / HYBRID) */
+    double start_s, end_s;
+} triosim_task_rec;      /* 32 B */
+typedef struct {
+    uint64_t code;       /* the flow's order-hash code (R19): collective (c<<32 | step<<16 | member, tree
+                            broadcast edges step = 1), P2P (1<<59 | tensor<<32 | micro-batch<<16 | dst) */
+    uint32_t src, dst;   /* GPU node ids */
+    double bytes;
+    double release_s;    /* dependencies met (R10, R11) */
+    double start_s;      /* activation after the route latency (R13) / photonic buffer grant (R20) */
+    double delivered_s;
+} triosim_flow_rec;      /* 48 B */
+
 #ifdef __cplusplus
 static_assert(sizeof(triosim_op) == 40, "op");
 static_assert(sizeof(triosim_tensor) == 16, "tensor");
@@ -182,6 +203,8 @@ static_assert(sizeof(triosim_link) == 24, "link");
 static_assert(sizeof(triosim_point) == 56, "point");
 static_assert(sizeof(triosim_photonic) == 32, "photonic");
 static_assert(sizeof(triosim_result) == 112, "result");
+static_assert(sizeof(triosim_task_rec) == 32, "task rec");
+static_assert(sizeof(triosim_flow_rec) == 48, "flow rec");
 #endif
 
 typedef struct triosim_ctx triosim_ctx;
@@ -252,6 +275,17 @@ triosim_status triosim_set_breakdown(triosim_ctx *ctx, int32_t sweep_id, int ena
 triosim_status triosim_breakdown(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
                                  double *layer_compute_s, double *layer_comm_s, int out_is_device,
                                  void *cuda_stream);
+
+/* Timeline of one design point (R23): runs the path for point `point` of sweep_id alone with a
+ * recording instantiation of the timeline kernel (same results, bit for bit; the point's result record
+ * is rewritten with them), then sorts the records on the device: tasks by (gpu, prog), flows by
+ * (release_s, code).  *n_tasks / *n_flows receive the totals (= the result's n_compute / n_flows); at
+ * most task_cap / flow_cap records are written to the caller-owned host arrays, and only when the
+ * totals fit are they the complete sorted timeline (call again with larger arrays otherwise).  A point
+ * whose status is not OK has no records.  Synchronous.  Errors: EINVAL, ENOTFOUND, ERANGE, ENOMEM, ECUDA. */
+triosim_status triosim_timeline(triosim_ctx *ctx, int32_t sweep_id, uint64_t point, triosim_task_rec *tasks,
+                                uint64_t task_cap, triosim_flow_rec *flows, uint64_t flow_cap, uint64_t *n_tasks,
+                                uint64_t *n_flows);
 
 /* Kernel launch counters since the context was created (K1, K2, K3 launches), for the bench. */
 triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3);

@@ -8,7 +8,7 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
-SRC = [os.path.join(HERE, "csrc", f) for f in ("ts_host.cu", "ts_kernels.cu", "ts_k3.cu", "ts_k3h.cu")]
+SRC = [os.path.join(HERE, "csrc", f) for f in ("ts_host.cu", "ts_kernels.cu", "ts_k3.cu", "ts_k3h.cu", "ts_timeline.cu")]
 HDR = [os.path.join(HERE, "csrc", "ts_internal.h"), os.path.join(ROOT, "include", "triosim.h")]
 OUT = os.environ.get("TS_BUILD_OUT", os.path.join(HERE, "libtriosim.so"))   # override: A/B variants
 OBJ = os.path.join(HERE, "csrc", "build")

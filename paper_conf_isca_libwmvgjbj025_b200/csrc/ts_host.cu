@@ -108,6 +108,11 @@ struct Sweep {
     // communication accumulators, staging for host-bound copies
     bool bd = false;
     DevBuf<double> d_lcomp, d_bd_acc, d_bd_stage;
+    // R23 timeline of one point (triosim_timeline)
+    DevBuf<triosim_task_rec> d_tl_tasks;
+    DevBuf<triosim_flow_rec> d_tl_flows;
+    DevBuf<unsigned long long> d_tl_cnt;
+    DevBuf<uint32_t> d_one;
 };
 
 int w_index(int W) { int i = 0; while ((2 << i) < W) i++; return i; }
@@ -442,7 +447,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     S->cost.assign(n_pts, 0.0);
     S->mode.assign(n_pts, 0);
     std::vector<PointDesc> pdesc(n_pts);
-    std::map<std::tuple<int, int, int, int, int, int, int, uint64_t, int, int>, uint32_t> cls_of;
+    std::map<std::tuple<int, int, int, int, int, int, int, uint64_t, uint32_t, int, int>, uint32_t> cls_of;
     std::vector<uint32_t> plan_pool;
     const uint32_t N = (uint32_t)T.ops.size(), NT = (uint32_t)T.ts.size();
 
@@ -532,9 +537,10 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         int key_mode = (pt.strategy == TRIOSIM_TP || hyb) ? pt.tp_mode : 0;
         int key_algo = mode != MODE_PIPE ? pt.coll_algo : 0;
         uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP || hyb) ? pt.bucket_bytes : 0;
+        uint32_t key_first = key_bucket ? pt.first_bucket_bytes : 0;   // R24
         int key_m = (mode == MODE_PIPE || hyb) ? (int)mbe : 0;
         auto key = std::make_tuple((int)pt.strategy + (dp_after ? 100 : 0), (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
-                                   hyb ? (int)tpd : 0, key_algo, key_bucket, key_m,
+                                   hyb ? (int)tpd : 0, key_algo, key_bucket, key_first, key_m,
                                    (mode == MODE_PIPE || hyb) ? plan_key : -2);
         auto ci = cls_of.find(key);
         uint32_t c;
@@ -552,6 +558,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.dp = hyb ? dp : 1;
             cd.b_loc = b_loc;
             cd.bucket_bytes = key_bucket;
+            cd.first_bucket = key_first;
             cd.r_b = (double)b_loc / (double)T.b0;
             if (mode == MODE_PIPE || hyb) {
                 if (plan_key < 0) {
@@ -739,6 +746,46 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
 // ------------------------------------------------------------------------------------------
 // simulate_batch
 // ------------------------------------------------------------------------------------------
+// K1b + K2 for every class of the sweep (cheap; part of every step)
+static cudaError_t enqueue_k1_k2(triosim_ctx *ctx, Sweep &S, Trace &T, cudaStream_t st) {
+    const uint32_t ncls = (uint32_t)S.classes.size();
+    cudaError_t e = launch_k1_rescale(S.d_cls.p, ncls, T.dev, S.d_dur.p, st);
+    if (e != cudaSuccess) return e;
+    if (ncls) ctx->n_k1++;
+    e = launch_k2_coll(S.d_cls.p, S.d_coll_list.p, (uint32_t)S.coll_list.size(), T.dev, S.d_dur.p, S.d_hooks.p,
+                       S.d_colls.p, S.d_scr_i32.p, st);
+    if (e != cudaSuccess) return e;
+    if (!S.coll_list.empty()) ctx->n_k2++;
+    e = launch_k2_pipe(S.d_cls.p, S.d_pipe_list.p, (uint32_t)S.pipe_list.size(), T.dev, S.d_dur.p, S.d_plans.p,
+                       S.d_stages.p, S.d_ents.p, S.d_sends.p, S.d_recvs.p, S.d_scr_u64.p, st);
+    if (e != cudaSuccess) return e;
+    if (!S.pipe_list.empty()) ctx->n_k2++;
+    e = launch_k2_hybrid(S.d_cls.p, S.d_hyb_list.p, (uint32_t)S.hyb_list.size(), T.dev, S.d_plans.p, S.d_stages.p,
+                         S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, st);
+    if (e != cudaSuccess) return e;
+    if (!S.hyb_list.empty()) ctx->n_k2++;
+    return cudaSuccess;
+}
+
+// K3 arguments shared by every launch group w of a sweep
+static K3Args k3_args(Sweep &S, int w) {
+    K3Args a;
+    std::memset(&a, 0, sizeof a);
+    a.counter = S.d_counter.p + w;
+    a.pts = S.d_pts.p;
+    a.cls = S.d_cls.p; a.topo = S.d_topo.p;
+    a.link_bw = S.d_bw.p; a.link_lat = S.d_lat.p; a.rt_off = S.d_rt_off.p; a.rt_len = S.d_rt_len.p;
+    a.rt_links = S.d_rt_links.p; a.ro = S.d_ro.p;
+    a.hooks = S.d_hooks.p; a.colls = S.d_colls.p; a.dur = S.d_dur.p;
+    a.stages = S.d_stages.p; a.ents = S.d_ents.p; a.sends = S.d_sends.p; a.recvs = S.d_recvs.p;
+    a.hst = S.d_hst.p; a.hents = S.d_hents.p; a.hsends = S.d_hsends.p;
+    a.out = S.d_res.p;
+    a.alg_ops = S.d_alg.p;
+    a.lmax = S.lmax[w];
+    a.pmax = S.pmax[w];
+    return a;
+}
+
 triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
                                       void *cuda_stream) {
     if (!ctx) return TRIOSIM_EINVAL;
@@ -756,18 +803,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     const uint32_t ncls = (uint32_t)S.classes.size();
     const int slot = ctx->timing ? ctx->n_timed % triosim_ctx::NT : -1;
     if (slot >= 0) CK(cudaEventRecord(ctx->t_begin[slot], st));
-    // K1b + K2 for every class of the sweep (cheap; part of every step)
-    CK(launch_k1_rescale(S.d_cls.p, ncls, T.dev, S.d_dur.p, st));
-    if (ncls) ctx->n_k1++;
-    CK(launch_k2_coll(S.d_cls.p, S.d_coll_list.p, (uint32_t)S.coll_list.size(), T.dev, S.d_dur.p, S.d_hooks.p,
-                      S.d_colls.p, S.d_scr_i32.p, st));
-    if (!S.coll_list.empty()) ctx->n_k2++;
-    CK(launch_k2_pipe(S.d_cls.p, S.d_pipe_list.p, (uint32_t)S.pipe_list.size(), T.dev, S.d_dur.p, S.d_plans.p,
-                      S.d_stages.p, S.d_ents.p, S.d_sends.p, S.d_recvs.p, S.d_scr_u64.p, st));
-    if (!S.pipe_list.empty()) ctx->n_k2++;
-    CK(launch_k2_hybrid(S.d_cls.p, S.d_hyb_list.p, (uint32_t)S.hyb_list.size(), T.dev, S.d_plans.p, S.d_stages.p,
-                        S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, st));
-    if (!S.hyb_list.empty()) ctx->n_k2++;
+    CK(enqueue_k1_k2(ctx, S, T, st));
     const uint32_t L = T.n_layers;
     if (S.bd) {
         CK(launch_k4_layer_compute(S.d_cls.p, ncls, T.dev, S.d_dur.p, S.d_stages.p, S.d_ents.p, S.d_hents.p,
@@ -794,19 +830,8 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         }
         if (n == 0) continue;
         const int W = W_OF[w / N_MODES], mode = w % N_MODES;
-        K3Args a;
-        std::memset(&a, 0, sizeof a);
-        a.pts = S.d_pts.p; a.work = wl; a.n_work = n; a.counter = S.d_counter.p + w;
-        a.cls = S.d_cls.p; a.topo = S.d_topo.p;
-        a.link_bw = S.d_bw.p; a.link_lat = S.d_lat.p; a.rt_off = S.d_rt_off.p; a.rt_len = S.d_rt_len.p;
-        a.rt_links = S.d_rt_links.p; a.ro = S.d_ro.p;
-        a.hooks = S.d_hooks.p; a.colls = S.d_colls.p; a.dur = S.d_dur.p;
-        a.stages = S.d_stages.p; a.ents = S.d_ents.p; a.sends = S.d_sends.p; a.recvs = S.d_recvs.p;
-        a.hst = S.d_hst.p; a.hents = S.d_hents.p; a.hsends = S.d_hsends.p;
-        a.out = S.d_res.p;
-        a.alg_ops = S.d_alg.p;
-        a.lmax = S.lmax[w];
-        a.pmax = S.pmax[w];
+        K3Args a = k3_args(S, w);
+        a.work = wl; a.n_work = n;
         if (S.bd) {
             a.bd = S.d_bd_acc.p;
             a.layer = T.d_layer.p;
@@ -880,6 +905,59 @@ triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t firs
         CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
     }
+    return TRIOSIM_OK;
+}
+
+triosim_status triosim_timeline(triosim_ctx *ctx, int32_t sweep_id, uint64_t point, triosim_task_rec *tasks,
+                                uint64_t task_cap, triosim_flow_rec *flows, uint64_t flow_cap, uint64_t *n_tasks,
+                                uint64_t *n_flows) {
+    if (!ctx || !n_tasks || !n_flows || (task_cap && !tasks) || (flow_cap && !flows))
+        return fail(ctx, TRIOSIM_EINVAL, "null argument");
+    CK(cudaSetDevice(ctx->device));
+    CK(cudaGetLastError());
+    auto it = ctx->sweeps.find(sweep_id);
+    if (it == ctx->sweeps.end()) return fail(ctx, TRIOSIM_ENOTFOUND, "unknown sweep %d", sweep_id);
+    Sweep &S = *it->second;
+    if (point >= S.n_pts) return fail(ctx, TRIOSIM_ERANGE, "point %llu outside sweep", (unsigned long long)point);
+    Trace &T = *ctx->traces.at(S.trace_handle);
+    *n_tasks = *n_flows = 0;
+    if (S.status[point] >= 0) return TRIOSIM_OK;   // decided on the host (R3): no timeline
+    cudaStream_t st = nullptr;
+    CK(enqueue_k1_k2(ctx, S, T, st));
+    if (S.d_tl_tasks.n < task_cap || !S.d_tl_tasks.p) CK(S.d_tl_tasks.alloc(task_cap));
+    if (S.d_tl_flows.n < flow_cap || !S.d_tl_flows.p) CK(S.d_tl_flows.alloc(flow_cap));
+    if (!S.d_tl_cnt.p) CK(S.d_tl_cnt.alloc(2));
+    if (!S.d_one.p) CK(S.d_one.alloc(1));
+    const uint32_t pi = (uint32_t)point;
+    CK(cudaMemcpyAsync(S.d_one.p, &pi, sizeof pi, cudaMemcpyHostToDevice, st));
+    CK(cudaMemsetAsync(S.d_tl_cnt.p, 0, 2 * sizeof(unsigned long long), st));
+    const int w = N_MODES * w_index(S.width[point]) + S.mode[point];
+    CK(cudaMemsetAsync(S.d_counter.p + w, 0, sizeof(unsigned int), st));
+    K3Args a = k3_args(S, w);
+    a.work = S.d_one.p;
+    a.n_work = 1;
+    a.tl_tasks = S.d_tl_tasks.p;
+    a.tl_flows = S.d_tl_flows.p;
+    a.tl_cnt = S.d_tl_cnt.p;
+    a.tl_task_cap = task_cap;
+    a.tl_flow_cap = flow_cap;
+    const int W = W_OF[w / N_MODES], mode = w % N_MODES;
+    if (mode == MODE_HYBRID) CK(launch_k3_hybrid(W, a, 1, st));
+    else CK(launch_k3(W, mode, a, 1, st));
+    ctx->n_k3++;
+    unsigned long long cnt[2] = {0, 0};
+    int32_t pst = 0;
+    CK(cudaMemcpyAsync(cnt, S.d_tl_cnt.p, sizeof cnt, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&pst, &S.d_res.p[point].status, sizeof pst, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (pst != TRIOSIM_PT_OK) return TRIOSIM_OK;   // rejected in K3 (R3) or deadlocked: no timeline
+    if (cnt[0] <= task_cap && cnt[1] <= flow_cap) CK(sort_timeline(S.d_tl_tasks.p, cnt[0], S.d_tl_flows.p, cnt[1], st));
+    const uint64_t kt = cnt[0] < task_cap ? cnt[0] : task_cap, kf = cnt[1] < flow_cap ? cnt[1] : flow_cap;
+    if (kt) CK(cudaMemcpyAsync(tasks, S.d_tl_tasks.p, kt * sizeof(triosim_task_rec), cudaMemcpyDeviceToHost, st));
+    if (kf) CK(cudaMemcpyAsync(flows, S.d_tl_flows.p, kf * sizeof(triosim_flow_rec), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    *n_tasks = cnt[0];
+    *n_flows = cnt[1];
     return TRIOSIM_OK;
 }
 

@@ -117,6 +117,7 @@ struct ClassDesc {
     uint32_t scratch_off, dp;            // dp: HYBRID data-parallel degree
     uint32_t hst_off, tcol_off, tcol_cap, dcol_off, dcol_cap;   // HYBRID pools
     uint32_t dp_after_bwd;               // HYBRID form of DataParallel: DP buckets trigger after the backward pass
+    uint32_t first_bucket;               // R24: cap of each gradient group's first bucket (0 = bucket_bytes)
     // written by K2
     uint32_t n_coll, need_ring, need_tree, n_prog_max;
     double coll_payload;
@@ -170,7 +171,16 @@ struct K3Args {
     double *bd;
     const uint32_t *layer;         // trace: layer of each operator
     uint32_t n_layers, pad3;
+    // R23 timeline (kernel variant LOG only): record slots counted in tl_cnt[0] (tasks), [1] (flows)
+    triosim_task_rec *tl_tasks;
+    triosim_flow_rec *tl_flows;
+    unsigned long long *tl_cnt;
+    uint64_t tl_task_cap, tl_flow_cap;
 };
+
+// K3 instantiations: V bit 0 = BD (R22 breakdown), bit 1 = LOG (R23 timeline; no ring fast-forward)
+constexpr int V_BD = 1, V_LOG = 2;
+__host__ __device__ constexpr int k3_variant(bool bd, bool log) { return (bd ? V_BD : 0) | (log ? V_LOG : 0); }
 
 // launchers (ts_kernels.cu)
 cudaError_t launch_k1_ingest(const TraceDev &T, cudaStream_t s);
@@ -183,7 +193,8 @@ cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
                              const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
                              RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
-// K3 variants: a.bd != nullptr selects the breakdown-recording (BD) instantiation
+// K3 variants: a.bd != nullptr selects the breakdown-recording (BD) instantiation, a.tl_cnt != nullptr the
+// timeline-recording (LOG) one
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu
 cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s);      // ts_k3h.cu
 // R22: per-class layer compute (left fold of t' over the representative rank's program) and the
@@ -194,6 +205,8 @@ cudaError_t launch_k4_layer_compute(const ClassDesc *cls, uint32_t n_cls, const 
 cudaError_t launch_k4_breakdown(const PointDesc *pts, const triosim_result *res, uint64_t first, uint64_t count,
                                 uint32_t n_layers, const double *lcomp, const double *acc, double *out_comp,
                                 double *out_comm, cudaStream_t s);
+// R23: canonical order of the recorded timeline (ts_timeline.cu)
+cudaError_t sort_timeline(triosim_task_rec *tasks, uint64_t nt, triosim_flow_rec *flows, uint64_t nf, cudaStream_t s);
 int k3h_max_blocks_per_sm(int W, uint32_t lmax, uint32_t pmax);   // dynamic smem: links (W > 32), ports
 size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax);
 int k3_max_blocks_per_sm(int W, int mode);

@@ -114,10 +114,13 @@ __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[
 #ifndef TS_K3_MINB
 #define TS_K3_MINB 1
 #endif
-// BD: also record the per-layer communication breakdown (R22) into a.bd (a separate instantiation,
-// so the plain timeline carries none of its state)
-template <int W, int MODE, bool BD>
+// V & V_BD: also record the per-layer communication breakdown (R22) into a.bd; V & V_LOG: record the
+// R23 timeline (every task and flow with its times) -- separate instantiations, so the plain timeline
+// carries none of their state
+template <int W, int MODE, int V>
 __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Args a) {
+    constexpr bool BD = (V & V_BD) != 0;
+    constexpr bool LOG = (V & V_LOG) != 0;
     constexpr int NSEG = 32 / W;
     constexpr int LMAX = lmax_warp(W);
     constexpr bool COLL = MODE != MODE_PIPE;   // DP / DDP / TP collectives
@@ -191,6 +194,27 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     // start or release time and the layer it is attributed to; category 0 TP / 1 DP / 2 P2P
     double bd_t0 = 0.0;
     uint32_t bd_l = 0, bd_cat = 0;
+    // R23 (LOG): record slot of this lane's flow in flight
+    unsigned long long tl_fs = 0;
+    auto tl_task = [&](uint32_t g, uint32_t prog, uint32_t op, uint32_t mb, double t0, double t1) {
+        const unsigned long long k = atomicAdd(&a.tl_cnt[0], 1ull);
+        if (k < a.tl_task_cap) {
+            triosim_task_rec r;
+            r.gpu = g; r.prog = prog; r.op = op; r.mb = mb; r.start_s = t0; r.end_s = t1;
+            a.tl_tasks[k] = r;
+        }
+    };
+    auto tl_release = [&](uint32_t src, uint32_t dst) {
+        tl_fs = atomicAdd(&a.tl_cnt[1], 1ull);
+        if (tl_fs < a.tl_flow_cap) {
+            triosim_flow_rec r;
+            r.code = fcode; r.src = src; r.dst = dst; r.bytes = fbytes; r.release_s = t;
+            r.start_s = r.delivered_s = 0.0;
+            a.tl_flows[tl_fs] = r;
+        }
+    };
+    auto tl_start = [&]() { if (tl_fs < a.tl_flow_cap) a.tl_flows[tl_fs].start_s = t; };
+    auto tl_deliver = [&]() { if (tl_fs < a.tl_flow_cap) a.tl_flows[tl_fs].delivered_s = t; };
 
 #define EV(kind, code)                                                  \
     do {                                                                \
@@ -355,7 +379,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 #ifdef TS_PROF
         const long long pf_a = clock64();
 #endif
-        if constexpr (COLL) {
+        if constexpr (COLL && !LOG) {
             if (__any_sync(FULL, have && running && ring_ff && !tree_cur)) {
                 const double tc = seg_min_shfl<W>(used && cst == CS_RUN ? t_end : dinf());
                 const int Dseg = __shfl_sync(FULL, D, sbase);
@@ -487,12 +511,15 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 if (used && fst == FS_ACT && t_drain == t) {
                     fst = FS_NONE;
                     EV(EV_DELIVER, fcode);
+                    if constexpr (LOG) tl_deliver();
                     delivered = dirty = true;
                 } else if (used && fst == FS_LAT && t_act == t) {
                     EV(EV_ACTIVATE, fcode);
+                    if constexpr (LOG) tl_start();
                     if (fbytes == 0.0 || flen == 0) {
                         fst = FS_NONE;
                         EV(EV_DELIVER, fcode);
+                        if constexpr (LOG) tl_deliver();
                         delivered = true;
                     } else {
                         fst = FS_ACT;
@@ -581,6 +608,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 t_act = t + Lring;
                                 alg += 1;
                                 fcode = ((uint64_t)cur << 32) | ((uint64_t)D << 16) | (uint64_t)li;
+                                if constexpr (LOG) tl_release(gpu, a.ro[TR.ro_off + (li + 1) % p]);
                             }
                         } else if (TREE && li >= 1) {
                             const unsigned um = started ? 0u : upm, dm = started ? 0u : dnm;
@@ -594,6 +622,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 t_act = t + load_route(a, TR, r, lats, hl);
                                 fcode = ((uint64_t)cur << 32) | (uint64_t)li;
                                 fup = uprel = rel = true;
+                                if constexpr (LOG) { fbytes = cS; tl_release(gpu, par); }
                             } else if (uprel && upd && !dnrel &&
                                        (par_i == 0 ? ((p <= 1 || ((um >> 1) & 1u)) && (p <= 2 || ((um >> 2) & 1u)))
                                                    : ((dm >> par_i) & 1u))) {
@@ -604,6 +633,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 fcode = ((uint64_t)cur << 32) | (1ull << 16) | (uint64_t)li;
                                 fup = false;
                                 dnrel = rel = true;
+                                if constexpr (LOG) { fbytes = cS; tl_release(par, gpu); }
                             }
                             if (rel) {
                                 fbytes = cS;
@@ -640,6 +670,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             alg += 2 * flen + 1;
                             fcode = (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg;
                             EV(EV_RELEASE, fcode);
+                            if constexpr (LOG) tl_release(gpu, dg);
                             if constexpr (BD) {
                                 bd_t0 = t;
                                 bd_l = a.layer[a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + se.pidx].op];
@@ -658,11 +689,13 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             if (h.wait >= 0) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
                             run_start = pos;
                             double te = t + h.dur;
+                            if constexpr (LOG) tl_task(gpu, pos, pos, 0, t, te);
                             busy = busy + h.dur;
                             uint32_t q = pos + 1, sig = h.nsig;
                             while (sig == 0 && q < nprog) {
                                 const OpHook h2 = HK[q];
                                 if (h2.wait >= 0) break;
+                                if constexpr (LOG) tl_task(gpu, q, q, 0, te, te + h2.dur);
                                 te = te + h2.dur;
                                 busy = busy + h2.dur;
                                 sig = h2.nsig;
@@ -697,6 +730,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             const double *du = a.dur + C->dur_off;
                             const double d0 = du[en.op];
                             double te = t + d0;
+                            if constexpr (LOG) tl_task(gpu, pos, en.op, j, t, te);
                             busy = busy + d0;
                             uint32_t ns = en.nsend;
                             q++;
@@ -707,6 +741,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 const StageEnt e2 = a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx];
                                 if (e2.nrecv) break;
                                 const double dd = du[e2.op];
+                                if constexpr (LOG) {
+                                    const uint32_t j2 = P == 0 ? q / SI.nF : P == 1 ? m - 1 - (q - m * SI.nF) / SI.nB : 0;
+                                    tl_task(gpu, q, e2.op, j2, te, te + dd);
+                                }
                                 te = te + dd;
                                 busy = busy + dd;
                                 ns = e2.nsend;
@@ -887,8 +925,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 
 template <int W, int MODE>
 static cudaError_t launch_wm(const K3Args &a, int grid, cudaStream_t s) {
-    if (a.bd) k3_timeline<W, MODE, true><<<grid, K3_THREADS, 0, s>>>(a);
-    else k3_timeline<W, MODE, false><<<grid, K3_THREADS, 0, s>>>(a);
+    if (a.tl_cnt) k3_timeline<W, MODE, V_LOG><<<grid, K3_THREADS, 0, s>>>(a);
+    else if (a.bd) k3_timeline<W, MODE, V_BD><<<grid, K3_THREADS, 0, s>>>(a);
+    else k3_timeline<W, MODE, 0><<<grid, K3_THREADS, 0, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -915,9 +954,9 @@ cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s
 template <int W>
 static int occ_w(int mode) {
     int nb = 0;
-    if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL, false>, K3_THREADS, 0);
-    else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE, false>, K3_THREADS, 0);
-    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE, false>, K3_THREADS, 0);
+    if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL, 0>, K3_THREADS, 0);
+    else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE, 0>, K3_THREADS, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE, 0>, K3_THREADS, 0);
     return nb;
 }
 

@@ -65,6 +65,8 @@ struct Flow {
     int len;
     uint32_t hl[4];
     uint64_t code;
+    uint32_t src, dst;            // endpoints (R23 timeline records only)
+    unsigned long long tl;        // R23 (LOG): record slot
 };
 
 // one boolean per segment lane: ballot bits (warp segments) or a shared-memory byte array (CTA)
@@ -107,6 +109,8 @@ __device__ __forceinline__ int route_len(const K3Args &a, const Topo &T, uint32_
 // (R20): a send request keyed by (release time t_upd, code); hl[0] = destination GPU, hl[1] = link slot
 __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f, uint32_t src, uint32_t dst,
                                         double bytes, uint64_t code, double t, double lats, uint64_t &alg) {
+    f.src = src;
+    f.dst = dst;
     if (T.phot) {
         f.len = 0;
         f.bytes = bytes;
@@ -146,9 +150,12 @@ __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f,
 }  // namespace
 
 
-// BD: also record the per-layer communication breakdown (R22) into a.bd (separate instantiation)
-template <int W, int NW, bool BD>
+// V & V_BD: also record the per-layer communication breakdown (R22) into a.bd; V & V_LOG: record the R23
+// timeline (separate instantiations)
+template <int W, int NW, int V>
 __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(const K3Args a) {
+    constexpr bool BD = (V & V_BD) != 0;
+    constexpr bool LOG = (V & V_LOG) != 0;
     constexpr int SL = NW == 1 ? W : 32 * NW;           // lanes per segment
     constexpr int NSEG = NW == 1 ? 32 / W : 1;          // segments per warp (NW = 1)
     constexpr int LMAXW = lmax_hybrid(W);               // warp segments: static link arrays
@@ -349,6 +356,26 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         double *q = a.bd + ((size_t)pidx * 3 + cat) * a.n_layers + l;
         *q = *q + dt;
     };
+    // R23 (LOG): task and flow records
+    auto tl_task = [&](uint32_t g, uint32_t prog, uint32_t op, uint32_t mbi, double t0, double t1) {
+        const unsigned long long k = atomicAdd(&a.tl_cnt[0], 1ull);
+        if (k < a.tl_task_cap) {
+            triosim_task_rec r;
+            r.gpu = g; r.prog = prog; r.op = op; r.mb = mbi; r.start_s = t0; r.end_s = t1;
+            a.tl_tasks[k] = r;
+        }
+    };
+    auto tl_release = [&](Flow &F) {
+        F.tl = atomicAdd(&a.tl_cnt[1], 1ull);
+        if (F.tl < a.tl_flow_cap) {
+            triosim_flow_rec r;
+            r.code = F.code; r.src = F.src; r.dst = F.dst; r.bytes = F.bytes; r.release_s = t;
+            r.start_s = r.delivered_s = 0.0;
+            a.tl_flows[F.tl] = r;
+        }
+    };
+    auto tl_start = [&](const Flow &F) { if (F.tl < a.tl_flow_cap) a.tl_flows[F.tl].start_s = t; };
+    auto tl_deliver = [&](const Flow &F) { if (F.tl < a.tl_flow_cap) a.tl_flows[F.tl].delivered_s = t; };
 
 #define EV(kind, code)                                                        \
     do {                                                                      \
@@ -474,6 +501,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             }
             if (rel) {
                 EV(EV_RELEASE, F.code);
+                if constexpr (LOG) tl_release(F);
                 if (F.t_act == t) more = true;
             }
         }
@@ -483,15 +511,18 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         if (F.st == FS_ACT && F.t_drain == t) {
             F.st = FS_NONE;
             EV(EV_DELIVER, F.code);
+            if constexpr (LOG) tl_deliver(F);
             if (TR.phot) p_t[F.hl[1] * NTHR + threadIdx.x] = t;   // R20: the logical link was last used now
             else dirty = true;
             return true;
         }
         if (F.st == FS_LAT && F.t_act == t) {
             EV(EV_ACTIVATE, F.code);
+            if constexpr (LOG) tl_start(F);
             if (F.bytes == 0.0 || F.len == 0) {
                 F.st = FS_NONE;
                 EV(EV_DELIVER, F.code);
+                if constexpr (LOG) tl_deliver(F);
                 return true;
             }
             F.st = FS_ACT;
@@ -692,6 +723,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         release(a, TR, FP, gpu, dg, se.bytes,
                                 (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg, t, lats, alg);
                         EV(EV_RELEASE, FP.code);
+                        if constexpr (LOG) tl_release(FP);
                         if constexpr (BD) {
                             bd_p_t0 = t;
                             bd_p_l = a.layer[ent_at(P, se.pidx).op];
@@ -726,6 +758,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         run_start = pos;
                         const double *du = a.dur + C->dur_off;
                         double te = t + du[en.op];
+                        if constexpr (LOG) tl_task(gpu, pos, en.op, j, t, te);
                         busy = busy + du[en.op];
                         bool sig = has_sig(en, j);
                         uint32_t q = pos + 1;
@@ -734,6 +767,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             decode(q, P2, j2, i2);
                             const HEnt e2 = ent_at(P2, i2);
                             if (has_wait(e2, P2, i2)) break;
+                            if constexpr (LOG) tl_task(gpu, q, e2.op, j2, te, te + du[e2.op]);
                             te = te + du[e2.op];
                             busy = busy + du[e2.op];
                             sig = has_sig(e2, j2);
@@ -862,6 +896,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         F.t_drain = (t + ph_lat) + F.bytes / ph_bw;
                         alg += 3;
                         EV(EV_ACTIVATE, F.code);
+                        if constexpr (LOG) tl_start(F);
                         if (F.t_drain == t) again = true;
                     }
                 };
@@ -1106,19 +1141,20 @@ size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
     return (W <= 32 ? 0 : (size_t)lmax * 16) + ph;
 }
 
-template <int W, int NW, bool BD>
+template <int W, int NW, int V>
 static cudaError_t launch_hb(const K3Args &a, int grid, cudaStream_t s) {
     const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, a.lmax, a.pmax);
     if (dyn > 0) {
-        const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW, BD>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+        const cudaError_t e = cudaFuncSetAttribute(k3_hybrid<W, NW, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
         if (e != cudaSuccess) return e;
     }
-    k3_hybrid<W, NW, BD><<<grid, NW == 1 ? K3_THREADS : 32 * NW, dyn, s>>>(a);
+    k3_hybrid<W, NW, V><<<grid, NW == 1 ? K3_THREADS : 32 * NW, dyn, s>>>(a);
     return cudaGetLastError();
 }
 template <int W, int NW>
 static cudaError_t launch_h(const K3Args &a, int grid, cudaStream_t s) {
-    return a.bd ? launch_hb<W, NW, true>(a, grid, s) : launch_hb<W, NW, false>(a, grid, s);
+    return a.tl_cnt ? launch_hb<W, NW, V_LOG>(a, grid, s)
+         : a.bd ? launch_hb<W, NW, V_BD>(a, grid, s) : launch_hb<W, NW, 0>(a, grid, s);
 }
 
 // W <= 32: W-lane segments in 256-thread CTAs; W = 64..1024: one point per CTA of W threads
@@ -1141,10 +1177,10 @@ cudaError_t launch_k3_hybrid(int W, const K3Args &a, int grid, cudaStream_t s) {
 template <int W, int NW>
 static int occ_h(uint32_t lmax, uint32_t pmax) {
     const size_t dyn = k3h_dyn_smem(NW == 1 ? W : 32 * NW, lmax, pmax);
-    if (dyn > 0 && cudaFuncSetAttribute(k3_hybrid<W, NW, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
+    if (dyn > 0 && cudaFuncSetAttribute(k3_hybrid<W, NW, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn) != cudaSuccess)
         return 0;
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW, false>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_hybrid<W, NW, 0>, NW == 1 ? K3_THREADS : 32 * NW, dyn);
     return nb;
 }
 

@@ -126,6 +126,13 @@ __device__ __forceinline__ double tensor_bytes(const TraceDev &T, uint32_t x, do
     return b;
 }
 
+// R24: cap of gradient bucket number k of a group (PyTorch DDP's first-bucket rule); 0 = one tensor per
+// AllReduce (Q5)
+__device__ __forceinline__ uint64_t bucket_cap(const ClassDesc &C, uint32_t k) {
+    if (C.bucket_bytes == 0) return 0;
+    return (k == 0 && C.first_bucket != 0) ? (uint64_t)C.first_bucket : C.bucket_bytes;
+}
+
 // ------------------------------------------------------------------------------------
 // K2 (COLL): one CTA per DP/DDP/TP class
 // ------------------------------------------------------------------------------------
@@ -153,7 +160,8 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
             if (C.p > 1) {
                 int i = 0;
                 while (i < nw) {
-                    // gradient bucket (reading Q5): greedy on the u64 byte sum
+                    // gradient bucket (reading Q5): greedy on the u64 byte sum, first cap per R24
+                    const uint64_t cap = bucket_cap(C, nc);
                     uint64_t sum = 0;
                     double S = 0.0;
                     int j = i;
@@ -162,7 +170,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         sum += T.ts[x].bytes_b0;
                         S = S + tensor_bytes(T, x, C.r_b, 1, C.tp_mode);
                         j++;
-                        if (C.bucket_bytes == 0 || sum >= C.bucket_bytes || j == nw) break;
+                        if (cap == 0 || sum >= cap || j == nw) break;
                     }
                     int trig = (C.strategy == TRIOSIM_DDP) ? T.prod[T.wgrad[j - 1]] : last_nonopt;
                     CE[nc].S = S;
@@ -483,7 +491,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                 if (s_stage[T.layer[T.prod[x]]] != s) continue;
                 sum += T.ts[x].bytes_b0;
                 open = true;
-                if (C.bucket_bytes == 0 || sum >= C.bucket_bytes) { nb++; sum = 0; open = false; }
+                const uint64_t cap = bucket_cap(C, nb);
+                if (cap == 0 || sum >= cap) { nb++; sum = 0; open = false; }
             }
             if (open) nb++;
         }
@@ -585,7 +594,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     last_prod = T.prod[x];
                     open = true;
                 }
-                if (open && (end || C.bucket_bytes == 0 || sum >= C.bucket_bytes)) {
+                const uint64_t cap = bucket_cap(C, b);
+                if (open && (end || cap == 0 || sum >= cap)) {
                     CollEnt ce;
                     ce.S = Sb;
                     ce.kind = CK_AR;

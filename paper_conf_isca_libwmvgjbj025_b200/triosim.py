@@ -20,7 +20,7 @@ LIB_PATH = os.environ.get("TRIOSIM_LIB", os.path.join(HERE, "libtriosim.so"))
 EXPORTS = ["triosim_create", "triosim_destroy", "triosim_last_error", "triosim_load_trace", "triosim_build_sweep",
            "triosim_simulate_batch", "triosim_results", "triosim_release", "triosim_launch_counts",
            "triosim_results_device_ptr", "triosim_work_counters", "triosim_timing", "triosim_timings",
-           "triosim_set_breakdown", "triosim_breakdown"]
+           "triosim_set_breakdown", "triosim_breakdown", "triosim_timeline"]
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENOTFOUND", -5: "ERANGE", -6: "EUNSUPPORTED"}
 
@@ -74,6 +74,7 @@ def load_library(path=LIB_PATH):
         L.triosim_timing.argtypes = [P, C.c_int]
         L.triosim_timings.argtypes = [P, P, P, i32]
         L.triosim_set_breakdown.argtypes = [P, i32, C.c_int]
+        L.triosim_timeline.argtypes = [P, i32, u64, P, u64, P, u64, C.POINTER(u64), C.POINTER(u64)]
         L.triosim_breakdown.argtypes = [P, i32, u64, u64, P, P, C.c_int, P]
         L.triosim_results_device_ptr.argtypes = [P, i32]
         L.triosim_results_device_ptr.restype = P
@@ -191,6 +192,22 @@ class Context:
         self._check("triosim_breakdown", self.L.triosim_breakdown(self.h, int(sweep_id), int(first), int(count),
                                                                   _ptr(comp), _ptr(comm), 0, sp))
         return comp, comm
+
+    def triosim_timeline(self, sweep_id: int, point: int, task_cap=None, flow_cap=None):
+        """R23 timeline of one point: (tasks TASK_REC_DTYPE sorted by (gpu, prog), flows FLOW_REC_DTYPE sorted
+        by (release, code)).  Without caps, a first call sizes the arrays."""
+        nt, nf = C.c_uint64(), C.c_uint64()
+        for _ in range(2):
+            tc = 0 if task_cap is None else int(task_cap)
+            fc = 0 if flow_cap is None else int(flow_cap)
+            tasks = np.zeros(tc, W.TASK_REC_DTYPE)
+            flows = np.zeros(fc, W.FLOW_REC_DTYPE)
+            self._check("triosim_timeline", self.L.triosim_timeline(self.h, int(sweep_id), int(point), _ptr(tasks), tc,
+                                                                    _ptr(flows), fc, C.byref(nt), C.byref(nf)))
+            if nt.value <= tc and nf.value <= fc:
+                return tasks[:nt.value], flows[:nf.value]
+            task_cap, flow_cap = nt.value, nf.value
+        raise TrioSimError("triosim_timeline", -1, "record counts changed between calls")
 
     def triosim_release(self, handle: int):
         self._check("triosim_release", self.L.triosim_release(self.h, int(handle)))

@@ -254,3 +254,24 @@ def test_wafer_passage_case_study(ctx):
     assert (got["comm_busy_s"][phot] >= 20e-3 * sw.points["lat_scale"][phot]).all()
     idx = sample(len(sw.points), 24, 66)
     check(got, sw, idx)
+
+
+def test_first_bucket_rule(ctx):
+    """R24 (PyTorch DDP's first-bucket cap) for DP, DDP and HYBRID points, ring and tree, against the oracle;
+    points differing only in the first cap fall in different structural classes."""
+    rng = np.random.Generator(np.random.PCG64(2400))
+    tr = W.resnet50_trace()
+    topos = [W.ring(8, 100e9, 2e-6), W.star(8, 80e9, 1e-6)]
+    pts = []
+    for _ in range(160):
+        st = int(rng.choice([W.ST_DP, W.ST_DDP, W.ST_HYBRID]))
+        cap = int(rng.choice([0, 1 << 20, 25 << 20]))
+        first = int(rng.choice([0, 1, 1 << 20, 4 << 20]))
+        kw = dict(dp=int(rng.choice([2, 4, 8])), B=0) if st != W.ST_HYBRID else dict(dp=2, tp=2, pp=2, m=2, B=0)
+        kw["B"] = kw["dp"] * int(kw.get("m", 1)) * 32
+        pts.append(W.make_point(int(rng.integers(2)), st, bucket=cap, first_bucket=first, algo=int(rng.integers(2)),
+                                bw=float(rng.uniform(0.2, 2)), lat=float(rng.uniform(0.5, 2)), **kw))
+    sw = W.Sweep("first-bucket", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    assert (got["status"] == 0).all()
+    check(got, sw, list(range(len(pts))))
