@@ -401,7 +401,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                     // blocks of up to four steps (eight instants): first the instant times (a short
                     // dependent chain of adds), then their hash terms, which are independent of each other
                     while (go) {
-                        double ti[8];
+                        double ti[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
                         int n = 0;
                         const int D0 = Dl;
 #pragma unroll
@@ -432,18 +432,23 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             }
                         }
                         if (used) {
+                            // all eight terms unconditionally (no branches: eight independent chains the
+                            // compiler interleaves), the ones past n masked out of the sum
+                            uint64_t add = 0;
 #pragma unroll
-                            for (int i = 0; i < 8; i++)
-                                if (i < n) {
-                                    const uint64_t m = mix64((uint64_t)__double_as_longlong(ti[i]));
-                                    const uint64_t k = (uint64_t)(D0 + (i >> 1));
-                                    if ((i & 1) == 0) {
-                                        acc += emix(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
-                                    } else {
-                                        acc += emix(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16)));
-                                        acc += emix(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
-                                    }
+                            for (int i = 0; i < 8; i++) {
+                                const uint64_t m = mix64((uint64_t)__double_as_longlong(ti[i]));
+                                const uint64_t k = (uint64_t)(D0 + (i >> 1));
+                                uint64_t term;
+                                if ((i & 1) == 0) {
+                                    term = emix(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
+                                } else {
+                                    term = emix(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16))) +
+                                           emix(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
                                 }
+                                add += i < n ? term : 0ull;
+                            }
+                            acc += add;
                             alg += 2u * (uint32_t)((n + 1) >> 1) + (uint32_t)(n >> 1);
                             nflow += (uint32_t)(n >> 1);
                         }
