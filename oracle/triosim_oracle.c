@@ -67,7 +67,8 @@ typedef struct {
 
 typedef struct {
     uint32_t topo;
-    uint8_t strategy, tp_mode, coll_algo, pad0;
+    uint8_t strategy, tp_mode, coll_algo;
+    uint8_t ring_chunks;           /* R25: chunks per ring step (0 or 1 = unchunked, R10) */
     uint16_t dp, tp, pp, pad1;
     uint32_t microbatches, global_batch;
     int32_t stage_plan;
@@ -254,6 +255,7 @@ typedef struct {
     GNode *n; long count, cap;
     IVec dep_from, dep_to;   /* edge list: node dep_from[i] waits for node dep_to[i] */
     int n_coll;
+    int nch;                 /* R25: chunks per ring step of this point's ring collectives (>= 1) */
     double coll_payload;     /* left fold of collective payloads in creation order */
     /* R22 per-layer breakdown: the representative rank of each layer, and the communications it
      * takes part in, attributed to the layer of the operator that triggers / produces them */
@@ -317,8 +319,8 @@ static uint64_t p2p_flow_code(uint32_t x, int j, int dst) {
  * per (GPU, group), reading Q24) or NULL.  Writes done[i] = barrier "this
  * collective is done on member i" (last flow touching it delivered).
  */
-static int build_collective_code(Graph *G, uint64_t c, const int *members, int p, int kind, int algo, double S,
-                                 const int *trig, const int *prev_done, int *done) {
+static int build_collective_code(Graph *G, uint64_t c, const int *members, int p, int kind, int algo, int nch,
+                                 double S, const int *trig, const int *prev_done, int *done) {
     G->n_coll++;
     G->coll_payload = G->coll_payload + S;
     int sb = add_barrier(G, NF_COLL_START, (uint64_t)c);
@@ -331,9 +333,14 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
     if (algo == ALG_RING || kind != CK_AR) {
         /* ring: K steps; flow (i,k) goes m_i -> m_(i+1); released at start if k == 0,
          * else when (i-1,k-1) [predecessor's chunk arrived] and (i,k-1) [own previous
-         * send] are both delivered (reading Q21). */
-        int K = (kind == CK_AR) ? 2 * (p - 1) : (p - 1);
-        double chunk = S / (double)p;
+         * send] are both delivered (reading Q21).
+         * R25 pipelined ring (NCCL chunking): each step's slice S/p is cut into
+         * nch chunks of S/(p*nch); member i sends its flows one at a time in the order
+         * q = k*nch + j; flow (i,q) is released when (i,q-1) [own previous chunk] and,
+         * for k >= 1, (i-1,q-nch) [chunk j of the predecessor's step k-1] are delivered.
+         * nch == 1 is the rule above. */
+        int K = ((kind == CK_AR) ? 2 * (p - 1) : (p - 1)) * nch;
+        double chunk = S / (double)p / (double)nch;
         int *id = (int *)malloc(sizeof(int) * (size_t)(p * (K > 0 ? K : 1)));
         if (!id) return -1;
         for (int k = 0; k < K; k++)
@@ -345,7 +352,7 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
                 if (k == 0) {
                     g_dep(G, f, sb);
                 } else {
-                    g_dep(G, f, id[(k - 1) * p + (i - 1 + p) % p]);
+                    if (k >= nch) g_dep(G, f, id[(k - nch) * p + (i - 1 + p) % p]);
                     g_dep(G, f, id[(k - 1) * p + i]);
                 }
             }
@@ -400,7 +407,7 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
 /* collectives of DP / DDP / TP: one group, numbered in creation order */
 static int build_collective(Graph *G, const int *members, int p, int kind, int algo, double S,
                             const int *trig, const int *prev_done, int *done) {
-    return build_collective_code(G, (uint64_t)G->n_coll, members, p, kind, algo, S, trig, prev_done, done);
+    return build_collective_code(G, (uint64_t)G->n_coll, members, p, kind, algo, G->nch, S, trig, prev_done, done);
 }
 
 /* ------------------------------------------------------------------ */
@@ -541,7 +548,8 @@ static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
 /* ------------------------------------------------------------------ */
 static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
                        int have_plan) {
-    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_TREE) return PT_BAD_CONFIG;
+    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_TREE ||
+        pt->ring_chunks > 16) return PT_BAD_CONFIG;   /* R25: at most 16 chunks per ring step */
     if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
         return PT_BAD_CONFIG;
     uint32_t dp = pt->dp, tpd = pt->tp, pp = pt->pp, m = pt->microbatches;
@@ -911,7 +919,7 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                         for (int t = 0; t < tp; t++) trig[t] = task[base + t][q];
                         G->cur_layer = (int)op->layer;
                         G->cur_cat = 0;
-                        if (build_collective_code(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, Sb, trig,
+                        if (build_collective_code(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, G->nch, Sb, trig,
                                                   have_prev ? prev : NULL, done)) goto out;
                         seq++;
                         memcpy(prev, done, sizeof(int) * (size_t)tp);
@@ -1023,7 +1031,7 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                     for (int d = 0; d < dp; d++) trig[d] = task[(d * S + s) * tp + t][qt];
                     G->cur_layer = (int)T->ops[pop[s][qt]].layer;
                     G->cur_cat = 1;
-                    if (build_collective_code(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, Sb, trig,
+                    if (build_collective_code(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, G->nch, Sb, trig,
                                               have_prev ? prev : NULL, done)) { free(w); goto out; }
                     seq++;
                     memcpy(prev, done, sizeof(int) * (size_t)dp);
@@ -1601,6 +1609,7 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
     if (!G->rep) { free(ro); return -1; }
     for (uint32_t l = 0; l < T->n_layers; l++) G->rep[l] = ro[0];
     G->cur_layer = -1;
+    G->nch = pt->ring_chunks > 1 ? (int)pt->ring_chunks : 1;   /* R25 */
     switch (pt->strategy) {
     case ST_DP: case ST_DDP: rc = expand_dp(T, pt, ro, G); break;
     case ST_TP: rc = expand_tp(T, pt, ro, G); break;

@@ -35,7 +35,7 @@ TENSOR_DTYPE = np.dtype([
     ("bytes_b0", "<u8"), ("category", "u1"), ("batch_scaled", "u1"), ("pad", "<u2"), ("param_id", "<u4")])
 LINK_DTYPE = np.dtype([("src", "<u4"), ("dst", "<u4"), ("bw_Bps", "<f8"), ("lat_s", "<f8")])
 POINT_DTYPE = np.dtype([
-    ("topo", "<u4"), ("strategy", "u1"), ("tp_mode", "u1"), ("coll_algo", "u1"), ("pad0", "u1"),
+    ("topo", "<u4"), ("strategy", "u1"), ("tp_mode", "u1"), ("coll_algo", "u1"), ("ring_chunks", "u1"),
     ("dp", "<u2"), ("tp", "<u2"), ("pp", "<u2"), ("pad1", "<u2"),
     ("microbatches", "<u4"), ("global_batch", "<u4"), ("stage_plan", "<i4"), ("first_bucket_bytes", "<u4"),
     ("bucket_bytes", "<u8"), ("bw_scale", "<f8"), ("lat_scale", "<f8")])
@@ -677,9 +677,10 @@ class Sweep:
 
 
 def make_point(topo, strategy, dp=1, tp=1, pp=1, m=1, B=1, bucket=0, bw=1.0, lat=1.0, tp_mode=TPM_MEGATRON,
-               algo=ALG_RING, plan=-1, first_bucket=0):
+               algo=ALG_RING, plan=-1, first_bucket=0, chunks=0):
     p = np.zeros((), POINT_DTYPE)
     p["first_bucket_bytes"] = first_bucket
+    p["ring_chunks"] = chunks
     p["topo"], p["strategy"], p["tp_mode"], p["coll_algo"] = topo, strategy, tp_mode, algo
     p["dp"], p["tp"], p["pp"], p["microbatches"], p["global_batch"] = dp, tp, pp, m, B
     p["stage_plan"], p["bucket_bytes"], p["bw_scale"], p["lat_scale"] = plan, bucket, bw, lat
