@@ -153,7 +153,11 @@ typedef struct {
 
 typedef struct {
     uint32_t topo;
-    uint8_t strategy, tp_mode, coll_algo, pad0;
+    uint8_t strategy, tp_mode, coll_algo;
+    uint8_t ring_chunks;     /* chunks per ring step, pipelined (NCCL-style; R25): each ring step's
+                                slice S/p is sent as ring_chunks flows of S/(p*ring_chunks), one at a time per
+                                member; 0 or 1 = unchunked (R10); > 16 -> TRIOSIM_PT_BAD_CONFIG; ignored by
+                                tree AllReduces */
     uint16_t dp, tp, pp, pad1;
     uint32_t microbatches, global_batch;
     int32_t stage_plan;      /* -1 = automatic balanced partition */

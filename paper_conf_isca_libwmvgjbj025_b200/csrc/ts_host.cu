@@ -467,7 +467,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto setst = [&](int st) { S->status[i] = st; };
         // R3, in order
         if (pt.topo >= n_topos) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
-        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 1) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 1 || pt.ring_chunks > 16) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
         if (!(pt.bw_scale > 0.0) || std::isinf(pt.bw_scale) || !(pt.lat_scale >= 0.0) || std::isinf(pt.lat_scale)) {
             setst(TRIOSIM_PT_BAD_CONFIG);
             continue;
@@ -539,8 +539,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         uint64_t key_bucket = (pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP || hyb) ? pt.bucket_bytes : 0;
         uint32_t key_first = key_bucket ? pt.first_bucket_bytes : 0;   // R24
         int key_m = (mode == MODE_PIPE || hyb) ? (int)mbe : 0;
+        int key_nch = mode != MODE_PIPE && pt.ring_chunks > 1 ? (int)pt.ring_chunks : 1;   // R25
         auto key = std::make_tuple((int)pt.strategy + (dp_after ? 100 : 0), (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
-                                   hyb ? (int)tpd : 0, key_algo, key_bucket, key_first, key_m,
+                                   hyb ? (int)tpd : 0, key_algo * 32 + key_nch, key_bucket, key_first, key_m,
                                    (mode == MODE_PIPE || hyb) ? plan_key : -2);
         auto ci = cls_of.find(key);
         uint32_t c;
@@ -559,6 +560,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.b_loc = b_loc;
             cd.bucket_bytes = key_bucket;
             cd.first_bucket = key_first;
+            cd.nch = (uint32_t)key_nch;
             cd.r_b = (double)b_loc / (double)T.b0;
             if (mode == MODE_PIPE || hyb) {
                 if (plan_key < 0) {

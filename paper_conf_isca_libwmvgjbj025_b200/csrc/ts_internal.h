@@ -118,6 +118,7 @@ struct ClassDesc {
     uint32_t hst_off, tcol_off, tcol_cap, dcol_off, dcol_cap;   // HYBRID pools
     uint32_t dp_after_bwd;               // HYBRID form of DataParallel: DP buckets trigger after the backward pass
     uint32_t first_bucket;               // R24: cap of each gradient group's first bucket (0 = bucket_bytes)
+    uint32_t nch, pad_nch;               // R25: chunks per ring step (>= 1)
     // written by K2
     uint32_t n_coll, need_ring, need_tree, n_prog_max;
     double coll_payload;

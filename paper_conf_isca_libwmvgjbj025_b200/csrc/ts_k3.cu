@@ -594,8 +594,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         running = started = true;
                         tree_cur = tree_algo && ce.kind == CK_AR;
                         cS = ce.S;
-                        chunk = ce.S / (double)p;
-                        K = (ce.kind == CK_AR) ? 2 * (p - 1) : (p - 1);
+                        // R25: nch chunks of S / p / nch per ring step, sent one at a time (q = k nch + j)
+                        chunk = ce.S / (double)p / (double)C->nch;
+                        K = ((ce.kind == CK_AR) ? 2 * (p - 1) : (p - 1)) * (int)C->nch;
                         D = 0;
                         ldone = uprel = upd = dnrel = dnd = false;
                         if (li == 0) { EV(EV_COLL_START, cur); alg += 1; }
@@ -604,8 +605,9 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                     if (used && running && fst == FS_NONE) {
                         bool rel = false;
                         if (!TREE || !tree_cur) {
-                            if (D < K && (D == 0 || Dp >= D)) {
-                                // ring step (i, k = D): m_i -> m_{i+1}, S/p bytes (Q21)
+                            if (D < K && (D < (int)C->nch || Dp >= D - (int)C->nch + 1)) {
+                                // ring step (i, k = D): m_i -> m_{i+1}, S/p bytes (Q21); R25: flat
+                                // chunk index q = D waits for the predecessor's chunk q - nch
                                 rel = true;
                                 flen = rring.len;
                                 hl[0] = hring[0]; hl[1] = hring[1]; hl[2] = hring[2]; hl[3] = hring[3];

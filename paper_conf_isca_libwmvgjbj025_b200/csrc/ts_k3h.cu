@@ -462,8 +462,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             G.running = started = true;
             G.tree_cur = tree_algo && ce.kind == CK_AR;
             G.cS = ce.S;
-            G.chunk = ce.S / (double)G.p;
-            G.K = ce.kind == CK_AR ? 2 * (G.p - 1) : (G.p - 1);
+            G.chunk = ce.S / (double)G.p / (double)C->nch;   // R25
+            G.K = (ce.kind == CK_AR ? 2 * (G.p - 1) : (G.p - 1)) * (int)C->nch;
             G.D = 0;
             G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = false;
             if (G.i == 0) {
@@ -479,7 +479,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             const uint64_t cc = (G.gid << 20) | G.cur;
             bool rel = false;
             if (!G.tree_cur) {
-                if (G.D < G.K && (G.D == 0 || Dp >= G.D)) {
+                if (G.D < G.K && (G.D < (int)C->nch || Dp >= G.D - (int)C->nch + 1)) {   // R25 chunk q waits for q - nch
                     release(a, TR, F, gpu, gpu_of_member(G, (G.i + 1) % G.p), G.chunk,
                             (cc << 32) | ((uint64_t)G.D << 16) | (uint64_t)G.i, t, lats, alg);
                     rel = true;

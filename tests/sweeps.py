@@ -113,3 +113,41 @@ def random_photonic(seed):
                          tp_mode=int(rng.integers(0, 2)), bucket=int(rng.choice([0, 1 << 30]))))
     sw = W.Sweep("phot", tr, topos, W.points_array(pts))
     return sw
+
+
+def random_chunked(seed):
+    """R25 pipelined rings: every ring-collective strategy with 0-8 chunks per step on uniform rings (the
+    K3 ring fast-forward), random asymmetric topologies, a photonic net and 48-64-rank points (CTA kernel)."""
+    rng = np.random.Generator(np.random.PCG64(2500 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 6)), max_ops_per_layer=3, b0=2)
+    topos = [W.ring(8, 50e9, 1e-6), W.ring(16, 100e9, 2e-6), W.star(8, 80e9, 1e-6),
+             W.random_topology(rng, n_gpus=6, n_switch=1, p_edge=0.3), W.perturb(W.ring_graph(8, 90e9, 1e-6), seed),
+             W.photonic(8, ports=2, link_bw=40e9, setup=1e-5, lat=1e-6, buf_slots=1),
+             W.ring(64, 50e9, 1e-6)]
+    pts = []
+    P = W.make_point
+    for _ in range(240):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        st = int(rng.choice([W.ST_DP, W.ST_DDP, W.ST_TP, W.ST_HYBRID]))
+        c = int(rng.integers(0, 9))
+        bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
+        algo = int(rng.integers(0, 2)) if rng.random() < 0.3 else W.ALG_RING
+        full = G == 64 or rng.random() < 0.5   # (on the 64-ring a partial ring closes over > 8 hops: R3 limit)
+        if st in (W.ST_DP, W.ST_DDP):
+            dp = G if full else int(rng.integers(2, G + 1))
+            pts.append(P(ti, st, dp=dp, B=dp * 2, algo=algo, bw=bw, lat=lat, chunks=c,
+                         bucket=int(rng.choice([0, 1 << 12, 1 << 30]))))
+        elif st == W.ST_TP:
+            tpd = G if full else int(rng.integers(2, G + 1))
+            pts.append(P(ti, st, tp=tpd, B=2, algo=algo, bw=bw, lat=lat, chunks=c, tp_mode=int(rng.integers(0, 2))))
+        else:
+            while True:
+                dp, tpd, pp = int(rng.integers(1, 5)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 3))
+                if dp * tpd * pp <= G and pp <= tr.n_layers:
+                    break
+            m = int(rng.integers(1, 3))
+            pts.append(P(ti, st, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m * 2, algo=algo, bw=bw, lat=lat, chunks=c,
+                         bucket=int(rng.choice([0, 1 << 12, 1 << 30])), tp_mode=int(rng.integers(0, 2))))
+    pts.append(P(0, W.ST_DDP, dp=8, B=16, chunks=17))   # R25 limit -> BAD_CONFIG
+    return W.Sweep("chunked", tr, topos, W.points_array(pts))

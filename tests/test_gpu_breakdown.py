@@ -64,6 +64,10 @@ def test_breakdown_random_hybrid(ctx, seed):
     _check(ctx, S.random_hybrid(seed))
 
 
+def test_breakdown_chunked_ring(ctx):
+    _check(ctx, S.random_chunked(0))
+
+
 def test_breakdown_large_points_cta_kernel(ctx):
     _check(ctx, S.large_points(0))
 

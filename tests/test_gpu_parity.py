@@ -275,3 +275,17 @@ def test_first_bucket_rule(ctx):
     got = ctx.run_sweep(sw)
     assert (got["status"] == 0).all()
     check(got, sw, list(range(len(pts))))
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_chunked_ring(ctx, seed):
+    """R25 pipelined rings (0-8 chunks per step) in every kernel that runs ring collectives -- warp
+    segments with and without the uniform-ring fast-forward, the hybrid kernel, photonic flows and a
+    64-rank CTA point -- against the oracle point by point."""
+    sw = S.random_chunked(seed)
+    got = ctx.run_sweep(sw)
+    assert got["status"][-1] == W.PT_BAD_CONFIG
+    assert (got["status"][:-1] == 0).sum() > 200
+    # HYBRID DP groups strided over the 64-ring may close over > 8 hops: the documented R3 kernel limit
+    assert (got["status"] == W.PT_TOO_LARGE).sum() <= 10
+    check(got, sw, list(range(len(sw.points))), allow_too_large=True)
