@@ -763,7 +763,7 @@ static cudaError_t enqueue_k1_k2(triosim_ctx *ctx, Sweep &S, Trace &T, cudaStrea
     if (e != cudaSuccess) return e;
     if (!S.pipe_list.empty()) ctx->n_k2++;
     e = launch_k2_hybrid(S.d_cls.p, S.d_hyb_list.p, (uint32_t)S.hyb_list.size(), T.dev, S.d_plans.p, S.d_stages.p,
-                         S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, st);
+                         S.d_hst.p, S.d_hents.p, S.d_hsends.p, S.d_recvs.p, S.d_colls.p, S.d_scr_u64.p, S.d_dur.p, st);
     if (e != cudaSuccess) return e;
     if (!S.hyb_list.empty()) ctx->n_k2++;
     return cudaSuccess;

@@ -63,10 +63,12 @@ struct StageInfo {
     uint64_t dst_mask;        // stages this stage sends to (route check)
 };
 struct StageEnt {
+    double dur;       // t' of the operator (K2 copy of K1b's dur[op]): the compute fold reads one array
     uint32_t op;
     uint16_t nsend, nrecv;
     uint32_t recv_off;
-    uint32_t pad;
+    uint32_t run;     // entries from here on (within this phase list) that one start folds (R16): the
+                      // next one has no receive and none before the last has a send
 };
 struct SendEnt {
     double bytes;
@@ -90,11 +92,14 @@ struct HStage {
     uint32_t pad;
 };
 struct HEnt {                 // per stage op entry (hybrid): the PIPE entry plus TP / DP hooks
+    double dur;                  // t' of the operator (K2 copy of K1b's dur[op]) for the compute fold
     uint32_t op;
     uint16_t nsend, nrecv;
     uint32_t recv_off;
     uint16_t tp_nsig, dp_nsig;   // TP collectives triggered (every instance); DP buckets (instance 0)
     int32_t tpw;                 // TP collective to wait for: (phase << 24) | index, or -1
+    uint32_t run, run0;          // fold run lengths from here within the phase list (R16) for micro-batch
+                                 // instances j > 0 / j == 0 (DP triggers only signal on instance 0)
     uint32_t pad;
 };
 struct HSend {
@@ -193,7 +198,8 @@ cudaError_t launch_k2_pipe(ClassDesc *cls, const uint32_t *list, uint32_t n, con
                            RecvEnt *recvs, unsigned long long *scratch_u64, cudaStream_t s);
 cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
                              const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
-                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, cudaStream_t s);
+                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch_u64, const double *dur,
+                             cudaStream_t s);
 // K3 variants: a.bd != nullptr selects the breakdown-recording (BD) instantiation, a.tl_cnt != nullptr the
 // timeline-recording (LOG) one
 cudaError_t launch_k3(int W, int mode, const K3Args &a, int grid, cudaStream_t s);   // ts_k3.cu

@@ -734,28 +734,31 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         if (ok) {
                             if (en.nrecv) EV(EV_TASK_START, ((uint64_t)gpu << 40) | q);
                             run_start = pos;
-                            const double *du = a.dur + C->dur_off;
-                            const double d0 = du[en.op];
-                            double te = t + d0;
-                            if constexpr (LOG) tl_task(gpu, pos, en.op, j, t, te);
-                            busy = busy + d0;
-                            uint32_t ns = en.nsend;
-                            q++;
-                            while (ns == 0 && q < nprog) {
-                                if (q < m * SI.nF) { P = 0; idx = q % SI.nF; }
-                                else if (q < m * (SI.nF + SI.nB)) { P = 1; idx = (q - m * SI.nF) % SI.nB; }
-                                else { P = 2; idx = q - m * (SI.nF + SI.nB); }
-                                const StageEnt e2 = a.ents[SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB) + idx];
-                                if (e2.nrecv) break;
-                                const double dd = du[e2.op];
-                                if constexpr (LOG) {
-                                    const uint32_t j2 = P == 0 ? q / SI.nF : P == 1 ? m - 1 - (q - m * SI.nF) / SI.nB : 0;
-                                    tl_task(gpu, q, e2.op, j2, te, te + dd);
+                            // fold (R16): K2's run from the head within its phase list, then on into the
+                            // next lists (micro-batch / phase) while the run ends at a list end without a
+                            // send and the next list's first operator waits for no receive.  One
+                            // sequential fp64 add per operator, over contiguous entries
+                            const StageEnt *L = a.ents + SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB);
+                            uint32_t len = P == 0 ? SI.nF : P == 1 ? SI.nB : SI.nO;
+                            uint32_t n = en.run, i0 = idx;
+                            double te = t;
+                            for (;;) {
+#pragma unroll 4
+                                for (uint32_t k = 0; k < n; k++) {
+                                    const double dd = L[i0 + k].dur;
+                                    if constexpr (LOG) tl_task(gpu, q + k, L[i0 + k].op, j, te, te + dd);
+                                    te = te + dd;
+                                    busy = busy + dd;
                                 }
-                                te = te + dd;
-                                busy = busy + dd;
-                                ns = e2.nsend;
-                                q++;
+                                q += n;
+                                const uint32_t last = i0 + n - 1;
+                                if (L[last].nsend != 0 || last + 1 < len || q >= nprog) break;
+                                if (q < m * SI.nF) { j = q / SI.nF; L = a.ents + SI.ent_off; len = SI.nF; }
+                                else if (q < m * (SI.nF + SI.nB)) { j = m - 1 - (q - m * SI.nF) / SI.nB; L = a.ents + SI.ent_off + SI.nF; len = SI.nB; }
+                                else { j = 0; L = a.ents + SI.ent_off + SI.nF + SI.nB; len = SI.nO; }
+                                i0 = 0;
+                                if (L[0].nrecv) break;
+                                n = L[0].run;
                             }
                             ntask += q - pos;
                             alg += 2 * (q - pos);

@@ -756,22 +756,29 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     if (ok) {
                         if (has_wait(en, P, idx)) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
                         run_start = pos;
-                        const double *du = a.dur + C->dur_off;
-                        double te = t + du[en.op];
-                        if constexpr (LOG) tl_task(gpu, pos, en.op, j, t, te);
-                        busy = busy + du[en.op];
-                        bool sig = has_sig(en, j);
-                        uint32_t q = pos + 1;
-                        while (!sig && q < nprog) {
-                            uint32_t P2, j2, i2;
-                            decode(q, P2, j2, i2);
-                            const HEnt e2 = ent_at(P2, i2);
-                            if (has_wait(e2, P2, i2)) break;
-                            if constexpr (LOG) tl_task(gpu, q, e2.op, j2, te, te + du[e2.op]);
-                            te = te + du[e2.op];
-                            busy = busy + du[e2.op];
-                            sig = has_sig(e2, j2);
-                            q++;
+                        // fold (R16): K2's run from the head within its phase list (run0 for micro-batch
+                        // instance 0), then on into the next lists while a run ends at a list end
+                        // without a signal and the next list's first operator waits for nothing
+                        const HEnt *L = a.hents + SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB);
+                        uint32_t len = P == 0 ? SI.nF : P == 1 ? SI.nB : SI.nO;
+                        uint32_t n = j == 0 ? en.run0 : en.run, i0 = idx, q = pos;
+                        double te = t;
+                        for (;;) {
+#pragma unroll 4
+                            for (uint32_t k = 0; k < n; k++) {
+                                const double dd = L[i0 + k].dur;
+                                if constexpr (LOG) tl_task(gpu, q + k, L[i0 + k].op, j, te, te + dd);
+                                te = te + dd;
+                                busy = busy + dd;
+                            }
+                            q += n;
+                            const uint32_t last = i0 + n - 1;
+                            if (has_sig(L[last], j) || last + 1 < len || q >= nprog) break;
+                            decode(q, P, j, i0);
+                            L = a.hents + SI.ent_off + (P == 0 ? 0 : P == 1 ? SI.nF : SI.nF + SI.nB);
+                            len = P == 0 ? SI.nF : P == 1 ? SI.nB : SI.nO;
+                            if (has_wait(L[0], P, 0)) break;
+                            n = j == 0 ? L[0].run0 : L[0].run;
                         }
                         ntask += q - pos;
                         alg += 2 * (q - pos);

@@ -366,11 +366,12 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_pipe(ClassDesc *cls, const uin
                 }
             }
             StageEnt en;
+            en.dur = dur[C.dur_off + o];
             en.op = o;
             en.nsend = (uint16_t)nsend;
             en.nrecv = 0;
             en.recv_off = 0;
-            en.pad = 0;
+            en.run = 1;
             ents[eoff[P] + ei[P]++] = en;
         }
     }
@@ -408,6 +409,15 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_pipe(ClassDesc *cls, const uin
             }
             en.nrecv = (uint16_t)nr;
         }
+        // pass 4: fold run lengths per phase list, back to front
+        const uint32_t base[3] = {si.ent_off, si.ent_off + si.nF, si.ent_off + si.nF + si.nB};
+        const uint32_t len[3] = {si.nF, si.nB, si.nO};
+        for (int P = 0; P < 3; P++)
+            for (int e = (int)len[P] - 2; e >= 0; e--) {
+                StageEnt &x = ents[base[P] + e];
+                const StageEnt &y = ents[base[P] + e + 1];
+                x.run = (x.nsend == 0 && y.nrecv == 0) ? y.run + 1 : 1;
+            }
     }
 }
 
@@ -436,7 +446,7 @@ __device__ __forceinline__ int tp_kind_dev(uint32_t role, uint32_t phase, uint8_
 __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const uint32_t *list, TraceDev T,
                                                          const uint32_t *plan_pool, StageInfo *stages, HStage *hst,
                                                          HEnt *ents, HSend *sends, RecvEnt *recvs, CollEnt *colls,
-                                                         unsigned long long *scratch) {
+                                                         unsigned long long *scratch, const double *dur) {
     ClassDesc &C = cls[list[blockIdx.x]];
     __shared__ uint16_t s_stage[K2P_MAX_LAYERS];
     __shared__ uint32_t s_cnt[64][6];
@@ -567,6 +577,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                 }
             }
             HEnt en;
+            en.dur = dur[C.dur_off + o];
+            en.run = en.run0 = 1;
             en.op = o;
             en.nsend = (uint16_t)nsend;
             en.nrecv = 0;
@@ -670,6 +682,23 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
             en.nrecv = (uint16_t)nr;
             en.tpw = tpw;
         }
+        {
+            // fold run lengths per phase list, back to front (K3h's has_wait / has_sig, R16): entry e
+            // folds e + 1 when e signals nothing and e + 1 waits for nothing; run0 counts DP triggers
+            // as signals (micro-batch instance 0)
+            const uint32_t base[3] = {si.ent_off, si.ent_off + si.nF, si.ent_off + si.nF + si.nB};
+            const uint32_t len[3] = {si.nF, si.nB, si.nO};
+            const bool dpw = dp > 1 && hs.ndp > 0;
+            for (int P = 0; P < 3; P++)
+                for (int e = (int)len[P] - 2; e >= 0; e--) {
+                    HEnt &x = ents[base[P] + e];
+                    const HEnt &y = ents[base[P] + e + 1];
+                    const bool yw = y.nrecv > 0 || y.tpw >= 0 || (P == 2 && (uint32_t)(e + 1) == hs.first_opt && dpw);
+                    const bool xs = x.nsend > 0 || x.tp_nsig > 0;
+                    x.run = (!xs && !yw) ? y.run + 1 : 1;
+                    x.run0 = (!xs && x.dp_nsig == 0 && !yw) ? y.run0 + 1 : 1;
+                }
+        }
         if (tp > 1) {
             const uint32_t scnt = si.SF + si.SB + si.SO;
             for (uint32_t q = 0; q < scnt; q++) {
@@ -733,9 +762,10 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
 
 cudaError_t launch_k2_hybrid(ClassDesc *cls, const uint32_t *list, uint32_t n, const TraceDev &T,
                              const uint32_t *plan_pool, StageInfo *stages, HStage *hst, HEnt *ents, HSend *sends,
-                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch, cudaStream_t s) {
+                             RecvEnt *recvs, CollEnt *colls, unsigned long long *scratch, const double *dur,
+                             cudaStream_t s) {
     if (n == 0) return cudaSuccess;
-    k2_hybrid<<<n, K2P_THREADS, 0, s>>>(cls, list, T, plan_pool, stages, hst, ents, sends, recvs, colls, scratch);
+    k2_hybrid<<<n, K2P_THREADS, 0, s>>>(cls, list, T, plan_pool, stages, hst, ents, sends, recvs, colls, scratch, dur);
     return cudaGetLastError();
 }
 
