@@ -112,7 +112,7 @@ enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 enum { CAT_INPUT = 0, CAT_WEIGHT = 1, CAT_WGRAD = 2, CAT_ACT = 3, CAT_AGRAD = 4, CAT_OTHER = 5 };
 enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4 };
 enum { TPM_PAPER = 0, TPM_MEGATRON = 1 };
-enum { ALG_RING = 0, ALG_TREE = 1 };
+enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2 };
 enum { ROLE_NONE = 0, ROLE_COL = 1, ROLE_ROW = 2, ROLE_LOCAL = 3, ROLE_GATHER = 4 };
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 #define OPF_BATCH_SCALED 1u
@@ -330,7 +330,46 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
         if (prev_done && g_dep(G, sb, prev_done[i])) return -1;
     }
     IVec fl = {0}; /* all flows of this collective */
-    if (algo == ALG_RING || kind != CK_AR) {
+    if (algo == ALG_REDBCAST && kind == CK_AR) {
+        /* R26 AllReduce as NCCL-style ring Reduce to member 0 followed by ring Broadcast from member 0
+         * ("reduce, scatter, and gather"), each a chain along the ring pipelined in nch chunks of
+         * S/nch.  Member i sends its flows one at a time (R25's single send engine) to m_(i+1): first
+         * its reduce chunks (i != 0), then its broadcast chunks (i != p-1); q = own send index.
+         *   reduce chunk j of i: after its own previous send; for i >= 2 after reduce chunk j of i-1
+         *     arrived (i = 1 starts the chain at the collective start);
+         *   broadcast chunk j of 0: after reduce chunk j of p-1 arrived (the reduced chunk is at 0);
+         *   broadcast chunk j of i >= 1: after its own previous send and broadcast chunk j of i-1. */
+        int **id = (int **)malloc(sizeof(int *) * (size_t)(p > 0 ? p : 1));
+        if (!id) return -1;
+        for (int i = 0; i < p; i++) {
+            id[i] = (int *)malloc(sizeof(int) * (size_t)(2 * nch));
+            if (!id[i]) return -1;
+        }
+        /* creation order: reduce chain (members 1..p-1, chunk-major), then broadcast chain (0..p-2) */
+        for (int j = 0; j < nch && p > 1; j++)
+            for (int i = 1; i < p; i++) {
+                int f = add_flow(G, members[i], members[(i + 1) % p], S / (double)nch, coll_flow_code(c, j, i), 0);
+                if (f < 0) return -1;
+                id[i][j] = f;
+                iv_push(&fl, f);
+                if (j == 0 && i == 1) g_dep(G, f, sb);
+                if (j > 0) g_dep(G, f, id[i][j - 1]);
+                if (i >= 2) g_dep(G, f, id[i - 1][j]);
+            }
+        for (int j = 0; j < nch && p > 1; j++)
+            for (int i = 0; i < p - 1; i++) {
+                int q = (i != 0 ? nch : 0) + j;
+                int f = add_flow(G, members[i], members[i + 1], S / (double)nch, coll_flow_code(c, q, i), 0);
+                if (f < 0) return -1;
+                id[i][q] = f;
+                iv_push(&fl, f);
+                if (q > 0) g_dep(G, f, id[i][q - 1]);
+                if (i == 0) g_dep(G, f, id[p - 1][j]);
+                else g_dep(G, f, id[i - 1][(i - 1 != 0 ? nch : 0) + j]);
+            }
+        for (int i = 0; i < p; i++) free(id[i]);
+        free(id);
+    } else if (algo != ALG_TREE || kind != CK_AR) {
         /* ring: K steps; flow (i,k) goes m_i -> m_(i+1); released at start if k == 0,
          * else when (i-1,k-1) [predecessor's chunk arrived] and (i,k-1) [own previous
          * send] are both delivered (reading Q21).
@@ -548,7 +587,7 @@ static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
 /* ------------------------------------------------------------------ */
 static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
                        int have_plan) {
-    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_TREE ||
+    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_REDBCAST ||
         pt->ring_chunks > 16) return PT_BAD_CONFIG;   /* R25: at most 16 chunks per ring step */
     if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
         return PT_BAD_CONFIG;
