@@ -150,6 +150,8 @@ typedef struct {
 #define TRIOSIM_TP_MEGATRON 1
 #define TRIOSIM_ALGO_RING 0
 #define TRIOSIM_ALGO_TREE 1
+#define TRIOSIM_ALGO_REDBCAST 2   /* AllReduce as ring Reduce to member 0 + ring Broadcast from it, pipelined in
+                                     ring_chunks chunks (R26); AllGather / ReduceScatter stay rings */
 
 typedef struct {
     uint32_t topo;

@@ -30,7 +30,11 @@
  * Parity pins (tests/test_oracle_*.py): closed forms CF1-CF14 (DESIGN.md
  * "Pins"), brute-force routing and partitioning, max-min invariants of the
  * progressive filling, and an exact-rational Python re-simulation of exported
- * task graphs.  Unpinned: absolute accuracy vs real hardware (P:244-300,
+ * task graphs.  Extensions R20-R26 (photonic network, per-layer breakdown,
+ * timeline, DDP first bucket, pipelined ring, reduce + broadcast AllReduce)
+ * carry their own pins (tests/test_oracle_{photonic,breakdown,timeline,
+ * closed_forms,chunked_ring,reduce_broadcast}.py).
+ * Unpinned: absolute accuracy vs real hardware (P:244-300,
  * needs the paper's traces and machines) -- "parity unpinned" for that only.
  */
 #include <stdint.h>

@@ -467,7 +467,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto setst = [&](int st) { S->status[i] = st; };
         // R3, in order
         if (pt.topo >= n_topos) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
-        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 1 || pt.ring_chunks > 16) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 2 || pt.ring_chunks > 16) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
         if (!(pt.bw_scale > 0.0) || std::isinf(pt.bw_scale) || !(pt.lat_scale >= 0.0) || std::isinf(pt.lat_scale)) {
             setst(TRIOSIM_PT_BAD_CONFIG);
             continue;

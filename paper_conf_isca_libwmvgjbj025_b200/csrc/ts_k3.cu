@@ -154,6 +154,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     double bstart = 0.0, cbusy = 0.0;
     uint32_t cur = 0;
     bool running = false, tree_cur = false, tree_algo = false, ring_fast = false, ring_uni = false;
+    bool rb_algo = false, rb_cur = false;   // R26: AllReduce as ring Reduce + ring Broadcast chains
     bool ring_ff = false;   // uniform ring whose lanes also share one route latency: ring fast-forward
 #ifdef TS_WATCHDOG
     unsigned int wd_iter = 0;
@@ -162,7 +163,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     long long pf_ff = 0, pf_t0 = 0;
     unsigned int pf_gen = 0, pf_entries = 0;
 #endif
-    int K = 0;
+    int K = 0, Kp = 0;   // this lane's / its ring predecessor's sends in the running collective
     double cS = 0.0, chunk = 0.0;
     // ---- per-lane state ----
     bool used = false;
@@ -255,6 +256,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 ncoll = C->n_coll;
                 m = C->m;
                 tree_algo = TREE && C->algo == TRIOSIM_ALGO_TREE;
+                rb_algo = COLL && C->algo == TRIOSIM_ALGO_REDBCAST;
                 if constexpr (BD) bd_cat = !COLL ? 2u : C->strategy == TRIOSIM_TP ? 0u : 1u;
                 t = 0.0;
                 tmix = mix64(0ull);
@@ -380,14 +382,14 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
         const long long pf_a = clock64();
 #endif
         if constexpr (COLL && !LOG) {
-            if (__any_sync(FULL, have && running && ring_ff && !tree_cur)) {
+            if (__any_sync(FULL, have && running && ring_ff && !tree_cur && !rb_cur)) {
                 const double tc = seg_min_shfl<W>(used && cst == CS_RUN ? t_end : dinf());
                 const int Dseg = __shfl_sync(FULL, D, sbase);
                 // segment-uniform copies (every used lane holds the same values; unused lanes follow them)
                 const double rbw0 = __shfl_sync(FULL, rbw, sbase), L0 = __shfl_sync(FULL, Lring, sbase);
                 const bool okl = !used || (fst == FS_LAT && t_act == t && D == Dseg && flen > 0);
                 const bool allok = (__ballot_sync(FULL, okl) & smask) == smask;   // (every lane votes)
-                const bool ok = allok && have && running && ring_ff && !tree_cur && chunk > 0.0 && Dseg < K && t < tc;
+                const bool ok = allok && have && running && ring_ff && !tree_cur && !rb_cur && chunk > 0.0 && Dseg < K && t < tc;
                 if (ok) {
 #ifdef TS_PROF
                     pf_entries++;
@@ -565,7 +567,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                     if (used && running && !ldone) {
                         bool dn;
                         if (!TREE || !tree_cur) {
-                            dn = D == K && Dp == K;
+                            dn = D == K && Dp == Kp;
                         } else {
                             const bool ku = (c1 >= p || ((upm >> c1) & 1u)) && (c2 >= p || ((upm >> c2) & 1u));
                             const bool kd = (c1 >= p || ((dnm >> c1) & 1u)) && (c2 >= p || ((dnm >> c2) & 1u));
@@ -597,6 +599,15 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         // R25: nch chunks of S / p / nch per ring step, sent one at a time (q = k nch + j)
                         chunk = ce.S / (double)p / (double)C->nch;
                         K = ((ce.kind == CK_AR) ? 2 * (p - 1) : (p - 1)) * (int)C->nch;
+                        Kp = K;
+                        rb_cur = rb_algo && ce.kind == CK_AR;
+                        if (rb_cur) {
+                            // R26: reduce chunks (members != 0), then broadcast chunks (members != p-1)
+                            const int c = (int)C->nch, pl = li == 0 ? p - 1 : li - 1;
+                            chunk = ce.S / (double)c;
+                            K = (li != 0 ? c : 0) + (li != p - 1 ? c : 0);
+                            Kp = (pl != 0 ? c : 0) + (pl != p - 1 ? c : 0);
+                        }
                         D = 0;
                         ldone = uprel = upd = dnrel = dnd = false;
                         if (li == 0) { EV(EV_COLL_START, cur); alg += 1; }
@@ -605,7 +616,17 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                     if (used && running && fst == FS_NONE) {
                         bool rel = false;
                         if (!TREE || !tree_cur) {
-                            if (D < K && (D < (int)C->nch || Dp >= D - (int)C->nch + 1)) {
+                            const int c = (int)C->nch;
+                            bool go;
+                            if (!rb_cur) {
+                                go = D < K && (D < c || Dp >= D - c + 1);
+                            } else if (li != 0 && D < c) {   // R26 reduce chunk D: after the predecessor's
+                                go = li == 1 || (!started && Dp >= D + 1);   // (member 1 starts the chain;
+                            } else {                          // Dp is the previous collective's at its start)
+                                const int j = D - (li != 0 ? c : 0);   // broadcast chunk j
+                                go = D < K && !started && Dp >= (li == 0 || li == 1 ? 0 : c) + j + 1;
+                            }
+                            if (go) {
                                 // ring step (i, k = D): m_i -> m_{i+1}, S/p bytes (Q21); R25: flat
                                 // chunk index q = D waits for the predecessor's chunk q - nch
                                 rel = true;

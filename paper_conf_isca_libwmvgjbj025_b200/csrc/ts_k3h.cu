@@ -92,7 +92,8 @@ struct Group {
     uint64_t gid;
     uint32_t ncoll, trig, donec, cur;
     bool running, tree_cur, ldone, uprel, upd, dnrel, dnd, fup;
-    int K, D;
+    bool rb_cur;              // R26: the running AllReduce is a ring Reduce + ring Broadcast
+    int K, D, Kp;             // this member's / its predecessor's sends in the running collective
     double cS, chunk;
     uint32_t flow_deliv;      // deliveries of this group's flows (for counts)
     double bd_t0;             // R22 (BD): start time of the running collective
@@ -403,7 +404,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         G.ncoll = ncoll;
         G.trig = G.donec = G.cur = 0;
         G.running = G.tree_cur = G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = G.fup = false;
-        G.K = G.D = 0;
+        G.K = G.D = G.Kp = 0;
+        G.rb_cur = false;
         G.cS = G.chunk = 0.0;
         G.flow_deliv = 0;
         G.bd_t0 = 0.0;
@@ -427,7 +429,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         if (G.member && G.running && !G.ldone) {
             bool dn;
             if (!G.tree_cur) {
-                dn = G.D == G.K && Dp == G.K;
+                dn = G.D == G.K && Dp == G.Kp;
             } else {
                 const bool ku = (c1 >= G.p || mb(upb, c1)) && (c2 >= G.p || mb(upb, c2));
                 const bool kd = (c1 >= G.p || mb(dnb, c1)) && (c2 >= G.p || mb(dnb, c2));
@@ -464,6 +466,15 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             G.cS = ce.S;
             G.chunk = ce.S / (double)G.p / (double)C->nch;   // R25
             G.K = (ce.kind == CK_AR ? 2 * (G.p - 1) : (G.p - 1)) * (int)C->nch;
+            G.Kp = G.K;
+            G.rb_cur = C->algo == TRIOSIM_ALGO_REDBCAST && ce.kind == CK_AR;
+            if (G.rb_cur) {
+                // R26: reduce chunks (members != 0), then broadcast chunks (members != p-1)
+                const int c = (int)C->nch, pl = G.i == 0 ? G.p - 1 : G.i - 1;
+                G.chunk = ce.S / (double)c;
+                G.K = (G.i != 0 ? c : 0) + (G.i != G.p - 1 ? c : 0);
+                G.Kp = (pl != 0 ? c : 0) + (pl != G.p - 1 ? c : 0);
+            }
             G.D = 0;
             G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = false;
             if (G.i == 0) {
@@ -479,7 +490,13 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             const uint64_t cc = (G.gid << 20) | G.cur;
             bool rel = false;
             if (!G.tree_cur) {
-                if (G.D < G.K && (G.D < (int)C->nch || Dp >= G.D - (int)C->nch + 1)) {   // R25 chunk q waits for q - nch
+                const int c = (int)C->nch;
+                bool go;
+                if (!G.rb_cur) go = G.D < G.K && (G.D < c || Dp >= G.D - c + 1);   // R25 chunk q waits for q - nch
+                // R26 (Dp is the previous collective's at this one's start)
+                else if (G.i != 0 && G.D < c) go = G.i == 1 || (!started && Dp >= G.D + 1);   // reduce chunk
+                else go = G.D < G.K && !started && Dp >= (G.i <= 1 ? 0 : c) + (G.D - (G.i != 0 ? c : 0)) + 1;   // broadcast
+                if (go) {
                     release(a, TR, F, gpu, gpu_of_member(G, (G.i + 1) % G.p), G.chunk,
                             (cc << 32) | ((uint64_t)G.D << 16) | (uint64_t)G.i, t, lats, alg);
                     rel = true;

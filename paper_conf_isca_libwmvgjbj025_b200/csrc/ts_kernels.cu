@@ -185,10 +185,11 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
             }
             C.n_coll = nc;
             C.coll_payload = payload;
-            C.need_ring = nc > 0 && C.algo == TRIOSIM_ALGO_RING;
+            C.need_ring = nc > 0 && C.algo != TRIOSIM_ALGO_TREE;
             C.need_tree = nc > 0 && C.algo == TRIOSIM_ALGO_TREE;
             C.n_compute = (uint64_t)C.p * T.n_ops;
-            uint64_t fl = C.algo == TRIOSIM_ALGO_RING ? 2ull * (C.p - 1) * C.p * C.nch : 2ull * (C.p - 1);
+            uint64_t fl = C.algo == TRIOSIM_ALGO_RING ? 2ull * (C.p - 1) * C.p * C.nch
+                        : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (C.p - 1) * C.nch : 2ull * (C.p - 1);
             C.n_flows = fl * nc;
             C.n_prog_max = T.n_ops;
         }
@@ -223,6 +224,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         payload = payload + S;
                         if (kind == CK_AG) any_ag = 1; else any_ar = 1;
                         if (kind == CK_AR && C.algo == TRIOSIM_ALGO_TREE) nfl += 2ull * (C.p - 1);
+                        else if (kind == CK_AR && C.algo == TRIOSIM_ALGO_REDBCAST) nfl += 2ull * (C.p - 1) * C.nch;
                         else nfl += (kind == CK_AR ? 2ull : 1ull) * (C.p - 1) * C.p * C.nch;
                         nc++;
                     }
@@ -230,7 +232,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
             }
             C.n_coll = nc;
             C.coll_payload = payload;
-            C.need_ring = any_ag || (any_ar && C.algo == TRIOSIM_ALGO_RING);
+            C.need_ring = any_ag || (any_ar && C.algo != TRIOSIM_ALGO_TREE);
             C.need_tree = any_ar && C.algo == TRIOSIM_ALGO_TREE;
             C.n_compute = (uint64_t)C.p * T.n_ops;
             C.n_flows = nfl;
@@ -736,7 +738,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     const uint32_t kind = colls[hs.tcol_off + e].kind;
                     const uint64_t reps = e < hs.TF + hs.TB ? m : 1;
                     const uint64_t per = kind == CK_AG ? (uint64_t)(tp - 1) * tp * C.nch
-                                       : C.algo == TRIOSIM_ALGO_TREE ? 2ull * (tp - 1) : 2ull * (tp - 1) * tp * C.nch;
+                                       : C.algo == TRIOSIM_ALGO_TREE ? 2ull * (tp - 1)
+                                       : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (tp - 1) * C.nch : 2ull * (tp - 1) * tp * C.nch;
                     nflow += reps * per;
                     ncoll += reps;
                     if (kind == CK_AG) any_ag = 1; else any_ar = 1;
@@ -746,7 +749,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
             for (int t = 0; t < tp; t++)
                 for (uint32_t b = 0; b < HS[s].ndp; b++) {
                     payload = payload + colls[HS[s].dcol_off + b].S;
-                    nflow += C.algo == TRIOSIM_ALGO_TREE ? 2ull * (dp - 1) : 2ull * (dp - 1) * dp * C.nch;
+                    nflow += C.algo == TRIOSIM_ALGO_TREE ? 2ull * (dp - 1)
+                           : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (dp - 1) * C.nch : 2ull * (dp - 1) * dp * C.nch;
                     ncoll++;
                     any_ar = 1;
                 }
@@ -755,7 +759,7 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
         C.n_coll = (uint32_t)ncoll;
         C.coll_payload = payload;
         C.n_prog_max = pmax;
-        C.need_ring = any_ag || (any_ar && C.algo == TRIOSIM_ALGO_RING);
+        C.need_ring = any_ag || (any_ar && C.algo != TRIOSIM_ALGO_TREE);
         C.need_tree = any_ar && C.algo == TRIOSIM_ALGO_TREE;
     }
 }

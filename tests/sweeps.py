@@ -151,3 +151,40 @@ def random_chunked(seed):
                          bucket=int(rng.choice([0, 1 << 12, 1 << 30])), tp_mode=int(rng.integers(0, 2))))
     pts.append(P(0, W.ST_DDP, dp=8, B=16, chunks=17))   # R25 limit -> BAD_CONFIG
     return W.Sweep("chunked", tr, topos, W.points_array(pts))
+
+
+def random_redbcast(seed):
+    """R26 AllReduce as ring Reduce + ring Broadcast (0-6 chunks) for DP / DDP / TP / HYBRID on uniform and
+    asymmetric rings, a star, random graphs, a photonic net and 64-rank points (CTA kernel)."""
+    rng = np.random.Generator(np.random.PCG64(2600 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(3, 6)), max_ops_per_layer=3, b0=2)
+    topos = [W.ring(8, 50e9, 1e-6), W.ring(16, 100e9, 2e-6), W.star(8, 80e9, 1e-6),
+             W.random_topology(rng, n_gpus=6, n_switch=1, p_edge=0.3), W.perturb(W.ring_graph(8, 90e9, 1e-6), seed),
+             W.photonic(8, ports=2, link_bw=40e9, setup=1e-5, lat=1e-6, buf_slots=1),
+             W.ring(64, 50e9, 1e-6)]
+    pts = []
+    P = W.make_point
+    for _ in range(200):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        st = int(rng.choice([W.ST_DP, W.ST_DDP, W.ST_TP, W.ST_HYBRID]))
+        c = int(rng.integers(0, 7))
+        bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
+        full = G == 64 or rng.random() < 0.5
+        kw = dict(algo=W.ALG_REDBCAST, bw=bw, lat=lat, chunks=c)
+        if st in (W.ST_DP, W.ST_DDP):
+            dp = G if full else int(rng.integers(1, G + 1))
+            pts.append(P(ti, st, dp=dp, B=dp * 2, bucket=int(rng.choice([0, 1 << 12, 1 << 30])), **kw))
+        elif st == W.ST_TP:
+            tpd = G if full else int(rng.integers(1, G + 1))
+            pts.append(P(ti, st, tp=tpd, B=2, tp_mode=int(rng.integers(0, 2)), **kw))
+        else:
+            while True:
+                dp, tpd, pp = int(rng.integers(1, 5)), int(rng.choice([1, 2, 4])), int(rng.integers(1, 3))
+                if dp * tpd * pp <= G and pp <= tr.n_layers:
+                    break
+            m = int(rng.integers(1, 3))
+            pts.append(P(ti, st, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m * 2, bucket=int(rng.choice([0, 1 << 12, 1 << 30])),
+                         tp_mode=int(rng.integers(0, 2)), **kw))
+    pts.append(P(0, W.ST_DDP, dp=8, B=16, algo=3))   # unknown algorithm -> BAD_CONFIG
+    return W.Sweep("redbcast", tr, topos, W.points_array(pts))

@@ -68,6 +68,10 @@ def test_breakdown_chunked_ring(ctx):
     _check(ctx, S.random_chunked(0))
 
 
+def test_breakdown_reduce_broadcast(ctx):
+    _check(ctx, S.random_redbcast(0))
+
+
 def test_breakdown_large_points_cta_kernel(ctx):
     _check(ctx, S.large_points(0))
 

@@ -289,3 +289,15 @@ def test_chunked_ring(ctx, seed):
     # HYBRID DP groups strided over the 64-ring may close over > 8 hops: the documented R3 kernel limit
     assert (got["status"] == W.PT_TOO_LARGE).sum() <= 10
     check(got, sw, list(range(len(sw.points))), allow_too_large=True)
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_reduce_broadcast(ctx, seed):
+    """R26 AllReduce as ring Reduce + ring Broadcast chains (0-6 chunks) in the warp, hybrid, photonic and
+    64-rank CTA kernels, against the oracle point by point."""
+    sw = S.random_redbcast(seed)
+    got = ctx.run_sweep(sw)
+    assert got["status"][-1] == W.PT_BAD_CONFIG
+    assert (got["status"][:-1] == 0).sum() > 170
+    assert (got["status"] == W.PT_TOO_LARGE).sum() <= 10
+    check(got, sw, list(range(len(sw.points))), allow_too_large=True)

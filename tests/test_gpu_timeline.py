@@ -77,7 +77,8 @@ def _sample(n, k, seed):
 
 
 @pytest.mark.parametrize("gen,seed", [(S.random_small, 0), (S.random_small, 1), (S.random_hybrid, 0),
-                                      (S.random_photonic, 0), (S.random_photonic, 1), (S.random_chunked, 0)])
+                                      (S.random_photonic, 0), (S.random_photonic, 1), (S.random_chunked, 0),
+                                      (S.random_redbcast, 0)])
 def test_timeline_random_sweeps(ctx, gen, seed):
     sw = gen(seed)
     assert _check(ctx, sw, _sample(len(sw.points), 40, 70 + seed)) > 15
