@@ -116,7 +116,7 @@ enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 enum { CAT_INPUT = 0, CAT_WEIGHT = 1, CAT_WGRAD = 2, CAT_ACT = 3, CAT_AGRAD = 4, CAT_OTHER = 5 };
 enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4 };
 enum { TPM_PAPER = 0, TPM_MEGATRON = 1 };
-enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2 };
+enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2, ALG_DBTREE = 3 };
 enum { ROLE_NONE = 0, ROLE_COL = 1, ROLE_ROW = 2, ROLE_LOCAL = 3, ROLE_GATHER = 4 };
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 #define OPF_BATCH_SCALED 1u
@@ -316,6 +316,45 @@ static uint64_t p2p_flow_code(uint32_t x, int j, int dst) {
 }
 
 /*
+ * One binary-heap tree AllReduce over the members (R10 tree, reading Q25): heap position h holds
+ * member h (mirror = 0) or member p-1-h (mirror = 1, R27's second tree).  The child at position h
+ * reduces to its parent carrying Sx once all of its own children's reduces arrived (leaves at the
+ * collective start sb); the parent broadcasts back once it holds the result (the root once both of
+ * its children's reduces arrived).  Flow code step = 2*mirror + {0 up, 1 down}, member = the
+ * child's member index.  Appends the flows to fl.
+ */
+static int heap_tree(Graph *G, uint64_t c, const int *members, int p, int mirror, double Sx, int sb, IVec *fl) {
+    int *up = (int *)malloc(sizeof(int) * (size_t)(p > 0 ? p : 1)), *dn = (int *)malloc(sizeof(int) * (size_t)(p > 0 ? p : 1));
+    if (!up || !dn) { free(up); free(dn); return -1; }
+    for (int h = 0; h < p; h++) up[h] = dn[h] = -1;
+#define MEM_AT(h) (mirror ? p - 1 - (h) : (h))
+    for (int h = p - 1; h >= 1; h--) {
+        up[h] = add_flow(G, members[MEM_AT(h)], members[MEM_AT((h - 1) / 2)], Sx, coll_flow_code(c, 2 * mirror, MEM_AT(h)), 0);
+        if (up[h] < 0) { free(up); free(dn); return -1; }
+        iv_push(fl, up[h]);
+    }
+    for (int h = 1; h < p; h++) {
+        dn[h] = add_flow(G, members[MEM_AT((h - 1) / 2)], members[MEM_AT(h)], Sx, coll_flow_code(c, 2 * mirror + 1, MEM_AT(h)), 0);
+        if (dn[h] < 0) { free(up); free(dn); return -1; }
+        iv_push(fl, dn[h]);
+    }
+#undef MEM_AT
+    for (int h = 1; h < p; h++) {
+        int nchild = 0;
+        for (int ch = 2 * h + 1; ch <= 2 * h + 2 && ch < p; ch++) { g_dep(G, up[h], up[ch]); nchild++; }
+        if (nchild == 0) g_dep(G, up[h], sb);
+        int par = (h - 1) / 2;
+        if (par == 0) {
+            for (int ch = 1; ch <= 2 && ch < p; ch++) g_dep(G, dn[h], up[ch]);
+        } else {
+            g_dep(G, dn[h], dn[par]);
+        }
+    }
+    free(up); free(dn);
+    return 0;
+}
+
+/*
  * One collective (R10; P:87-89 ring AllReduce, P:174 reduce/scatter/gather,
  * P:192 ring tasks handed to the network model).  members[] are GPU nodes in
  * ring order.  trig[i] = task whose completion makes member i's input ready;
@@ -373,7 +412,7 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
             }
         for (int i = 0; i < p; i++) free(id[i]);
         free(id);
-    } else if (algo != ALG_TREE || kind != CK_AR) {
+    } else if ((algo != ALG_TREE && algo != ALG_DBTREE) || kind != CK_AR) {
         /* ring: K steps; flow (i,k) goes m_i -> m_(i+1); released at start if k == 0,
          * else when (i-1,k-1) [predecessor's chunk arrived] and (i,k-1) [own previous
          * send] are both delivered (reading Q21).
@@ -400,33 +439,21 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
                 }
             }
         free(id);
+    } else if (algo == ALG_DBTREE) {
+        /* R27 double binary tree AllReduce (NCCL's trees, P:174 / P:398; reading in DESIGN.md R27): the
+         * payload is split in two halves S/2; half A runs the R10 tree over heap position = member
+         * index, half B the same tree over the mirrored positions (member i at position p-1-i), so
+         * for even p every interior node of one tree is a leaf of the other.  Both trees run at
+         * once; flow steps 0/1 (A up/down) and 2/3 (B up/down), member field = the child. */
+        if (heap_tree(G, c, members, p, 0, S / 2.0, sb, &fl) || heap_tree(G, c, members, p, 1, S / 2.0, sb, &fl)) {
+            iv_free(&fl);
+            return -1;
+        }
     } else {
         /* tree AllReduce (extension, reading Q25): binary heap over member index,
          * reduce i -> parent(i) carrying S once all children's reduces arrived;
          * broadcast parent(i) -> i once parent(i) holds the result. */
-        int *up = (int *)malloc(sizeof(int) * (size_t)p), *dn = (int *)malloc(sizeof(int) * (size_t)p);
-        if (!up || !dn) { free(up); free(dn); return -1; }
-        for (int i = 0; i < p; i++) up[i] = dn[i] = -1;
-        for (int i = p - 1; i >= 1; i--) {
-            up[i] = add_flow(G, members[i], members[(i - 1) / 2], S, coll_flow_code(c, 0, i), 0);
-            iv_push(&fl, up[i]);
-        }
-        for (int i = 1; i < p; i++) {
-            dn[i] = add_flow(G, members[(i - 1) / 2], members[i], S, coll_flow_code(c, 1, i), 0);
-            iv_push(&fl, dn[i]);
-        }
-        for (int i = 1; i < p; i++) {
-            int nch = 0;
-            for (int ch = 2 * i + 1; ch <= 2 * i + 2 && ch < p; ch++) { g_dep(G, up[i], up[ch]); nch++; }
-            if (nch == 0) g_dep(G, up[i], sb);
-            int par = (i - 1) / 2;
-            if (par == 0) {
-                for (int ch = 1; ch <= 2 && ch < p; ch++) g_dep(G, dn[i], up[ch]);
-            } else {
-                g_dep(G, dn[i], dn[par]);
-            }
-        }
-        free(up); free(dn);
+        if (heap_tree(G, c, members, p, 0, S, sb, &fl)) { iv_free(&fl); return -1; }
     }
     for (int i = 0; i < p; i++) {
         done[i] = add_barrier(G, 0, 0);
@@ -591,7 +618,7 @@ static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
 /* ------------------------------------------------------------------ */
 static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
                        int have_plan) {
-    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_REDBCAST ||
+    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_DBTREE ||
         pt->ring_chunks > 16) return PT_BAD_CONFIG;   /* R25: at most 16 chunks per ring step */
     if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
         return PT_BAD_CONFIG;

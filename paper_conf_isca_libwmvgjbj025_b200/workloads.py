@@ -62,7 +62,7 @@ ROLE_NONE, ROLE_COL, ROLE_ROW, ROLE_LOCAL, ROLE_GATHER = 0, 1, 2, 3, 4
 OPF_BATCH_SCALED = 1
 ST_DP, ST_DDP, ST_TP, ST_PP, ST_HYBRID = range(5)
 TPM_PAPER, TPM_MEGATRON = 0, 1
-ALG_RING, ALG_TREE, ALG_REDBCAST = 0, 1, 2
+ALG_RING, ALG_TREE, ALG_REDBCAST, ALG_DBTREE = 0, 1, 2, 3
 PT_OK, PT_BAD_BATCH, PT_BAD_DEGREES, PT_NO_ROUTE, PT_TOO_LARGE, PT_DEADLOCK, PT_BAD_PLAN, PT_BAD_CONFIG = range(8)
 
 MiB = 1 << 20

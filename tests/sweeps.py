@@ -186,5 +186,5 @@ def random_redbcast(seed):
             m = int(rng.integers(1, 3))
             pts.append(P(ti, st, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m * 2, bucket=int(rng.choice([0, 1 << 12, 1 << 30])),
                          tp_mode=int(rng.integers(0, 2)), **kw))
-    pts.append(P(0, W.ST_DDP, dp=8, B=16, algo=3))   # unknown algorithm -> BAD_CONFIG
+    pts.append(P(0, W.ST_DDP, dp=8, B=16, algo=4))   # unknown algorithm -> BAD_CONFIG
     return W.Sweep("redbcast", tr, topos, W.points_array(pts))
