@@ -152,6 +152,8 @@ typedef struct {
 #define TRIOSIM_ALGO_TREE 1
 #define TRIOSIM_ALGO_REDBCAST 2   /* AllReduce as ring Reduce to member 0 + ring Broadcast from it, pipelined in
                                      ring_chunks chunks (R26); AllGather / ReduceScatter stay rings */
+/* coll_algo 3 (double binary tree, R27) is defined by the oracle only; this library version
+   reports TRIOSIM_PT_BAD_CONFIG for it, as for any coll_algo > 2. */
 
 typedef struct {
     uint32_t topo;
