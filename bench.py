@@ -210,7 +210,7 @@ def main():
     ap.add_argument("--ref-points", type=int, default=300)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--points", type=int, default=0,
                     help="simulate a seeded prefix of this many points of the sweep (0 = config default)")
     ap.add_argument("--shard", action="store_true",
@@ -321,7 +321,8 @@ def main():
     assert out_host.tobytes() == res.tobytes()
     h2d = (sw.trace.ops.nbytes + sw.trace.tensors.nbytes + sw.trace.io.nbytes + sw.points.nbytes +
            sum(t.links.nbytes + t.ring_order.nbytes for t in sw.topos))
-    e2e_ms = float(np.max(e2e_t)) * 1e3 if e2e_t else float("nan")
+    # mean over consecutive steps (what a user calling the API in a loop sees), then max over ranks
+    e2e_ms = float(np.mean(e2e_t)) * 1e3 if e2e_t else float("nan")
     e2e_points = total_points
     if world > 1:
         t = torch.tensor([e2e_ms], device="cuda", dtype=torch.float64)
@@ -392,7 +393,8 @@ def main():
                              "frac": round(alg_b / (k3 / 1e3) / 1e9 / float(pk.get("hbm_gbs", 6650.0)), 7),
                              "algorithmic_bytes_per_launch": int(alg_b), "peak_source": src},
             "e2e": {"value": round(e2e_points / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(n * rec), "ms_per_step": round(e2e_ms, 3)},
+                    "d2h_bytes_per_step": int(n * rec), "ms_per_step": round(e2e_ms, 3),
+                    "steps": len(e2e_t), "timing": "wall clock, mean of consecutive API calls, max over ranks"},
             "gpu_launches": int(gpu_launches),
             "setup_ms": setup_ms,
             "clocks": clk.summary(),
