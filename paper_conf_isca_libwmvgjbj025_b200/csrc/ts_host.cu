@@ -13,6 +13,8 @@
 #include <cstdio>
 #include <cstring>
 #include <map>
+#include <mutex>
+#include <cstdlib>
 #include <memory>
 #include <string>
 #include <tuple>
@@ -23,16 +25,84 @@ using namespace ts;
 
 namespace {
 
+// Device block cache: load_trace / build_sweep / release run every step of a user's loop (bench.py's
+// e2e), and each of them would otherwise pay ~50 cudaMalloc / cudaFree (cudaFree synchronises the
+// device).  Freed blocks are kept per (device, capacity) and reused for a request of at least half
+// their size.  A block is only returned to the cache where no launch can still use it: release() and
+// set_breakdown() synchronise the device first, and a reallocated buffer synchronises before it gives
+// its old block back (what cudaFree did implicitly).  TS_NO_BLOCK_CACHE=1 turns the cache off.
+struct BlockCache {
+    std::mutex mu;
+    std::multimap<std::pair<int, size_t>, void *> blocks;
+    size_t bytes = 0;
+    static constexpr size_t kMaxBytes = size_t(4) << 30;
+    bool on = getenv("TS_NO_BLOCK_CACHE") == nullptr || atoi(getenv("TS_NO_BLOCK_CACHE")) == 0;
+    cudaError_t get(void **p, size_t want, size_t *cap, int *dev) {
+        cudaError_t e = cudaGetDevice(dev);
+        if (e != cudaSuccess) return e;
+        want = (want + 511) & ~size_t(511);
+        if (on) {
+            std::lock_guard<std::mutex> g(mu);
+            auto it = blocks.lower_bound({*dev, want});
+            if (it != blocks.end() && it->first.first == *dev && it->first.second <= 2 * want) {
+                *p = it->second;
+                *cap = it->first.second;
+                bytes -= *cap;
+                blocks.erase(it);
+                return cudaSuccess;
+            }
+        }
+        *cap = want;
+        e = cudaMalloc(p, want);
+        if (e == cudaErrorMemoryAllocation && on) {   // give the cached blocks of this device back, retry
+            cudaGetLastError();
+            trim(*dev);
+            e = cudaMalloc(p, want);
+        }
+        return e;
+    }
+    void put(void *p, size_t cap, int dev) {
+        if (on) {
+            std::lock_guard<std::mutex> g(mu);
+            if (bytes + cap <= kMaxBytes) {
+                blocks.insert({{dev, cap}, p});
+                bytes += cap;
+                return;
+            }
+        }
+        cudaFree(p);
+    }
+    void trim(int dev) {
+        std::lock_guard<std::mutex> g(mu);
+        for (auto it = blocks.begin(); it != blocks.end();) {
+            if (it->first.first == dev) { cudaFree(it->second); bytes -= it->first.second; it = blocks.erase(it); }
+            else ++it;
+        }
+    }
+};
+BlockCache &block_cache() {
+    static BlockCache *c = new BlockCache();   // never destroyed: no CUDA calls during static teardown
+    return *c;
+}
+
 template <class T>
 struct DevBuf {
     T *p = nullptr;
-    size_t n = 0;
-    ~DevBuf() { if (p) cudaFree(p); }
+    size_t n = 0, cap = 0;
+    int dev = 0;
+    ~DevBuf() { if (p) block_cache().put(p, cap, dev); }
     cudaError_t alloc(size_t count) {
-        if (p) { cudaFree(p); p = nullptr; }
+        if (p) {
+            cudaDeviceSynchronize();   // a launch may still use the old block (cudaFree synchronised too)
+            block_cache().put(p, cap, dev);
+            p = nullptr;
+        }
         n = count;
         if (count == 0) count = 1;
-        return cudaMalloc((void **)&p, count * sizeof(T));
+        void *q = nullptr;
+        cudaError_t e = block_cache().get(&q, count * sizeof(T), &cap, &dev);
+        p = e == cudaSuccess ? (T *)q : nullptr;
+        return e;
     }
     cudaError_t upload(const std::vector<T> &v) {
         cudaError_t e = alloc(v.size());
@@ -42,6 +112,7 @@ struct DevBuf {
 };
 
 struct Trace {
+    ~Trace() { cudaDeviceSynchronize(); }   // before the members' blocks go back to the cache
     std::vector<triosim_op> ops;
     std::vector<triosim_tensor> ts;
     std::vector<uint32_t> io;
@@ -63,6 +134,7 @@ struct Trace {
 };
 
 struct Sweep {
+    ~Sweep() { cudaDeviceSynchronize(); }   // before the members' blocks go back to the cache
     int trace_handle = -1;
     uint64_t n_pts = 0;
     std::vector<int32_t> status;            // host-side status per point (-1 = simulate)
@@ -204,7 +276,9 @@ void triosim_destroy(triosim_ctx *ctx) {
         if (ctx->t_mid[i]) cudaEventDestroy(ctx->t_mid[i]);
         if (ctx->t_end[i]) cudaEventDestroy(ctx->t_end[i]);
     }
+    const int dev = ctx->device;
     delete ctx;
+    block_cache().trim(dev);   // destroy gives the device memory back
 }
 
 const char *triosim_last_error(const triosim_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
