@@ -14,6 +14,7 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <chrono>
 #include <cstdlib>
 #include <memory>
 #include <string>
@@ -80,6 +81,18 @@ struct BlockCache {
         }
     }
 };
+// TS_HOST_TIMING=1: wall time of build_sweep's host phases on stderr (diagnostics only)
+struct PhaseTimer {
+    bool on = getenv("TS_HOST_TIMING") != nullptr;
+    std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+    void mark(const char *what) {
+        if (!on) return;
+        auto n = std::chrono::steady_clock::now();
+        fprintf(stderr, "[ts_host] %-14s %8.3f ms\n", what, std::chrono::duration<double, std::milli>(n - t).count());
+        t = n;
+    }
+};
+
 BlockCache &block_cache() {
     static BlockCache *c = new BlockCache();   // never destroyed: no CUDA calls during static teardown
     return *c;
@@ -508,11 +521,13 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         for (uint32_t k = 0; k < plans->n_plans; k++)
             if (plans->off[k + 1] < plans->off[k]) return fail(ctx, TRIOSIM_EINVAL, "bad plan offsets");
 
+    PhaseTimer PT;
     std::vector<HostTopo> HT(n_topos);
     for (uint32_t i = 0; i < n_topos; i++) {
         triosim_status st = prep_topology(ctx, topos[i], i, HT[i]);
         if (st != TRIOSIM_OK) return st;
     }
+    PT.mark("topologies");
     auto S = std::make_unique<Sweep>();
     S->trace_handle = trace_id;
     S->n_pts = n_pts;
@@ -675,6 +690,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         S->cost[i] = cost;
     }
 
+    PT.mark("points");
     // per-class pools
     uint32_t dur_n = 0, hook_n = 0, coll_n = 0, scr_i = 0, scr_u = 0, stage_n = 0, ent_n = 0, send_n = 0, recv_n = 0;
     uint32_t hst_n = 0, hent_n = 0, hsend_n = 0;
@@ -712,6 +728,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.scratch_off = scr_u; scr_u += NT;
         }
     }
+    PT.mark("class pools");
     // topologies to the device
     std::vector<TopoDev> td(n_topos);
     std::vector<double> bw, lat;
@@ -755,6 +772,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             }
         }
     }
+    PT.mark("routes");
     CK(S->d_topo.upload(td));
     CK(S->d_bw.upload(bw));
     CK(S->d_lat.upload(lat));
@@ -785,6 +803,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     std::memset(res0.data(), 0, sizeof(triosim_result) * n_pts);
     for (uint64_t i = 0; i < n_pts; i++) res0[i].status = S->status[i] < 0 ? TRIOSIM_PT_OK : S->status[i];
     CK(S->d_res.upload(res0));
+    PT.mark("uploads");
     // work lists per width, most expensive first (LPT)
     std::vector<uint64_t> order;
     for (uint64_t i = 0; i < n_pts; i++) if (S->status[i] < 0) order.push_back(i);
@@ -811,7 +830,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     CK(S->d_counter.alloc(N_GROUPS));
     CK(S->d_alg.alloc(1));
     CK(cudaMemset(S->d_alg.p, 0, sizeof(unsigned long long)));
+    PT.mark("work lists");
     CK(cudaDeviceSynchronize());
+    PT.mark("sync");
     int h = ctx->next_handle++;
     T.n_sweeps++;
     ctx->sweeps[h] = std::move(S);
