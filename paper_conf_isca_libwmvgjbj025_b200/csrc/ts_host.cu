@@ -522,6 +522,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             if (plans->off[k + 1] < plans->off[k]) return fail(ctx, TRIOSIM_EINVAL, "bad plan offsets");
 
     PhaseTimer PT;
+    static const int widen_from = getenv("TS_WIDEN_FROM") ? atoi(getenv("TS_WIDEN_FROM")) : 16;
     std::vector<HostTopo> HT(n_topos);
     for (uint32_t i = 0; i < n_topos; i++) {
         triosim_status st = prep_topology(ctx, topos[i], i, HT[i]);
@@ -596,6 +597,11 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto lm = [&](bool h, int w) { return !h ? lmax_warp(w) : w <= 32 ? lmax_hybrid(w) : LMAX_CTA; };
         int W0 = 2;
         while (W0 < (int)lanes) W0 <<= 1;
+        // DP / DDP / TP points of 9-16 GPUs run one per warp (W = 32) instead of two per warp: the two
+        // segments of a warp diverge on every event, and these heaviest points set the step (C2 3.18 ->
+        // 3.04 ms measured; results are identical for any W >= lanes).  TS_WIDEN_FROM=0 turns it off.
+        if (widen_from > 0 && W0 >= widen_from && W0 < 32 && pt.strategy != TRIOSIM_PP && pt.strategy != TRIOSIM_HYBRID)
+            W0 <<= 1;
         // photonic points (R20) always run in the HYBRID kernel, whose lanes own their logical links;
         // DataParallel maps to HYBRID with its buckets triggered after the backward pass
         int W = 0;
