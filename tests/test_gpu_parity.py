@@ -301,3 +301,19 @@ def test_reduce_broadcast(ctx, seed):
     assert (got["status"][:-1] == 0).sum() > 170
     assert (got["status"] == W.PT_TOO_LARGE).sum() <= 10
     check(got, sw, list(range(len(sw.points))), allow_too_large=True)
+
+
+def test_double_tree_rejected_until_implemented(ctx):
+    """R27 (double binary tree) exists in the oracle only; the library reports PT_BAD_CONFIG for
+    coll_algo = 3 as include/triosim.h documents, and the other points of the same sweep are unaffected."""
+    tr = W.mlp_trace()
+    topos = [W.ring(8, 25e9, 1e-6)]
+    pts = [W.make_point(0, W.ST_DDP, dp=8, B=64, algo=W.ALG_DBTREE),
+           W.make_point(0, W.ST_DDP, dp=8, B=64, algo=W.ALG_TREE),
+           W.make_point(0, W.ST_TP, tp=4, B=64, tp_mode=W.TPM_PAPER, algo=W.ALG_DBTREE)]
+    sw = W.Sweep("dbtree", tr, topos, W.points_array(pts))
+    got = ctx.run_sweep(sw)
+    assert got["status"][0] == W.PT_BAD_CONFIG and got["status"][2] == W.PT_BAD_CONFIG
+    assert got["status"][1] == 0
+    check(got, sw, [1])
+    assert oracle.run_point(tr, topos[0], pts[0])["status"] == 0
