@@ -811,12 +811,34 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     CK(S->d_res.upload(res0));
     PT.mark("uploads");
     // work lists per width, most expensive first (LPT)
-    std::vector<uint64_t> order;
-    for (uint64_t i = 0; i < n_pts; i++) if (S->status[i] < 0) order.push_back(i);
-    std::stable_sort(order.begin(), order.end(), [&](uint64_t a, uint64_t b) {
-        if (S->cost[a] != S->cost[b]) return S->cost[a] > S->cost[b];
-        return pdesc[a].cls < pdesc[b].cls;
+    // The cost estimate is a function of the structural class, so the order (cost desc, class, index)
+    // is a counting sort by class followed by a sort of the classes (was a 10k-point stable_sort, 0.6 ms).
+    // The order only schedules work; results do not depend on it.
+    const size_t ncls = S->classes.size();
+    std::vector<double> ccost(ncls, -1.0);
+    std::vector<uint64_t> cstart(ncls + 1, 0);
+    for (uint64_t i = 0; i < n_pts; i++)
+        if (S->status[i] < 0) {
+            const uint32_t c = pdesc[i].cls;
+            cstart[c + 1]++;
+            if (S->cost[i] > ccost[c]) ccost[c] = S->cost[i];
+        }
+    std::vector<uint32_t> corder(ncls);
+    for (uint32_t c = 0; c < ncls; c++) corder[c] = c;
+    std::sort(corder.begin(), corder.end(), [&](uint32_t a, uint32_t b) {
+        if (ccost[a] != ccost[b]) return ccost[a] > ccost[b];
+        return a < b;
     });
+    std::vector<uint64_t> cpos(ncls, 0);
+    {
+        uint64_t off = 0;
+        for (uint32_t c : corder) { cpos[c] = off; off += cstart[c + 1]; }
+        cstart.back() = off;   // total simulated points
+    }
+    std::vector<uint64_t> order(cstart.back());
+    for (uint64_t i = 0; i < n_pts; i++)
+        if (S->status[i] < 0) order[cpos[pdesc[i].cls]++] = i;
+    PT.mark("wl sort");
     for (uint64_t i : order) {
         const int g = N_MODES * w_index(S->width[i]) + S->mode[i];
         S->work[g].push_back((uint32_t)i);
@@ -829,10 +851,12 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     }
     for (int g = 0; g < N_GROUPS; g++)
         if (S->lmax[g] || S->pmax[g]) S->occ[g] = k3h_max_blocks_per_sm(W_OF[g / N_MODES], S->lmax[g], S->pmax[g]);
+    PT.mark("wl lists");
     for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
         CK(S->d_work_tmp[w].alloc(S->work[w].size()));
     }
+    PT.mark("wl uploads");
     CK(S->d_counter.alloc(N_GROUPS));
     CK(S->d_alg.alloc(1));
     CK(cudaMemset(S->d_alg.p, 0, sizeof(unsigned long long)));
