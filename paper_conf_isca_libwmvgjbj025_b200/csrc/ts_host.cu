@@ -552,6 +552,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         }
     }
 
+    decltype(cls_of)::key_type last_key{};
+    uint32_t last_c = 0;
+    bool have_last = false;
     for (uint64_t i = 0; i < n_pts; i++) {
         triosim_point pt = pts[i];
         auto setst = [&](int st) { S->status[i] = st; };
@@ -638,9 +641,13 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto key = std::make_tuple((int)pt.strategy + (dp_after ? 100 : 0), (int)lanes, (int)b_loc, key_mode, hyb ? (int)dp : 0,
                                    hyb ? (int)tpd : 0, key_algo * 32 + key_nch, key_bucket, key_first, key_m,
                                    (mode == MODE_PIPE || hyb) ? plan_key : -2);
-        auto ci = cls_of.find(key);
+        // consecutive points of a sweep usually share their class (bandwidth / latency scales are not part
+        // of it): reuse the previous lookup
         uint32_t c;
-        if (ci == cls_of.end()) {
+        auto ci = (have_last && key == last_key) ? cls_of.end() : cls_of.find(key);
+        if (have_last && key == last_key) {
+            c = last_c;
+        } else if (ci == cls_of.end()) {
             ClassDesc cd;
             std::memset(&cd, 0, sizeof cd);
             cd.mode = mode;
@@ -672,6 +679,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         } else {
             c = ci->second;
         }
+        last_key = key;
+        last_c = c;
+        have_last = true;
         PointDesc &pd = pdesc[i];
         pd.bw_scale = pt.bw_scale;
         pd.lat_scale = pt.lat_scale;
