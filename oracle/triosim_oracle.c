@@ -1191,7 +1191,6 @@ static uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     return z ^ (z >> 31);
 }
-static uint64_t emix(uint64_t v) { return (v ^ (v >> 29)) * 0xbf58476d1ce4e5b9ull; }
 static uint64_t dbits(double d) { uint64_t u; memcpy(&u, &d, 8); return u; }
 
 /* ------------------------------------------------------------------ */
@@ -1360,8 +1359,8 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
             }                                                                \
         }                                                                    \
     } while (0)
-/* R19: order hash = sum over events of emix(mix64(bits(t)) ^ (kind << 60 | code)) */
-#define EVENT(kind, code) do { acc += emix(tmix ^ (((uint64_t)(kind) << 60) | (code))); nev++; } while (0)
+/* R19: order hash = sum mod 2^64 over events of mix64(mix64(bits(t)) ^ (kind << 60 | code)) */
+#define EVENT(kind, code) do { acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (code))); nev++; } while (0)
 
         for (;;) {
             uint64_t acc = 0;

@@ -30,8 +30,6 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     return z ^ (z >> 31);
 }
-// per-event mix: one xorshift-multiply round (the per-instant time hash tmix is a full mix64)
-__device__ __forceinline__ uint64_t emix(uint64_t v) { return (v ^ (v >> 29)) * 0xbf58476d1ce4e5b9ull; }
 __device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
 
 #ifndef TS_SEGMIN_REDUX
@@ -219,7 +217,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
 
 #define EV(kind, code)                                                  \
     do {                                                                \
-        acc += emix(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code))); \
+        acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code))); \
         nev = true;                                                     \
     } while (0)
 
@@ -443,10 +441,10 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 const uint64_t k = (uint64_t)(D0 + (i >> 1));
                                 uint64_t term;
                                 if ((i & 1) == 0) {
-                                    term = emix(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
+                                    term = mix64(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
                                 } else {
-                                    term = emix(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16))) +
-                                           emix(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
+                                    term = mix64(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16))) +
+                                           mix64(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
                                 }
                                 add += i < n ? term : 0ull;
                             }

@@ -26,7 +26,6 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     return z ^ (z >> 31);
 }
-__device__ __forceinline__ uint64_t emix(uint64_t v) { return (v ^ (v >> 29)) * 0xbf58476d1ce4e5b9ull; }
 __device__ __forceinline__ double dinf() { return __longlong_as_double(0x7ff0000000000000ll); }
 
 template <int W>
@@ -380,7 +379,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
 
 #define EV(kind, code)                                                        \
     do {                                                                      \
-        acc += emix(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code)));   \
+        acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code)));   \
         nev = true;                                                           \
     } while (0)
 
