@@ -295,6 +295,15 @@ triosim_status triosim_timeline(triosim_ctx *ctx, int32_t sweep_id, uint64_t poi
                                 uint64_t task_cap, triosim_flow_rec *flows, uint64_t flow_cap, uint64_t *n_tasks,
                                 uint64_t *n_flows);
 
+/* Automatic GPipe stage plan (R8; P:188 user-specified stages, "automatically assigns layers to
+ * GPUs to balance workloads"), the one build_sweep uses for stage_plan = -1: the contiguous split of the
+ * trace's layers (n_layers = 1 + the largest FWD layer id) into n_stages stages minimising the largest
+ * stage cost -- the left fold in layer order of the per-layer sums of time_s -- ties broken towards the
+ * lexicographically smallest first_layer vector.  Host-only (no context, no device); writes n_stages
+ * first layers (first_layer[0] = 0).  Errors: EINVAL (NULL pointers, no ops, n_stages == 0 or
+ * > n_layers, an op layer >= n_layers, a negative / non-finite time). */
+triosim_status triosim_stage_partition(const triosim_trace_desc *t, uint32_t n_stages, uint32_t *first_layer);
+
 /* Kernel launch counters since the context was created (K1, K2, K3 launches), for the bench. */
 triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3);
 

@@ -242,6 +242,8 @@ static triosim_status fail(triosim_ctx *c, triosim_status st, const char *fmt, .
 
 extern "C" {
 
+static std::vector<uint32_t> stage_partition(const triosim_op *ops, uint32_t n_ops, uint32_t L, uint32_t S);
+
 triosim_status triosim_create(int cuda_device, triosim_ctx **out) {
     if (!out) return TRIOSIM_EINVAL;
     *out = nullptr;
@@ -295,6 +297,19 @@ void triosim_destroy(triosim_ctx *ctx) {
 }
 
 const char *triosim_last_error(const triosim_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+triosim_status triosim_stage_partition(const triosim_trace_desc *t, uint32_t n_stages, uint32_t *first_layer) {
+    if (!t || !first_layer || !t->ops || t->n_ops == 0 || n_stages == 0) return TRIOSIM_EINVAL;
+    uint32_t L = 0;
+    for (uint32_t o = 0; o < t->n_ops; o++)
+        if (t->ops[o].phase == TRIOSIM_PHASE_FWD) L = std::max(L, t->ops[o].layer + 1);
+    if (n_stages > L) return TRIOSIM_EINVAL;
+    for (uint32_t o = 0; o < t->n_ops; o++)
+        if (t->ops[o].layer >= L || !(t->ops[o].time_s >= 0.0) || std::isinf(t->ops[o].time_s)) return TRIOSIM_EINVAL;
+    const std::vector<uint32_t> fl = stage_partition(t->ops, t->n_ops, L, n_stages);
+    std::copy(fl.begin(), fl.end(), first_layer);
+    return TRIOSIM_OK;
+}
 
 triosim_status triosim_launch_counts(const triosim_ctx *ctx, uint64_t *k1, uint64_t *k2, uint64_t *k3) {
     if (!ctx) return TRIOSIM_EINVAL;
@@ -389,39 +404,73 @@ triosim_status triosim_load_trace(triosim_ctx *ctx, const triosim_trace_desc *t,
 // ------------------------------------------------------------------------------------------
 // host helpers: routing (BFS, ascending neighbours, first discovery) and the PP partition
 // ------------------------------------------------------------------------------------------
-static std::vector<uint32_t> auto_partition(const Trace &T, int S) {
-    const int L = (int)T.n_layers;
+// R8 automatic stage plan ("automatically assigns layers to GPUs to balance workloads"): the
+// contiguous partition of the L layers into S stages that minimises the largest stage cost -- the
+// left fold, in layer order, of the per-layer sums of trace times -- with ties broken towards the
+// lexicographically smallest vector of first layers.  Computed here as (1) a binary search of the
+// optimum V over the sorted candidate stage costs, with feasibility "the suffix from layer i splits
+// into s stages of cost <= V" decided per V by interval reachability (a stage starting at i may end
+// anywhere up to the last layer whose fold from i stays <= V, because adding non-negative times
+// never decreases a fold), then (2) a left-to-right pass taking each stage's end as early as the
+// rest stays feasible.  O(S L log L) per plan; pinned by exhaustive search (tests/test_abi_cpu.py).
+static std::vector<uint32_t> stage_partition(const triosim_op *ops, uint32_t n_ops, uint32_t L, uint32_t S) {
     std::vector<double> lc(L, 0.0);
-    for (const auto &op : T.ops) lc[op.layer] = lc[op.layer] + op.time_s;
-    std::vector<double> cost((size_t)L * L, 0.0);
-    for (int a = 0; a < L; a++) {
+    for (uint32_t o = 0; o < n_ops; o++) lc[ops[o].layer] = lc[ops[o].layer] + ops[o].time_s;
+    // fold[a][b - a]: left fold of lc[a..b]; end[a] (per V): last b with fold(a, b) <= V
+    std::vector<std::vector<double>> fold(L);
+    std::vector<double> cand;
+    cand.reserve((size_t)L * (L + 1) / 2);
+    for (uint32_t a = 0; a < L; a++) {
+        fold[a].resize(L - a);
         double s = 0.0;
-        for (int b = a; b < L; b++) { s = s + lc[b]; cost[(size_t)a * L + b] = s; }
+        for (uint32_t b = a; b < L; b++) { s = s + lc[b]; fold[a][b - a] = s; cand.push_back(s); }
     }
-    std::vector<double> best((size_t)(S + 1) * (L + 1), INFINITY);
-    auto B = [&](int s, int i) -> double & { return best[(size_t)s * (L + 1) + i]; };
-    for (int i = 0; i < L; i++) B(1, i) = cost[(size_t)i * L + L - 1];
-    for (int s = 2; s <= S; s++)
-        for (int i = 0; i + s <= L; i++) {
-            double b = INFINITY;
-            for (int j = i + 1; L - j >= s - 1; j++) {
-                double a = cost[(size_t)i * L + j - 1], r = B(s - 1, j);
-                double mx = a > r ? a : r;
-                if (mx < b) b = mx;
-            }
-            B(s, i) = b;
+    std::sort(cand.begin(), cand.end());
+    cand.erase(std::unique(cand.begin(), cand.end()), cand.end());
+    // ok[s][i] (s = 1..S, i = 0..L): layers i..L-1 split into exactly s non-empty stages of cost <= V
+    std::vector<std::vector<char>> ok(S + 1, std::vector<char>(L + 1, 0));
+    std::vector<uint32_t> last(L);
+    std::vector<uint32_t> pre(L + 2);
+    auto feasible = [&](double V) -> bool {
+        for (uint32_t a = 0; a < L; a++) {
+            // fold(a, .) is non-decreasing: binary search the last end that fits
+            const auto &f = fold[a];
+            last[a] = (uint32_t)(std::upper_bound(f.begin(), f.end(), V) - f.begin());   // stages a..a+last-1 fit
         }
-    const double V = B(S, 0);
+        for (uint32_t i = 0; i <= L; i++) ok[1][i] = (i < L && last[i] == L - i);
+        for (uint32_t s = 2; s <= S; s++) {
+            // ok[s][i] = any ok[s-1][j] for j in [i+1, i+last[i]]: prefix counts of ok[s-1]
+            pre[0] = 0;
+            for (uint32_t j = 0; j <= L; j++) pre[j + 1] = pre[j] + (ok[s - 1][j] ? 1u : 0u);
+            for (uint32_t i = 0; i <= L; i++) {
+                ok[s][i] = 0;
+                if (i < L && last[i] >= 1) {
+                    const uint32_t lo = i + 1, hi = i + last[i];   // inclusive
+                    ok[s][i] = pre[hi + 1] - pre[lo] > 0;
+                }
+            }
+        }
+        return ok[S][0] != 0;
+    };
+    size_t lo = 0, hi = cand.size() - 1;   // cand[hi] (the whole fold's max) is always feasible for S <= L
+    while (lo < hi) {
+        const size_t mid = lo + (hi - lo) / 2;
+        if (feasible(cand[mid])) hi = mid; else lo = mid + 1;
+    }
+    feasible(cand[lo]);
     std::vector<uint32_t> fl(S, 0);
-    int i = 0;
-    for (int s = S; s >= 2; s--) {
-        int jj = -1;
-        for (int j = i + 1; L - j >= s - 1; j++)
-            if (cost[(size_t)i * L + j - 1] <= V && B(s - 1, j) <= V) { jj = j; break; }
-        fl[S - s + 1] = (uint32_t)jj;
-        i = jj;
+    uint32_t i = 0;
+    for (uint32_t k = 1; k < S; k++) {
+        const uint32_t rest = S - k;   // stages still to place after this one
+        uint32_t j = i + 1;
+        while (j < L && !(j <= i + last[i] && ok[rest][j])) j++;
+        fl[k] = j;
+        i = j;
     }
     return fl;
+}
+static std::vector<uint32_t> auto_partition(const Trace &T, int S) {
+    return stage_partition(T.ops.data(), (uint32_t)T.ops.size(), T.n_layers, (uint32_t)S);
 }
 
 struct HostTopo {
@@ -623,7 +672,10 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         }
         // photonic tree collectives: a broadcast flow parent -> child lives in the child's lane but needs the
         // parent's logical links (ports are the sender's, R20); not supported by this kernel
-        if (tp.photonic && pt.coll_algo == TRIOSIM_ALGO_TREE && pt.strategy != TRIOSIM_PP) W = 0;
+        // (a class without collective groups -- dp = tp = 1 -- has no tree to run)
+        if (tp.photonic && pt.coll_algo == TRIOSIM_ALGO_TREE && (dp > 1 || tpd > 1)) W = 0;
+        // K2's pipeline / hybrid expansion keeps the layer -> stage map in shared memory (K2P_MAX_LAYERS)
+        if ((pt.strategy == TRIOSIM_PP || pt.strategy == TRIOSIM_HYBRID) && T.n_layers > K2P_MAX_LAYERS) W = 0;
         if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
         const uint32_t mbe = pt.microbatches;   // after a DDP / TP -> HYBRID mapping this is 1
         // structural class

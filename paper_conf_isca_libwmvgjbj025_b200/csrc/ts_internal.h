@@ -225,5 +225,6 @@ constexpr int N_WIDTHS = 10;            // W = 2, 4, 8, 16, 32 (warp segments), 
 constexpr int N_MODES = 4;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 constexpr int MAX_PORTS = 8;            // photonic ports per GPU the hybrid kernel holds (R20)
+constexpr uint32_t K2P_MAX_LAYERS = 2048;   // trace layers the PP / HYBRID expansion (K2) stages in shared memory
 
 }  // namespace ts

@@ -264,7 +264,6 @@ cudaError_t launch_k2_coll(ClassDesc *cls, const uint32_t *list, uint32_t n, con
 // K2 (PIPE): one CTA per GPipe class; thread s builds stage s
 // ------------------------------------------------------------------------------------
 constexpr int K2P_THREADS = 64;
-constexpr int K2P_MAX_LAYERS = 2048;
 
 __global__ void __launch_bounds__(K2P_THREADS) k2_pipe(ClassDesc *cls, const uint32_t *list, TraceDev T,
                                                        const double *dur, const uint32_t *plan_pool,

@@ -20,7 +20,7 @@ LIB_PATH = os.environ.get("TRIOSIM_LIB", os.path.join(HERE, "libtriosim.so"))
 EXPORTS = ["triosim_create", "triosim_destroy", "triosim_last_error", "triosim_load_trace", "triosim_build_sweep",
            "triosim_simulate_batch", "triosim_results", "triosim_release", "triosim_launch_counts",
            "triosim_results_device_ptr", "triosim_work_counters", "triosim_timing", "triosim_timings",
-           "triosim_set_breakdown", "triosim_breakdown", "triosim_timeline"]
+           "triosim_set_breakdown", "triosim_breakdown", "triosim_timeline", "triosim_stage_partition"]
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENOTFOUND", -5: "ERANGE", -6: "EUNSUPPORTED"}
 
@@ -87,6 +87,20 @@ def load_library(path=LIB_PATH):
 
 def _ptr(a):
     return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+def triosim_stage_partition(trace: W.Trace, n_stages: int) -> list:
+    """Automatic GPipe stage plan (R8) as build_sweep computes it: host-only, no device."""
+    L = load_library()
+    ops = np.ascontiguousarray(trace.ops, W.OP_DTYPE)
+    ts = np.ascontiguousarray(trace.tensors, W.TENSOR_DTYPE)
+    io = np.ascontiguousarray(trace.io, np.uint32)
+    d = _TraceDesc(len(ops), len(ts), len(io), int(trace.trace_batch), _ptr(ops), _ptr(ts), _ptr(io))
+    out = np.zeros(max(int(n_stages), 1), np.uint32)
+    st = L.triosim_stage_partition(C.byref(d), int(n_stages), _ptr(out))
+    if st != 0:
+        raise TrioSimError("triosim_stage_partition", st)
+    return [int(x) for x in out[:n_stages]]
 
 
 class Context:

@@ -1,6 +1,6 @@
 """Per-source-line instruction / stall-sample attribution of an ncu capture (run here, no GPU).
 
-    python profiles/sass_lines.py <capture.ncu-rep> <libtriosim.so> <mangled kernel> [top]
+    python profiles/sass_lines.py <capture.ncu-rep | source-page.csv[.gz]> <libtriosim.so> <mangled kernel> [top] [section]
 
 Joins ncu's SASS source page (per-instruction counts, by address order) with nvdisasm -g line
 info of the same cubin, and prints the hottest source lines.
@@ -16,8 +16,12 @@ import tempfile
 
 
 def main(rep, so, fn, top=40, section=None):
-    sass = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                          capture_output=True, text=True).stdout
+    if rep.endswith(".csv.gz") or rep.endswith(".csv"):   # a source page exported on the GPU box
+        import gzip
+        sass = (gzip.open(rep, "rt") if rep.endswith(".gz") else open(rep)).read()
+    else:
+        sass = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                              capture_output=True, text=True).stdout
     allrows = list(csv.reader(io.StringIO(sass)))
     starts = [i for i, r in enumerate(allrows) if r and r[0] == "Kernel Name"] + [len(allrows)]
     rows = None

@@ -66,3 +66,45 @@ def test_product_never_imports_oracle():
             if f.endswith((".py", ".cu", ".h", ".cpp")):
                 s = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in s and "from oracle" not in s and "triosim_oracle" not in s, f
+
+
+# ---------------- the product's automatic stage plan (R8), host-only ----------------
+def _brute_force_plan(tr, S):
+    """Every composition of the layers into S contiguous non-empty stages; the smallest max stage cost
+    (left fold of per-layer sums of trace times), ties -> the lexicographically smallest first layers."""
+    import itertools
+    L = int(tr.n_layers)
+    lc = [0.0] * L
+    for op in tr.ops:
+        lc[int(op["layer"])] = lc[int(op["layer"])] + float(op["time_s"])
+    best = None
+    for cut in itertools.combinations(range(1, L), S - 1):
+        b = (0,) + cut + (L,)
+        worst = 0.0
+        for k in range(S):
+            c = 0.0
+            for l in range(b[k], b[k + 1]):
+                c = c + lc[l]
+            worst = max(worst, c)
+        key = (worst, b[:-1])
+        if best is None or key < best:
+            best = key
+    return list(best[1])
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_stage_partition_matches_exhaustive_search(lib, seed):
+    rng = np.random.Generator(np.random.PCG64(100 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(2, 10)))
+    if seed % 3 == 0:   # ties: equal layer costs
+        tr.ops["time_s"] = 2.0 ** -10
+    for S in range(1, int(tr.n_layers) + 1):
+        assert triosim.triosim_stage_partition(tr, S) == _brute_force_plan(tr, S), (seed, S)
+
+
+def test_stage_partition_rejects_bad_arguments(lib):
+    tr = W.mlp_trace()
+    with pytest.raises(triosim.TrioSimError):
+        triosim.triosim_stage_partition(tr, 0)
+    with pytest.raises(triosim.TrioSimError):
+        triosim.triosim_stage_partition(tr, int(tr.n_layers) + 1)
