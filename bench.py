@@ -1,15 +1,19 @@
 #!/usr/bin/env python
 """Benchmark: simulated design points / s on B200 (BASELINE.json metric), configs[1] workload
-(ResNet-50 DP/DDP sweep, 10,000 points, 2-16 simulated GPUs on an NVLink-style ring).
+(ResNet-50 DDP sweep, 10,000 points, 2-16 simulated GPUs on an NVLink-style ring).
 
 One step = one pass of the whole hot path over the sweep: K1b operator rescale + K2 task-graph
 expansion for every structural class + K3 timeline for every point, results written to device
-memory (and all-gathered over NCCL when N > 1).  Inputs are resident in HBM (built once).
+memory, then (N > 1) one NCCL all-gather of the 112-B records and their scatter into sweep order.
+Inputs are resident in HBM (built once).
 
-    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--config c2|c3|c4|c5|...]
 
-Under torchrun each rank simulates its own full sweep (weak scaling) and the per-point records are
-gathered with one NCCL all_gather per step.  Rank 0 prints one JSON line.
+--gpus N > 1 without torchrun re-launches itself under torch.distributed.run (one process per GPU).
+Multi-GPU: the sweep at N GPUs is configs[1]'s family at N x 10,000 distinct
+points (its bandwidth axis refined N-fold; N = 1 is configs[1] itself), dealt to the ranks by estimated
+cost in snake order -- every point simulated exactly once, per-GPU work fixed (weak scaling).
+--scaling strong instead deals the fixed 10,000-point sweep.  Rank 0 prints one JSON line.
 """
 from __future__ import annotations
 
@@ -34,7 +38,7 @@ UNIT = "points/s"
 CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1, "c5": W.sweep_c5,
            "wafer": W.sweep_wafer}
 DEFAULT_POINTS = {"c5": 296}   # configs[4]'s 966k-point sweep: a seeded prefix (two waves of 1024-thread CTAs)
-WORKLOAD = {"c2": "configs[1]: ResNet-50 DP/DDP, 2-16 simulated GPUs on an NVLink-style ring, 10k-point "
+WORKLOAD = {"c2": "configs[1]: ResNet-50 DDP (data parallel), 2-16 simulated GPUs on an NVLink-style ring, 10k-point "
                   "bandwidth x latency x batch x bucket sweep",
             "c3": "configs[2]: BERT-large Megatron/paper TP 2/4/8, ring/star/mesh/cube-mesh/ring-graph/"
                   "double-ring topologies incl. asymmetric",
@@ -186,18 +190,58 @@ def run_reference(args):
 # ------------------------------------------------------------------------------------------
 # our arm
 # ------------------------------------------------------------------------------------------
+OPS_PER_TASK = 2      # algorithmic fp64 ops per operator instance (rescale + fold)
+OPS_PER_WF_CALL = 80  # algorithmic fp64 ops per water-filling call (|A| <= 16)
+DEFAULT_NBW = {"c2": 25, "c3": 8, "c4": 25, "c5": 25, "wafer": 10}
+
+
+def make_sweep(cfg, scale=1, npts=0):
+    """The config's sweep; scale > 1 refines its bandwidth axis scale-fold (distinct points, same mix)."""
+    f = CONFIGS[cfg]
+    sw = f(n_bw=DEFAULT_NBW[cfg] * scale) if (scale > 1 and cfg in DEFAULT_NBW) else f()
+    if npts and npts < len(sw.points):
+        sw = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[:npts], sw.plans)
+    return sw
+
+
+def algorithmic_fp64(res):
+    """SURVEY 8(d).2's algorithmic fp64 count of the simulated points: 2 per operator instance plus
+    80 per water-filling call (counts from the result records, which the oracle pins)."""
+    ok = res["status"] == 0
+    return int(OPS_PER_TASK * res["n_compute"][ok].astype(np.int64).sum()
+               + OPS_PER_WF_CALL * res["n_wf_calls"][ok].astype(np.int64).sum())
+
+
 def algorithmic_bytes(sw):
-    """Bytes the method must read / write per sweep: the trace tables once
-    per class, per point its descriptor (56 B), its topology's used links and routes, its
-    result record (112 B)."""
+    """SURVEY 8(d).2's algorithmic bytes: per point the trace SoA read once (16 B per operator: time f64,
+    packed flags, layer), the weight-gradient sizes (8 B each), its topology's links (24 B each) and route
+    table (5 B per GPU pair), its descriptor (56 B) and its result record (112 B)."""
     tr = sw.trace
-    trace_b = tr.ops.nbytes + tr.tensors.nbytes + tr.io.nbytes
-    ncls = len({(int(p["strategy"]), int(p["dp"]), int(p["tp"]), int(p["pp"]), int(p["global_batch"]),
-                 int(p["bucket_bytes"]), int(p["microbatches"]), int(p["tp_mode"]), int(p["coll_algo"]))
-                for p in sw.points})
-    per_pt = W.POINT_DTYPE.itemsize + W.RESULT_DTYPE.itemsize
-    topo_b = sum(sw.topos[int(p["topo"])].links.nbytes for p in sw.points)
-    return ncls * trace_b + len(sw.points) * per_pt + topo_b
+    n_wg = int((tr.tensors["category"] == W.CAT_WGRAD).sum())
+    per_trace = 16 * len(tr.ops) + 8 * n_wg
+    topo_b = np.asarray([t.links.nbytes + 5 * t.n_gpus * t.n_gpus for t in sw.topos])
+    return int(len(sw.points) * (per_trace + W.POINT_DTYPE.itemsize + W.RESULT_DTYPE.itemsize)
+               + topo_b[sw.points["topo"].astype(np.int64)].sum())
+
+
+def issue_evidence(cfg):
+    """Warp-instruction counts of the K3 launches of one step from a committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", f"ncu_issue_{cfg}.json")) as f:
+            return json.load(f)
+    except Exception:
+        return None
+
+
+def relaunch(n):
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -213,56 +257,63 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--points", type=int, default=0,
                     help="simulate a seeded prefix of this many points of the sweep (0 = config default)")
-    ap.add_argument("--shard", action="store_true",
-                    help="strong scaling: deal one sweep to the ranks by cost instead of a full sweep per rank")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: N x the sweep (distinct points) over N GPUs; strong: one sweep dealt to N GPUs")
+    ap.add_argument("--sweep-scale", type=int, default=0,
+                    help="bandwidth-axis refinement of the sweep (0 = N for weak scaling, 1 for strong)")
+    ap.add_argument("--dump-records", default="", help="rank 0 writes the sweep-ordered records here")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch(args.gpus))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        print(json.dumps({"error": f"--gpus {args.gpus} but WORLD_SIZE {world}"}), flush=True)
+        sys.exit(2)
 
     import torch
     import torch.distributed as dist
     from paper_conf_isca_libwmvgjbj025_b200 import dist as D, triosim
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    dev_idx = 0 if os.environ.get("TS_SHARE_GPU") == "1" else local   # TS_SHARE_GPU: test-only, ranks share GPU 0
+    torch.cuda.set_device(dev_idx)
+    backend = os.environ.get("TS_DIST_BACKEND", "nccl")
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_idx))
+        else:
+            dist.init_process_group(backend)
 
-    sw = CONFIGS[args.config]()
-    npts = args.points or DEFAULT_POINTS.get(args.config, 0)
-    if npts and npts < len(sw.points):
-        sw = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[:npts], sw.plans)
+    scale = args.sweep_scale or (world if args.scaling == "weak" else 1)
+    sw = make_sweep(args.config, scale, args.points or DEFAULT_POINTS.get(args.config, 0))
     n_sweep = len(sw.points)
-    if args.shard and world > 1:
-        tr = sw.trace
-        wg = tr.tensors[tr.tensors["category"] == W.CAT_WGRAD]
-        costs = D.point_cost(sw.points, len(tr.ops), len(wg), int(wg["bytes_b0"].sum()))
-        maxc = max(D.shard_sizes(n_sweep, world, costs))
-        sw = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[D.shard_points(costs, world, rank)], sw.plans)
-    n = len(sw.points)
-    maxc = maxc if (args.shard and world > 1) else n
-    ctx = triosim.Context(local)
+    plan = D.ShardPlan(D.sweep_cost(sw), world, rank)
+    sub = plan.sub_sweep(sw)
+    n = len(sub.points)
+    ctx = triosim.Context(dev_idx)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    tid = ctx.triosim_load_trace(sw.trace)
+    tid = ctx.triosim_load_trace(sub.trace)
     t1 = time.perf_counter()
-    sid = ctx.triosim_build_sweep(tid, sw.topos, sw.points, sw.plans or None)
+    sid = ctx.triosim_build_sweep(tid, sub.topos, sub.points, sub.plans or None)
     t2 = time.perf_counter()
     setup_ms = {"load_trace": round((t1 - t0) * 1e3, 3), "build_sweep": round((t2 - t1) * 1e3, 3)}
     stream = torch.cuda.Stream()
     rec = W.RESULT_DTYPE.itemsize
-    res_local = torch.zeros(n * rec, dtype=torch.uint8, device="cuda")
+    res_local = torch.zeros(max(n, 1) * rec, dtype=torch.uint8, device="cuda")
+    res_all = torch.zeros(n_sweep * rec, dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
 
     def step():
-        ctx.triosim_simulate_batch(sid, 0, n, stream.cuda_stream)
-        ctx.triosim_results(sid, 0, n, device_ptr=res_local.data_ptr(), stream=stream.cuda_stream)
-        if world > 1:
-            with torch.cuda.stream(stream):
-                D.gather_records(res_local, world, maxc)   # one NCCL all-gather of the records
+        if n:
+            ctx.triosim_simulate_batch(sid, 0, n, stream.cuda_stream)
+            ctx.triosim_results(sid, 0, n, device_ptr=res_local.data_ptr(), stream=stream.cuda_stream)
+        with torch.cuda.stream(stream):
+            plan.gather(res_local[: n * rec], out=res_all)   # one all-gather + scatter into sweep order
 
     for _ in range(args.warmup):
         step()
@@ -270,7 +321,7 @@ def main():
     k0 = ctx.launch_counts()
     ctx.timing(True)
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    with Clocks(local) as clk:
+    with Clocks(dev_idx) as clk:
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
@@ -287,43 +338,48 @@ def main():
     step_ms = [a.elapsed_time(b) for a, b in evs]
     tot_ms, k3_ms = ctx.timings()
     ctx.timing(False)
-    alg_ops = ctx.work_counters(sid)
+    kernel_ops = ctx.work_counters(sid)
     ms = float(np.mean(step_ms))
+    k3 = float(np.mean(k3_ms)) if len(k3_ms) else float("nan")
     if world > 1:
-        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        t = torch.tensor([ms, k3], device="cuda", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-    total_points = n_sweep if (args.shard and world > 1) else n * world
-    value = total_points / (ms / 1e3)
+        ms, k3 = float(t[0].item()), float(t[1].item())
+    value = n_sweep / (ms / 1e3)
     gpu_launches = sum(k1) - sum(k0)
-    res = ctx.triosim_results(sid, 0, n)
+    if world > 1:
+        t = torch.tensor([gpu_launches], device="cuda", dtype=torch.int64)
+        dist.all_reduce(t)
+        gpu_launches = int(t.item())
+    res = res_all.cpu().numpy().view(W.RESULT_DTYPE).copy()
     n_ok = int((res["status"] == 0).sum())
+    if args.dump_records and rank == 0:
+        res.tofile(args.dump_records)
 
-    # end to end through the public API with host buffers: H2D of the trace / topologies / points
-    # from pinned host memory, the full path, D2H of the results, every step
+    # end to end through the public API with host buffers, every step: H2D of this rank's trace / topologies
+    # / points from pinned host memory (load_trace, build_sweep), simulate, results, the all-gather into
+    # sweep order and the D2H of the sweep's records on rank 0 (D.simulate_sharded)
     pin = {k: torch.from_numpy(v.view(np.uint8)).pin_memory().numpy().view(v.dtype) for k, v in
-           (("ops", sw.trace.ops), ("ts", sw.trace.tensors), ("io", sw.trace.io), ("pts", sw.points))}
-    tr_pinned = W.Trace(sw.trace.name, pin["ops"], pin["ts"], pin["io"], sw.trace.trace_batch, sw.trace.n_layers)
+           (("ops", sub.trace.ops), ("ts", sub.trace.tensors), ("io", sub.trace.io), ("pts", sub.points))}
+    sub_pinned = W.Sweep(sub.name, W.Trace(sub.trace.name, pin["ops"], pin["ts"], pin["io"], sub.trace.trace_batch,
+                                           sub.trace.n_layers), sub.topos, pin["pts"], sub.plans)
     e2e_t = []
-    out_host = torch.empty(n * rec, dtype=torch.uint8).pin_memory().numpy().view(W.RESULT_DTYPE)
     for i in range(args.e2e_steps + 1):
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         t0 = time.perf_counter()
-        t2 = ctx.triosim_load_trace(tr_pinned)
-        s2 = ctx.triosim_build_sweep(t2, sw.topos, pin["pts"], sw.plans or None)
-        ctx.triosim_simulate_batch(s2, 0, n, stream.cuda_stream)
-        ctx.triosim_results(s2, 0, n, out=out_host, stream=stream.cuda_stream)
-        ctx.triosim_release(s2)
-        ctx.triosim_release(t2)
+        with torch.cuda.stream(stream):
+            host = D.simulate_sharded(ctx, sw, plan, sub=sub_pinned, host_on_rank0=True)
         dt = time.perf_counter() - t0
         if i > 0:
             e2e_t.append(dt)
-    assert out_host.tobytes() == res.tobytes()
-    h2d = (sw.trace.ops.nbytes + sw.trace.tensors.nbytes + sw.trace.io.nbytes + sw.points.nbytes +
-           sum(t.links.nbytes + t.ring_order.nbytes for t in sw.topos))
-    # mean over consecutive steps (what a user calling the API in a loop sees), then max over ranks
+        if rank == 0:
+            assert host.tobytes() == res.tobytes(), "e2e records differ from the device-timed step"
+    h2d = int(sum((sub.trace.ops.nbytes + sub.trace.tensors.nbytes + sub.trace.io.nbytes + len(plan.shards[r]) *
+                   W.POINT_DTYPE.itemsize + sum(t.links.nbytes + t.ring_order.nbytes for t in sw.topos))
+                  for r in range(world)))
     e2e_ms = float(np.mean(e2e_t)) * 1e3 if e2e_t else float("nan")
-    e2e_points = total_points
     if world > 1:
         t = torch.tensor([e2e_ms], device="cuda", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -331,7 +387,7 @@ def main():
 
     # the p = 8 slice of C2 timed on its own, per-tensor and 25 MiB buckets
     slices = {}
-    if args.config == "c2" and rank == 0 and not args.shard:
+    if args.config == "c2" and world == 1:
         for name, bucket in (("p8_per_tensor", 0), ("p8_bucket_25MiB", 25 << 20)):
             sel = (sw.points["dp"] == 8) & (sw.points["bucket_bytes"] == bucket)
             if not sel.any():
@@ -358,43 +414,53 @@ def main():
 
     if rank == 0:
         pk, src = peaks()
-        k3 = float(np.mean(k3_ms)) if len(k3_ms) else float("nan")
         clock_mhz = float(pk.get("sm_max_mhz", 1965.0))
         peak_ops = N_SMS * FP64_LANES_PER_SM * clock_mhz * 1e6
+        alg_ops = algorithmic_fp64(res) / world          # per rank (one K3 phase), whole sweep / N
         achieved = alg_ops / (k3 / 1e3)
-        traffic = None
-        try:
-            with open(os.path.join(ROOT, "profiles", "k3_ncu_summary.json")) as f:
-                traffic = json.load(f).get(f"dram_bytes_per_launch_{args.config}")
-        except Exception:
-            pass
-        alg_b = algorithmic_bytes(sw)
+        alg_b = algorithmic_bytes(sw) / world
+        iss = issue_evidence(args.config)
+        roof = {"bound": "alu", "kernel": "k3_timeline (K3 phase: every K3 launch of the step)",
+                "achieved": round(achieved / 1e12, 6), "peak": round(peak_ops / 1e12, 3),
+                "unit": "TFLOP/s (fp64, non-tensor)", "frac": round(achieved / peak_ops, 6),
+                "traffic": None if iss is None else iss.get("dram_bytes_per_step"),
+                "traffic_source": None if iss is None else f"profiles/ncu_issue_{args.config}.json ({iss.get('run')})",
+                "k3_ms": round(k3, 4), "alg_fp64_ops_per_launch": int(alg_ops),
+                "alg_derivation": f"SURVEY 8(d).2: {OPS_PER_TASK} x n_compute + {OPS_PER_WF_CALL} x n_wf_calls summed "
+                                  "over the step's points (counts from the result records), / K3 phase time",
+                "kernel_executed_fp64_ops_per_launch": int(kernel_ops),
+                "peak_source": f"{N_SMS} SMs x {FP64_LANES_PER_SM} fp64 lanes x {clock_mhz} MHz (sm_max_mhz {src}; "
+                               "derived, MEASURED_PEAKS.json has no fp64 entry)"}
+        if iss is not None and iss.get("warp_inst_per_step"):
+            ipeak = N_SMS * 4 * clock_mhz * 1e6
+            roof["issue"] = {"warp_inst_per_step": iss["warp_inst_per_step"], "peak_warp_inst_per_s": ipeak,
+                             "frac": round(iss["warp_inst_per_step"] / (k3 / 1e3) / ipeak, 4),
+                             "warps_active_pct": iss.get("warps_active_pct"),
+                             "lane_efficiency": iss.get("lane_efficiency"),
+                             "source": f"profiles/ncu_issue_{args.config}.json ({iss.get('run')}): ncu "
+                                       "smsp__inst_executed.sum over the step's K3 launches / (148 SMs x 4 "
+                                       "schedulers x sm_max_mhz) / measured K3 phase time"}
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "scaling": "strong" if (args.shard and world > 1) else "weak",
-            "config": {"workload": WORKLOAD[args.config], "points": n, "points_ok": n_ok,
-                       "sweep_points": len(CONFIGS[args.config]().points) if npts else n_sweep,
+            "scaling": args.scaling,
+            "config": {"workload": WORKLOAD[args.config], "points": n_sweep, "points_ok": n_ok,
+                       "points_per_rank": [len(s) for s in plan.shards], "sweep_scale": scale,
                        "trace": sw.trace.name, "ops": int(len(sw.trace.ops)),
-                       "parallelism": (f"one sweep dealt to {world} ranks by cost; records all-gathered over NCCL"
-                                       if (args.shard and world > 1) else
-                                       f"each of {world} rank(s) simulates a full sweep (weak scaling); "
-                                       "records all-gathered over NCCL"),
+                       "parallelism": (f"{n_sweep} distinct points dealt to {world} rank(s) by estimated cost (snake "
+                                       "order), each simulated once; records all-gathered over "
+                                       f"{backend if world > 1 else 'NCCL'} and scattered into sweep order"),
                        "l2": "flushed (256 MB write) before every timed step"},
-            "roofline": {"bound": "alu", "kernel": "k3_timeline", "achieved": round(achieved / 1e12, 6),
-                         "peak": round(peak_ops / 1e12, 3), "unit": "TFLOP/s (fp64, non-tensor)",
-                         "frac": round(achieved / peak_ops, 6), "traffic": traffic,
-                         "k3_ms": round(k3, 4), "alg_fp64_ops_per_launch": int(alg_ops),
-                         "peak_source": f"{N_SMS} SMs x {FP64_LANES_PER_SM} fp64 lanes x {clock_mhz} MHz "
-                                        f"(sm_max_mhz {src})"},
+            "roofline": roof,
             "hbm_roofline": {"bound": "hbm", "achieved": round(alg_b / (k3 / 1e3) / 1e9, 3),
                              "peak": pk.get("hbm_gbs"), "unit": "GB/s",
                              "frac": round(alg_b / (k3 / 1e3) / 1e9 / float(pk.get("hbm_gbs", 6650.0)), 7),
                              "algorithmic_bytes_per_launch": int(alg_b), "peak_source": src},
-            "e2e": {"value": round(e2e_points / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(n * rec), "ms_per_step": round(e2e_ms, 3),
-                    "steps": len(e2e_t), "timing": "wall clock, mean of consecutive API calls, max over ranks"},
+            "e2e": {"value": round(n_sweep / (e2e_ms / 1e3), 1), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": int(n_sweep * rec), "ms_per_step": round(e2e_ms, 3),
+                    "steps": len(e2e_t), "timing": "wall clock, mean of consecutive public-API calls "
+                                                   "(dist.simulate_sharded), max over ranks"},
             "gpu_launches": int(gpu_launches),
             "setup_ms": setup_ms,
             "clocks": clk.summary(),

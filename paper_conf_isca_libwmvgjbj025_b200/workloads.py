@@ -704,24 +704,33 @@ def sweep_c1() -> Sweep:
     return Sweep("c1_mlp_dp2", tr, [topo], points_array(pts))
 
 
-def sweep_c2(trace=None, seed=2) -> Sweep:
-    """configs[1]: ResNet-50 DP, p in {2,4,8,16} on a ring, 25 bandwidths x 10 latencies x
-    5 per-GPU batches x 2 bucket sizes -> 10,000 points (seeded order)."""
+def sweep_c2(trace=None, seed=2, n_bw=25) -> Sweep:
+    """configs[1]: ResNet-50 DDP (data parallel), p in {2,4,8,16} on a ring, 25 bandwidths x 10
+    latencies x 5 per-GPU batches x 2 bucket sizes -> 10,000 points (seeded order).  n_bw > 25 refines
+    the bandwidth axis (the multi-GPU bench's N x 10k-point sweeps; n_bw = 25 is configs[1] itself)."""
     tr = trace if trace is not None else resnet50_trace()
     ps = [2, 4, 8, 16]
     topos = [ring(p) for p in ps]
-    bws = np.logspace(np.log10(10e9), np.log10(900e9), 25)
+    bws = np.logspace(np.log10(10e9), np.log10(900e9), n_bw)
     lats = np.logspace(np.log10(0.5e-6), np.log10(20e-6), 10)
-    pts = []
-    for ti, p in enumerate(ps):
-        for b in (16, 32, 64, 128, 256):
-            for bucket in (0, 25 * MiB):
-                for bw in bws:
-                    for lat in lats:
-                        pts.append(make_point(ti, ST_DDP, dp=p, B=p * b, bucket=bucket, bw=float(bw), lat=float(lat)))
-    arr = points_array(pts)
+    batches, buckets = (16, 32, 64, 128, 256), (0, 25 * MiB)
+    n = len(ps) * len(batches) * len(buckets) * n_bw * len(lats)
+    ti, bi, ki, wi, li = np.meshgrid(np.arange(len(ps)), np.arange(len(batches)), np.arange(len(buckets)),
+                                     np.arange(n_bw), np.arange(len(lats)), indexing="ij")
+    arr = np.zeros(n, POINT_DTYPE)
+    pv = np.asarray(ps)[ti.ravel()]
+    arr["topo"] = ti.ravel()
+    arr["strategy"] = ST_DDP
+    arr["tp_mode"] = TPM_MEGATRON
+    arr["coll_algo"] = ALG_RING
+    arr["dp"], arr["tp"], arr["pp"], arr["microbatches"] = pv, 1, 1, 1
+    arr["global_batch"] = pv * np.asarray(batches)[bi.ravel()]
+    arr["stage_plan"] = -1
+    arr["bucket_bytes"] = np.asarray(buckets, np.uint64)[ki.ravel()]
+    arr["bw_scale"] = bws[wi.ravel()]
+    arr["lat_scale"] = lats[li.ravel()]
     perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
-    return Sweep("c2_resnet50_dp", tr, topos, arr[perm])
+    return Sweep("c2_resnet50_ddp", tr, topos, arr[perm])
 
 
 def sweep_c3(trace=None, seed=3, n_bw=8, n_lat=4) -> Sweep:
