@@ -1,0 +1,56 @@
+"""Full-sweep GPU parity: EVERY point of configs[0..3] (C1 2, C2 10,000, C3 9,216,
+C4 9,600) and the stratified configs[4] parity sample, simulated by the CUDA path through the C ABI in the
+launch configuration bench.py times (one simulate_batch over the whole sweep), compared element by
+element with the oracle's records written by tests/golden/make_goldens.py (which calls only oracle/).
+
+Bit-exact on status, counts, payload and order hash; |gpu - oracle| <= 1e-9 |oracle| on times.  No
+point may come back PT_TOO_LARGE (the oracle has no kernel limits; the expected list is empty).
+"""
+import os
+import sys
+
+import numpy as np
+import pytest
+
+from paper_conf_isca_libwmvgjbj025_b200 import workloads as W
+from tests.parity import compare
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, os.path.join(HERE, "golden"))
+import make_goldens as G  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+EXPECTED_TOO_LARGE = {"c1": [], "c2": [], "c3": [], "c4": [], "c5": []}
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_isca_libwmvgjbj025_b200 import triosim
+    c = triosim.Context(0)
+    yield c
+    c.close()
+
+
+def load(name):
+    path = os.path.join(HERE, "golden", f"{name}.npz")
+    if not os.path.exists(path):
+        pytest.fail(f"missing golden file {path}: run tests/golden/make_goldens.py {name}")
+    z = np.load(path)
+    return z["records"].view(W.RESULT_DTYPE), str(z["digest"])
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c3", "c4", "c5"])
+def test_full_sweep_matches_oracle(ctx, name):
+    ref, digest = load(name)
+    sw = G.SWEEPS[name]()
+    assert G.sweep_digest(sw) == digest, "the seeded generator no longer reproduces the golden sweep"
+    assert len(ref) == len(sw.points)
+    got = ctx.run_sweep(sw)
+    too_large = np.flatnonzero(got["status"] == W.PT_TOO_LARGE).tolist()
+    assert too_large == EXPECTED_TOO_LARGE[name]
+    bad, ulp = compare(got, ref)
+    assert not bad, f"{len(bad)} mismatches, first: {bad[:5]}"
+    print(f"{name}: {len(ref)} points bit-exact on counts/hash, {ulp} time fields differ in the last bits")
