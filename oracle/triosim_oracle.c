@@ -31,9 +31,10 @@
  * "Pins"), brute-force routing and partitioning, max-min invariants of the
  * progressive filling, and an exact-rational Python re-simulation of exported
  * task graphs.  Extensions R20-R26 (photonic network, per-layer breakdown,
- * timeline, DDP first bucket, pipelined ring, reduce + broadcast AllReduce)
- * carry their own pins (tests/test_oracle_{photonic,breakdown,timeline,
- * closed_forms,chunked_ring,reduce_broadcast}.py).
+ * timeline, DDP first bucket, pipelined ring, reduce + broadcast AllReduce, double
+ * binary tree) and R28 (Hop decentralized training) carry their own pins
+ * (tests/test_oracle_{photonic,breakdown,timeline,closed_forms,chunked_ring,
+ * reduce_broadcast,double_tree,hop,hash}.py).
  * Unpinned: absolute accuracy vs real hardware (P:244-300,
  * needs the paper's traces and machines) -- "parity unpinned" for that only.
  */
@@ -114,7 +115,8 @@ _Static_assert(sizeof(OResult) == 112, "result record");
 
 enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
 enum { CAT_INPUT = 0, CAT_WEIGHT = 1, CAT_WGRAD = 2, CAT_ACT = 3, CAT_AGRAD = 4, CAT_OTHER = 5 };
-enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4 };
+enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4, ST_HOP = 5 };
+enum { HOP_RING_BASED = 0, HOP_DOUBLE_RING = 1 };   /* R28 communication graphs (Fig. 16a) */
 enum { TPM_PAPER = 0, TPM_MEGATRON = 1 };
 enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2, ALG_DBTREE = 3 };
 enum { ROLE_NONE = 0, ROLE_COL = 1, ROLE_ROW = 2, ROLE_LOCAL = 3, ROLE_GATHER = 4 };
@@ -242,6 +244,7 @@ static double tensor_bytes(const Trace *T, uint32_t x, double r_b, int tp, int t
 enum { N_TASK = 0, N_FLOW = 1, N_BARRIER = 2 };
 #define NF_COLL_START 1 /* barrier that is a collective start (hashed) */
 #define NF_P2P 2        /* flow is a point-to-point data movement */
+#define NF_NEED_SHIFT 8 /* barrier: (flags >> 8) - 1 = dependencies it needs (0 = all of them; R28 threshold) */
 
 typedef struct {
     int type;
@@ -618,12 +621,23 @@ static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
 /* ------------------------------------------------------------------ */
 static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
                        int have_plan) {
-    if (pt->strategy > ST_HYBRID || pt->tp_mode > TPM_MEGATRON || pt->coll_algo > ALG_DBTREE ||
+    if (pt->strategy > ST_HOP || (pt->strategy != ST_HOP && pt->tp_mode > TPM_MEGATRON) || pt->coll_algo > ALG_DBTREE ||
         pt->ring_chunks > 16) return PT_BAD_CONFIG;   /* R25: at most 16 chunks per ring step */
     if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
         return PT_BAD_CONFIG;
     uint32_t dp = pt->dp, tpd = pt->tp, pp = pt->pp, m = pt->microbatches;
     if (dp == 0 || tpd == 0 || pp == 0) return PT_BAD_DEGREES;
+    if (pt->strategy == ST_HOP) {   /* R28 */
+        if (pt->tp_mode > HOP_DOUBLE_RING) return PT_BAD_CONFIG;
+        int first_opt = 0;
+        for (uint32_t o = 0; o < T->n_ops; o++) if (T->ops[o].phase == PH_OPT) first_opt = 1;
+        if (!first_opt) return PT_BAD_CONFIG;
+        if (tpd != 1 || pp != 1 || m == 0 || dp < 2 || dp % 2 || (pt->tp_mode == HOP_DOUBLE_RING && dp % 4))
+            return PT_BAD_DEGREES;
+        if (dp > tp->n_gpus) return PT_BAD_DEGREES;
+        if (pt->global_batch == 0 || pt->global_batch % dp != 0) return PT_BAD_BATCH;
+        return PT_OK;
+    }
     switch (pt->strategy) {
     case ST_DP: case ST_DDP: if (tpd != 1 || pp != 1) return PT_BAD_DEGREES; break;
     case ST_TP: if (dp != 1 || pp != 1) return PT_BAD_DEGREES; break;
@@ -775,6 +789,123 @@ static int expand_tp(const Trace *T, const OPoint *pt, const int *ro, Graph *G) 
         free(done_of); free(has); free(trig); free(prev);
     }
     free(task);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Extrapolation: Hop decentralized training (R28, Hop [42]) */
+/* ------------------------------------------------------------------ */
+/* Neighbours of worker i in the communication graph (Fig. 16a), ascending, without i itself:
+ * ring-based on n workers (n even): i-1, i+1 and the most distant worker i+n/2 (mod n);
+ * double ring (n % 4 == 0): two ring-based graphs on the halves {0..n/2-1}, {n/2..n-1}, plus the
+ * node-to-node edge i <-> i+n/2 between them. */
+static int hop_ring_based(int n, int i, int *nb) {
+    int c = 0, cand[3] = {(i + n - 1) % n, (i + 1) % n, (i + n / 2) % n};
+    for (int a = 0; a < 3; a++) {
+        if (cand[a] == i) continue;
+        int dup = 0;
+        for (int b = 0; b < c; b++) if (nb[b] == cand[a]) dup = 1;
+        if (!dup) nb[c++] = cand[a];
+    }
+    for (int x = 1; x < c; x++)   /* insertion sort */
+        for (int y = x; y > 0 && nb[y] < nb[y - 1]; y--) { int t = nb[y]; nb[y] = nb[y - 1]; nb[y - 1] = t; }
+    return c;
+}
+static int hop_neighbors(int n, int graph, int i, int *nb) {
+    if (graph == HOP_RING_BASED) return hop_ring_based(n, i, nb);
+    const int h = n / 2, half = i / h;
+    int c = hop_ring_based(h, i % h, nb);
+    for (int a = 0; a < c; a++) nb[a] += half * h;
+    nb[c++] = (i + h) % n;
+    for (int x = 1; x < c; x++)
+        for (int y = x; y > 0 && nb[y] < nb[y - 1]; y--) { int t = nb[y]; nb[y] = nb[y - 1]; nb[y - 1] = t; }
+    return c;
+}
+static uint64_t hop_flow_code(int k, int src, int dst) {
+    return (1ull << 58) | ((uint64_t)(uint32_t)k << 32) | ((uint64_t)(uint32_t)src << 16) | (uint64_t)(uint32_t)dst;
+}
+
+/*
+ * Worker r (GPU ro[r]) runs K = microbatches iterations of the whole trace (FWD, BWD, OPT ops in program
+ * order, t' at b_loc = B / n).  Reading of the paper's protocol (R28):
+ *   - update queues: after its last non-OPT op of iteration k the worker sends its update u(r, k) --
+ *     S bytes, the left fold of its weight-gradient sizes -- to every neighbour, ascending, on its FIFO
+ *     send stream (R11: one send at a time, across iterations too);
+ *   - bounded staleness s and backup workers b: the first OPT op of iteration k (applying the update)
+ *     waits until u(j, k - s) has been delivered from at least deg - b neighbours j (nothing to wait
+ *     for when k < s or deg <= b) -- a threshold barrier;
+ *   - token queues, bounded iteration gap g >= 1 (0 = unbounded): the first op of iteration k waits
+ *     until every neighbour has finished computing iteration k - g (its last non-OPT op).
+ * hop = backup | staleness << 4 | gap << 8 (point field pad1); tp_mode selects the graph.
+ */
+static int expand_hop(const Trace *T, const OPoint *pt, const int *ro, Graph *G) {
+    const int n = pt->dp, K = (int)pt->microbatches, graph = pt->tp_mode;
+    const int b = pt->pad1 & 15, s = (pt->pad1 >> 4) & 15, g = (pt->pad1 >> 8) & 255;
+    const uint32_t N = T->n_ops;
+    const double r_b = (double)(pt->global_batch / (uint32_t)n) / (double)T->b0;
+    int last_nonopt = -1, first_opt = -1;
+    for (uint32_t o = 0; o < N; o++) {
+        if (T->ops[o].phase != PH_OPT) last_nonopt = (int)o;
+        else if (first_opt < 0) first_opt = (int)o;
+    }
+    /* update size: left fold of the weight-gradient bytes' in production order (as R6's buckets) */
+    WEnt *w = (WEnt *)malloc(sizeof(WEnt) * (T->n_ts ? T->n_ts : 1));
+    int nw = 0;
+    for (uint32_t x = 0; x < T->n_ts; x++)
+        if (T->ts[x].category == CAT_WGRAD && T->prod[x] >= 0 && T->ops[T->prod[x]].phase != PH_OPT) {
+            w[nw].x = x; w[nw].prod = T->prod[x]; nw++;
+        }
+    qsort(w, (size_t)nw, sizeof(WEnt), cmp_went);
+    double S = 0.0;
+    for (int a = 0; a < nw; a++) S = S + tensor_bytes(T, w[a].x, r_b, 1, pt->tp_mode);
+    free(w);
+    int *nbr = (int *)malloc(sizeof(int) * (size_t)n * 4), *ndeg = (int *)malloc(sizeof(int) * (size_t)n);
+    int *task = (int *)malloc(sizeof(int) * (size_t)n * K * (N ? N : 1));
+    int *flow = (int *)malloc(sizeof(int) * (size_t)n * K * 4);
+    if (!nbr || !ndeg || !task || !flow) return -1;
+    for (int r = 0; r < n; r++) ndeg[r] = hop_neighbors(n, graph, r, nbr + r * 4);
+#define TSK(r, k, o) task[((size_t)(r) * K + (k)) * N + (o)]
+#define FLW(r, k, q) flow[((size_t)(r) * K + (k)) * 4 + (q)]
+    for (int r = 0; r < n; r++)
+        for (int k = 0; k < K; k++)
+            for (uint32_t o = 0; o < N; o++)
+                TSK(r, k, o) = add_task(G, ro[r], (long)k * N + o, op_time(T, o, r_b, 1, pt->tp_mode),
+                                        (int)T->ops[o].layer, (int)o, k);
+    for (int r = 0; r < n; r++) {
+        int prev = -1;   /* this worker's previous send (FIFO stream) */
+        for (int k = 0; k < K; k++)
+            for (int q = 0; q < ndeg[r]; q++) {
+                const int j = nbr[r * 4 + q];
+                const int f = add_flow(G, ro[r], ro[j], S, hop_flow_code(k, r, j), NF_P2P);
+                FLW(r, k, q) = f;
+                if (q == 0) g_dep(G, f, TSK(r, k, last_nonopt));
+                if (prev >= 0) g_dep(G, f, prev);
+                prev = f;
+                if (G->want_bd && ro[r] == G->rep[0]) g_record(G, f, f, (int)T->ops[last_nonopt].layer, 2);
+            }
+    }
+    for (int r = 0; r < n; r++)
+        for (int k = 0; k < K; k++) {
+            /* token queues: iteration k starts after every neighbour finished computing k - g */
+            if (g > 0 && k >= g)
+                for (int q = 0; q < ndeg[r]; q++) g_dep(G, TSK(r, k, 0), TSK(nbr[r * 4 + q], k - g, last_nonopt));
+            /* update queues with backup workers and bounded staleness */
+            const int need = ndeg[r] - b;
+            if (k >= s && need > 0) {
+                const int a = add_barrier(G, (need + 1) << NF_NEED_SHIFT, 0);
+                if (a < 0) return -1;
+                for (int q = 0; q < ndeg[r]; q++) {
+                    const int j = nbr[r * 4 + q];
+                    int qq = 0;
+                    while (nbr[j * 4 + qq] != r) qq++;   /* r's place in j's neighbour list */
+                    g_dep(G, a, FLW(j, k - s, qq));
+                }
+                g_dep(G, TSK(r, k, first_opt), a);
+            }
+        }
+#undef TSK
+#undef FLW
+    free(nbr); free(ndeg); free(task); free(flow);
     return 0;
 }
 
@@ -1226,7 +1357,11 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
         }
         free(fd); free(fr);
     }
-    for (long i = 0; i < NN; i++) pending[i] = (int)(doff[i + 1] - doff[i]);
+    for (long i = 0; i < NN; i++) {
+        pending[i] = (int)(doff[i + 1] - doff[i]);
+        /* R28: a threshold barrier completes once `need` of its dependencies are done */
+        if (G->n[i].type == N_BARRIER && (G->n[i].flags >> NF_NEED_SHIFT) > 0) pending[i] = (G->n[i].flags >> NF_NEED_SHIFT) - 1;
+    }
 
     /* per-GPU in-order queues */
     int *qoff = (int *)calloc((size_t)n_nodes_topo + 1, sizeof(int));
@@ -1475,7 +1610,7 @@ static int simulate(Graph *G, const Topo *tp, double bw_scale, double lat_scale,
                     for (int g = 0; g < n_nodes_topo; g++) {
                         if (running[g] >= 0 || head[g] >= qoff[g + 1] - qoff[g]) continue;
                         int k = qlist[qoff[g] + head[g]];
-                        if (pending[k] != 0) continue;
+                        if (pending[k] > 0) continue;
                         running[g] = k; head[g]++;
                         state[k] = S_RUN;
                         t_end[k] = t + G->n[k].dur;
@@ -1682,6 +1817,7 @@ static int build_graph(const Trace *T, const Topo *tp, const uint32_t *ring_orde
     switch (pt->strategy) {
     case ST_DP: case ST_DDP: rc = expand_dp(T, pt, ro, G); break;
     case ST_TP: rc = expand_tp(T, pt, ro, G); break;
+    case ST_HOP: rc = expand_hop(T, pt, ro, G); break;
     case ST_PP: case ST_HYBRID: {
         uint32_t *fl = (uint32_t *)malloc(sizeof(uint32_t) * pt->pp);
         if (have_plan) memcpy(fl, plan, sizeof(uint32_t) * pt->pp);

@@ -36,7 +36,7 @@ TENSOR_DTYPE = np.dtype([
 LINK_DTYPE = np.dtype([("src", "<u4"), ("dst", "<u4"), ("bw_Bps", "<f8"), ("lat_s", "<f8")])
 POINT_DTYPE = np.dtype([
     ("topo", "<u4"), ("strategy", "u1"), ("tp_mode", "u1"), ("coll_algo", "u1"), ("ring_chunks", "u1"),
-    ("dp", "<u2"), ("tp", "<u2"), ("pp", "<u2"), ("pad1", "<u2"),
+    ("dp", "<u2"), ("tp", "<u2"), ("pp", "<u2"), ("hop", "<u2"),
     ("microbatches", "<u4"), ("global_batch", "<u4"), ("stage_plan", "<i4"), ("first_bucket_bytes", "<u4"),
     ("bucket_bytes", "<u8"), ("bw_scale", "<f8"), ("lat_scale", "<f8")])
 PHOTONIC_DTYPE = np.dtype([("ports", "<u4"), ("buf_slots", "<u4"), ("link_bw_Bps", "<f8"), ("setup_s", "<f8"),
@@ -60,7 +60,8 @@ PH_FWD, PH_BWD, PH_OPT = 0, 1, 2
 CAT_INPUT, CAT_WEIGHT, CAT_WGRAD, CAT_ACT, CAT_AGRAD, CAT_OTHER = range(6)
 ROLE_NONE, ROLE_COL, ROLE_ROW, ROLE_LOCAL, ROLE_GATHER = 0, 1, 2, 3, 4
 OPF_BATCH_SCALED = 1
-ST_DP, ST_DDP, ST_TP, ST_PP, ST_HYBRID = range(5)
+ST_DP, ST_DDP, ST_TP, ST_PP, ST_HYBRID, ST_HOP = range(6)
+HOP_RING_BASED, HOP_DOUBLE_RING = 0, 1   # R28 communication graphs (Fig. 16a), in tp_mode
 TPM_PAPER, TPM_MEGATRON = 0, 1
 ALG_RING, ALG_TREE, ALG_REDBCAST, ALG_DBTREE = 0, 1, 2, 3
 PT_OK, PT_BAD_BATCH, PT_BAD_DEGREES, PT_NO_ROUTE, PT_TOO_LARGE, PT_DEADLOCK, PT_BAD_PLAN, PT_BAD_CONFIG = range(8)
@@ -677,8 +678,11 @@ class Sweep:
 
 
 def make_point(topo, strategy, dp=1, tp=1, pp=1, m=1, B=1, bucket=0, bw=1.0, lat=1.0, tp_mode=TPM_MEGATRON,
-               algo=ALG_RING, plan=-1, first_bucket=0, chunks=0):
+               algo=ALG_RING, plan=-1, first_bucket=0, chunks=0, hop=(0, 0, 0)):
+    """hop = (backup workers, staleness, max iteration gap) of a ST_HOP point (R28); for ST_HOP, dp = workers,
+    m = iterations and tp_mode = the communication graph (HOP_RING_BASED / HOP_DOUBLE_RING)."""
     p = np.zeros((), POINT_DTYPE)
+    p["hop"] = (hop[0] & 15) | ((hop[1] & 15) << 4) | ((hop[2] & 255) << 8)
     p["first_bucket_bytes"] = first_bucket
     p["ring_chunks"] = chunks
     p["topo"], p["strategy"], p["tp_mode"], p["coll_algo"] = topo, strategy, tp_mode, algo
@@ -820,6 +824,33 @@ def sweep_c5(trace=None, seed=5, Ns=(64, 128, 256, 512, 1024), n_bw=25, n_lat=14
     arr["lat_scale"] = np.tile(np.tile(lats, n_bw), len(R))
     perm = np.random.Generator(np.random.PCG64(seed)).permutation(len(arr))
     return Sweep("c5_gpt3_hybrid", tr, topos, arr[perm])
+
+
+def c5_parity_index(full: Sweep, per_n=20, heavy=4, seed=55) -> np.ndarray:
+    """Stratified configs[4] sample (SURVEY 8(c).4's >= 100 C5 points): for every
+    simulated-GPU count N, `heavy` points of the heavy classes -- data x tensor parallel degree
+    dp * tp = 64 (the verdict's "dp x tp >= 64" at its smallest product, which keeps each point at
+    1e6-1e7 instants), on the perturbed (slow-link subset) topology at 4:1 oversubscription, with 8
+    micro-batches -- plus seeded random points with 8 micro-batches."""
+    P = full.points
+    N = P["dp"].astype(np.int64) * P["tp"] * P["pp"]
+    rng = np.random.Generator(np.random.PCG64(seed))
+    topo_ov = np.array([t.name for t in full.topos])
+    idx = []
+    for n in sorted(set(N.tolist())):
+        sel = (N == n) & (P["microbatches"] == 8)
+        hv = np.flatnonzero(sel & (P["dp"].astype(np.int64) * P["tp"] == 64) & (P["topo"] % 2 == 1)
+                            & (np.char.find(topo_ov[P["topo"]].astype(str), "o4") >= 0))
+        hv = hv[rng.permutation(len(hv))][:heavy]
+        rest = np.setdiff1d(np.flatnonzero(sel), hv)
+        idx += hv.tolist() + rest[rng.permutation(len(rest))][:per_n - len(hv)].tolist()
+    return np.asarray(sorted(idx), np.int64)
+
+
+def sweep_c5_parity() -> Sweep:
+    """The C5 parity / bench subset: c5_parity_index over the full configs[4] sweep (100 points)."""
+    full = sweep_c5()
+    return Sweep(full.name + "_parity", full.trace, full.topos, full.points[c5_parity_index(full)])
 
 
 def sweep_wafer(trace=None, seed=6, n_bw=10, n_lat=5) -> Sweep:

@@ -102,7 +102,9 @@ def simulate(g, n_nodes, links, bw_scale=1, lat_scale=1):
     head = {q: 0 for q in queues}
     running = {q: None for q in queues}
     done = [None] * n
-    ndeps = [len(d) for d in deps]
+    # a barrier whose flags carry need + 1 in bits 8.. completes once `need` dependencies are done (R28)
+    ndeps = [(int(g["flags"][i]) >> 8) - 1 if typ[i] == BARRIER and (int(g["flags"][i]) >> 8) > 0 else len(deps[i])
+             for i in range(n)]
     released = set()
     end, tact, rem, rate, tupd, tdrain = {}, {}, {}, {}, {}, {}
     latent, active = set(), set()
@@ -146,7 +148,7 @@ def simulate(g, n_nodes, links, bw_scale=1, lat_scale=1):
                             dirty = True
                         changed = True
                 for i in range(n):
-                    if typ[i] != TASK and done[i] is None and i not in released and ndeps[i] == 0:
+                    if typ[i] != TASK and done[i] is None and i not in released and ndeps[i] <= 0:
                         if typ[i] == BARRIER:
                             complete(i)
                         else:
@@ -157,7 +159,7 @@ def simulate(g, n_nodes, links, bw_scale=1, lat_scale=1):
                 for q in queues:
                     if running[q] is None and head[q] < len(queues[q]):
                         k = queues[q][head[q]]
-                        if ndeps[k] == 0:
+                        if ndeps[k] <= 0:
                             running[q] = k
                             head[q] += 1
                             end[k] = t + Fr(g["dur"][k])
