@@ -36,7 +36,7 @@ from paper_conf_isca_libwmvgjbj025_b200 import workloads as W  # noqa: E402
 METRIC = "simulated design points/sec"
 UNIT = "points/s"
 CONFIGS = {"c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4, "c1": W.sweep_c1, "c5": W.sweep_c5,
-           "wafer": W.sweep_wafer}
+           "c5_subset": W.sweep_c5_parity, "wafer": W.sweep_wafer, "hop": W.sweep_hop}
 DEFAULT_POINTS = {"c5": 296}   # configs[4]'s 966k-point sweep: a seeded prefix (two waves of 1024-thread CTAs)
 WORKLOAD = {"c2": "configs[1]: ResNet-50 DDP (data parallel), 2-16 simulated GPUs on an NVLink-style ring, 10k-point "
                   "bandwidth x latency x batch x bucket sweep",
@@ -46,6 +46,11 @@ WORKLOAD = {"c2": "configs[1]: ResNet-50 DDP (data parallel), 2-16 simulated GPU
             "c1": "configs[0]: 4-layer MLP DDP on 2 GPUs, one uniform link",
             "c5": "configs[4]: GPT-3-class DP x TP x PP on 64-1024 simulated GPUs, hierarchical 1:1 / 2:1 / 4:1 "
                   "topology incl. a seeded slow-link subset (966k-point sweep, seeded prefix)",
+            "c5_subset": "configs[4] stratified subset: 100 GPT-3-class DP x TP x PP points, 20 per N in {64..1024} "
+                         "simulated GPUs incl. the dp x tp = 64 heavy class on the perturbed 4:1 topologies (the C5 "
+                         "parity sample, W.sweep_c5_parity)",
+            "hop": "NEXT 4: Hop decentralized training (P:348-364, Fig. 16), VGG-11 bs128 on 8 workers, ring-based / "
+                   "double-ring graphs, 8 random 1-10x slowdown groups, 0 / 1 backup worker, staleness + token gap",
             "wafer": "NEXT 1: 84-GPU 12x7 wafer, DDP ResNet-50, ring over the electrical mesh vs Passage photonic "
                      "logical links (P:330-342)"}
 FP64_LANES_PER_SM = 64     # B200 FP64 pipe: 64 DFMA/DADD/DMUL lanes per SM per clock
@@ -192,7 +197,7 @@ def run_reference(args):
 # ------------------------------------------------------------------------------------------
 OPS_PER_TASK = 2      # algorithmic fp64 ops per operator instance (rescale + fold)
 OPS_PER_WF_CALL = 80  # algorithmic fp64 ops per water-filling call (|A| <= 16)
-DEFAULT_NBW = {"c2": 25, "c3": 8, "c4": 25, "c5": 25, "wafer": 10}
+DEFAULT_NBW = {"c2": 25, "c3": 8, "c4": 25, "c5": 25, "wafer": 10, "hop": 5}
 
 
 def make_sweep(cfg, scale=1, npts=0):

@@ -45,7 +45,7 @@ typedef int32_t triosim_status;
 #define TRIOSIM_PT_BAD_BATCH 1   /* global_batch not divisible by dp * microbatches (Q3, Q12) */
 #define TRIOSIM_PT_BAD_DEGREES 2 /* zero / inconsistent degrees, dp*tp*pp > GPUs, pp > layers or > 64 */
 #define TRIOSIM_PT_NO_ROUTE 3    /* a needed (src, dst) GPU pair has no path */
-#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 1024 ranks, > 12288 links, > 8 hops) */
+#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 1024 ranks, > 8192 links, > 8 hops) */
 #define TRIOSIM_PT_DEADLOCK 5    /* the task graph cannot make progress */
 #define TRIOSIM_PT_BAD_PLAN 6    /* explicit stage plan invalid for this point */
 #define TRIOSIM_PT_BAD_CONFIG 7  /* unknown enum, topology index out of range, bw_scale <= 0, lat_scale < 0 */
@@ -146,14 +146,24 @@ typedef struct {
 #define TRIOSIM_TP 2      /* tensor parallel */
 #define TRIOSIM_PP 3      /* GPipe pipeline parallel */
 #define TRIOSIM_HYBRID 4  /* DP x TP x PP (extension, R9) */
+#define TRIOSIM_HOP 5     /* Hop heterogeneity-aware decentralized training (R28): dp = workers
+                             (even; <= 32 on this library's kernel), microbatches = iterations, tp_mode = the
+                             communication graph (TRIOSIM_HOP_*), hop = backup | staleness << 4 | max gap << 8 */
+#define TRIOSIM_HOP_RING_BASED 0   /* Fig. 16a top: ring plus each worker's most distant worker */
+#define TRIOSIM_HOP_DOUBLE_RING 1  /* Fig. 16a bottom: two ring-based graphs joined node to node (dp % 4 == 0) */
 #define TRIOSIM_TP_PAPER 0
 #define TRIOSIM_TP_MEGATRON 1
 #define TRIOSIM_ALGO_RING 0
 #define TRIOSIM_ALGO_TREE 1
 #define TRIOSIM_ALGO_REDBCAST 2   /* AllReduce as ring Reduce to member 0 + ring Broadcast from it, pipelined in
                                      ring_chunks chunks (R26); AllGather / ReduceScatter stay rings */
-/* coll_algo 3 (double binary tree, R27) is defined by the oracle only; this library version
-   reports TRIOSIM_PT_BAD_CONFIG for it, as for any coll_algo > 2. */
+#define TRIOSIM_ALGO_RSAG 4       /* AllReduce as a ring ReduceScatter followed by a ring AllGather: two collectives
+                                     of the group, the AllGather starting once every member finished the
+                                     ReduceScatter ("reduce, scatter, and gather"; R29) */
+#define TRIOSIM_ALGO_DBTREE 3     /* NCCL-style double binary tree AllReduce: two heap trees over mirrored member
+                                     positions, S/2 each, both at once (R27); runs in the hybrid kernel,
+                                     whose lanes hold the second tree on a spare flow slot -- TRIOSIM_PT_TOO_LARGE
+                                     for HYBRID points with both dp > 1 and tp > 1, and over photonic links */
 
 typedef struct {
     uint32_t topo;
@@ -162,7 +172,9 @@ typedef struct {
                                 slice S/p is sent as ring_chunks flows of S/(p*ring_chunks), one at a time per
                                 member; 0 or 1 = unchunked (R10); > 16 -> TRIOSIM_PT_BAD_CONFIG; ignored by
                                 tree AllReduces */
-    uint16_t dp, tp, pp, pad1;
+    uint16_t dp, tp, pp;
+    uint16_t hop;            /* TRIOSIM_HOP only (R28): backup workers (bits 0-3) | staleness (4-7) | max iteration
+                                gap, 0 = unbounded (8-15); ignored otherwise */
     uint32_t microbatches, global_batch;
     int32_t stage_plan;      /* -1 = automatic balanced partition */
     uint32_t first_bucket_bytes;  /* cap of each gradient group's first bucket (PyTorch DDP's first-bucket
@@ -243,18 +255,22 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
 
 /* Simulate points [first, first+count) of sweep_id: operator rescale (K1), task-graph
  * expansion (K2) and the timeline kernel (K3) on `cuda_stream` (cudaStream_t; NULL = the
- * legacy default stream).  Asynchronous and stream-ordered; returns after enqueue.
+ * legacy default stream).  Asynchronous and stream-ordered; returns after enqueue, for partial
+ * ranges too (the kernels skip the points outside the range).
  * Errors: ERANGE, ENOTFOUND, ECUDA. */
 triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
                                       void *cuda_stream);
 
-/* Copy result records [first, first+count) to out.  out_is_device == 0: host memory, the call
- * synchronises the stream of the last simulate_batch.  out_is_device != 0: a device pointer on
- * the context's GPU; the copy is enqueued on `cuda_stream` (stream-ordered, asynchronous). */
+/* Copy result records [first, first+count) to out.  out_is_device == 0: host memory; the call first
+ * synchronises the stream of the sweep's last simulate_batch (if it is not cuda_stream), then copies on
+ * cuda_stream and synchronises it.  out_is_device != 0: a device pointer on the context's GPU; the copy
+ * is enqueued on `cuda_stream` (stream-ordered, asynchronous: order it after simulate_batch yourself). */
 triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
                                triosim_result *out, int out_is_device, void *cuda_stream);
 
-/* Free a trace or sweep handle (a trace must outlive its sweeps). */
+/* Free a trace or sweep handle (a trace must outlive its sweeps).  Its device blocks go to a per-process
+ * cache that later load_trace / build_sweep calls reuse (at most TS_BLOCK_CACHE_MB, default 512 MiB, of idle
+ * blocks; TS_NO_BLOCK_CACHE=1 disables it; triosim_destroy returns them to the driver). */
 triosim_status triosim_release(triosim_ctx *ctx, int32_t handle);
 
 /* Per-layer breakdown ("the communication time and computation time of each layer or stage";

@@ -118,7 +118,7 @@ enum { CAT_INPUT = 0, CAT_WEIGHT = 1, CAT_WGRAD = 2, CAT_ACT = 3, CAT_AGRAD = 4,
 enum { ST_DP = 0, ST_DDP = 1, ST_TP = 2, ST_PP = 3, ST_HYBRID = 4, ST_HOP = 5 };
 enum { HOP_RING_BASED = 0, HOP_DOUBLE_RING = 1 };   /* R28 communication graphs (Fig. 16a) */
 enum { TPM_PAPER = 0, TPM_MEGATRON = 1 };
-enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2, ALG_DBTREE = 3 };
+enum { ALG_RING = 0, ALG_TREE = 1, ALG_REDBCAST = 2, ALG_DBTREE = 3, ALG_RSAG = 4 };
 enum { ROLE_NONE = 0, ROLE_COL = 1, ROLE_ROW = 2, ROLE_LOCAL = 3, ROLE_GATHER = 4 };
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 #define OPF_BATCH_SCALED 1u
@@ -477,10 +477,31 @@ static int build_collective_code(Graph *G, uint64_t c, const int *members, int p
     return 0;
 }
 
+/* R29 (NEXT 3; "NCCL-style collective communication, including reduce, scatter, and gather"):
+ * coll_algo = RSAG runs every AllReduce as two collectives of its group -- a ring ReduceScatter, then a
+ * ring AllGather of the same payload S, codes c and c + 1 -- so the AllGather starts (R10 barrier) once
+ * every member has finished the ReduceScatter.  *used = collectives created (1 or 2). */
+static int build_allreduce(Graph *G, uint64_t c, const int *members, int p, int kind, int algo, double S,
+                           const int *trig, const int *prev_done, int *done, uint64_t *used) {
+    if (algo == ALG_RSAG && kind == CK_AR) {
+        int *mid = (int *)malloc(sizeof(int) * (size_t)(p > 0 ? p : 1));
+        if (!mid) return -1;
+        int rc = build_collective_code(G, c, members, p, CK_RS, ALG_RING, G->nch, S, trig, prev_done, mid);
+        if (!rc) rc = build_collective_code(G, c + 1, members, p, CK_AG, ALG_RING, G->nch, S, trig, mid, done);
+        free(mid);
+        *used = 2;
+        return rc;
+    }
+    *used = 1;
+    return build_collective_code(G, c, members, p, kind, algo == ALG_RSAG ? ALG_RING : algo, G->nch, S, trig,
+                                 prev_done, done);
+}
+
 /* collectives of DP / DDP / TP: one group, numbered in creation order */
 static int build_collective(Graph *G, const int *members, int p, int kind, int algo, double S,
                             const int *trig, const int *prev_done, int *done) {
-    return build_collective_code(G, (uint64_t)G->n_coll, members, p, kind, algo, G->nch, S, trig, prev_done, done);
+    uint64_t used;
+    return build_allreduce(G, (uint64_t)G->n_coll, members, p, kind, algo, S, trig, prev_done, done, &used);
 }
 
 /* ------------------------------------------------------------------ */
@@ -621,7 +642,7 @@ static int auto_partition(const Trace *T, int S, uint32_t *first_layer) {
 /* ------------------------------------------------------------------ */
 static int point_check(const Trace *T, const Topo *tp, const OPoint *pt, const uint32_t *plan, uint32_t plan_len,
                        int have_plan) {
-    if (pt->strategy > ST_HOP || (pt->strategy != ST_HOP && pt->tp_mode > TPM_MEGATRON) || pt->coll_algo > ALG_DBTREE ||
+    if (pt->strategy > ST_HOP || (pt->strategy != ST_HOP && pt->tp_mode > TPM_MEGATRON) || pt->coll_algo > ALG_RSAG ||
         pt->ring_chunks > 16) return PT_BAD_CONFIG;   /* R25: at most 16 chunks per ring step */
     if (!(pt->bw_scale > 0.0) || isinf(pt->bw_scale) || !(pt->lat_scale >= 0.0) || isinf(pt->lat_scale))
         return PT_BAD_CONFIG;
@@ -1120,9 +1141,10 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                         for (int t = 0; t < tp; t++) trig[t] = task[base + t][q];
                         G->cur_layer = (int)op->layer;
                         G->cur_cat = 0;
-                        if (build_collective_code(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, G->nch, Sb, trig,
-                                                  have_prev ? prev : NULL, done)) goto out;
-                        seq++;
+                        uint64_t used = 1;
+                        if (build_allreduce(G, (gid << 20) | seq, members, tp, kind, pt->coll_algo, Sb, trig,
+                                            have_prev ? prev : NULL, done, &used)) goto out;
+                        seq += used;
                         memcpy(prev, done, sizeof(int) * (size_t)tp);
                         have_prev = 1;
                         if (hm_put(&tpc, (gid << 40) | ((uint64_t)x << 16) | (uint64_t)pmb[s][q], (int)dtab.n)) goto out;
@@ -1232,9 +1254,10 @@ static int expand_hybrid(const Trace *T, const OPoint *pt, const int *ro, const 
                     for (int d = 0; d < dp; d++) trig[d] = task[(d * S + s) * tp + t][qt];
                     G->cur_layer = (int)T->ops[pop[s][qt]].layer;
                     G->cur_cat = 1;
-                    if (build_collective_code(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, G->nch, Sb, trig,
-                                              have_prev ? prev : NULL, done)) { free(w); goto out; }
-                    seq++;
+                    uint64_t used = 1;
+                    if (build_allreduce(G, (gid << 20) | seq, members, dp, CK_AR, pt->coll_algo, Sb, trig,
+                                        have_prev ? prev : NULL, done, &used)) { free(w); goto out; }
+                    seq += used;
                     memcpy(prev, done, sizeof(int) * (size_t)dp);
                     have_prev = 1;
                     i = j;

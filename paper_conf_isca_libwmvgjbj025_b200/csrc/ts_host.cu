@@ -36,7 +36,9 @@ struct BlockCache {
     std::mutex mu;
     std::multimap<std::pair<int, size_t>, void *> blocks;
     size_t bytes = 0;
-    static constexpr size_t kMaxBytes = size_t(4) << 30;
+    // at most TS_BLOCK_CACHE_MB (default 512) MiB of idle blocks are kept; a failing cudaMalloc of ours
+    // empties the cache of that device first, and triosim_destroy empties it
+    const size_t kMaxBytes = size_t(getenv("TS_BLOCK_CACHE_MB") ? atol(getenv("TS_BLOCK_CACHE_MB")) : 512) << 20;
     bool on = getenv("TS_NO_BLOCK_CACHE") == nullptr || atoi(getenv("TS_NO_BLOCK_CACHE")) == 0;
     cudaError_t get(void **p, size_t want, size_t *cap, int *dev) {
         cudaError_t e = cudaGetDevice(dev);
@@ -130,6 +132,7 @@ struct Trace {
     std::vector<triosim_tensor> ts;
     std::vector<uint32_t> io;
     uint32_t b0 = 0, n_layers = 0;
+    int32_t first_opt = -1;   // first OPT-phase op (R28 needs one to apply updates)
     std::vector<int32_t> prod;
     // trace-level facts the host needs (route needs, cost estimates, partitions)
     uint32_t n_wgrad = 0;
@@ -181,7 +184,6 @@ struct Sweep {
     DevBuf<triosim_result> d_res;
     std::vector<uint32_t> work[N_GROUPS];    // per (W index, mode)
     DevBuf<uint32_t> d_work[N_GROUPS];
-    DevBuf<uint32_t> d_work_tmp[N_GROUPS];
     std::vector<int> mode;                   // per point
     uint32_t lmax[N_GROUPS] = {};            // hybrid CTA groups: largest topology (links) among their points
     uint32_t pmax[N_GROUPS] = {};            // hybrid groups: most photonic ports among their points (R20)
@@ -341,6 +343,7 @@ triosim_status triosim_load_trace(triosim_ctx *ctx, const triosim_trace_desc *t,
         const triosim_op &op = tr->ops[o];
         if (op.phase > 2 || op.phase < last_phase) return fail(ctx, TRIOSIM_EINVAL, "op %u: phases not FWD* BWD* OPT*", o);
         last_phase = op.phase;
+        if (op.phase == 2 && tr->first_opt < 0) tr->first_opt = (int32_t)o;
         if (!(op.time_s >= 0.0) || std::isinf(op.time_s)) return fail(ctx, TRIOSIM_EINVAL, "op %u: bad time", o);
         if ((uint64_t)op.io_off + op.n_in + op.n_out > t->n_io) return fail(ctx, TRIOSIM_EINVAL, "op %u: io out of range", o);
         if (op.tp_role > 7) return fail(ctx, TRIOSIM_EINVAL, "op %u: bad tp_role", o);
@@ -609,7 +612,11 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto setst = [&](int st) { S->status[i] = st; };
         // R3, in order
         if (pt.topo >= n_topos) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
-        if (pt.strategy > TRIOSIM_HYBRID || pt.tp_mode > 1 || pt.coll_algo > 2 || pt.ring_chunks > 16) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+        if (pt.strategy > TRIOSIM_HOP || (pt.strategy != TRIOSIM_HOP && pt.tp_mode > 1) ||
+            pt.coll_algo > TRIOSIM_ALGO_RSAG || pt.ring_chunks > 16) {
+            setst(TRIOSIM_PT_BAD_CONFIG);
+            continue;
+        }
         if (!(pt.bw_scale > 0.0) || std::isinf(pt.bw_scale) || !(pt.lat_scale >= 0.0) || std::isinf(pt.lat_scale)) {
             setst(TRIOSIM_PT_BAD_CONFIG);
             continue;
@@ -617,6 +624,56 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         const HostTopo &tp = HT[pt.topo];
         const uint32_t dp = pt.dp, tpd = pt.tp, pp = pt.pp, mb = pt.microbatches;
         bool bad = dp == 0 || tpd == 0 || pp == 0;
+        if (!bad && pt.strategy == TRIOSIM_HOP) {
+            // R28: graph, an OPT op to apply updates, n even (double ring: n % 4 == 0), one iteration at least
+            if (pt.tp_mode > TRIOSIM_HOP_DOUBLE_RING || T.first_opt < 0) { setst(TRIOSIM_PT_BAD_CONFIG); continue; }
+            if (tpd != 1 || pp != 1 || mb == 0 || dp < 2 || dp % 2 || (pt.tp_mode == TRIOSIM_HOP_DOUBLE_RING && dp % 4) ||
+                dp > tp.n_gpus) { setst(TRIOSIM_PT_BAD_DEGREES); continue; }
+            if (pt.global_batch == 0 || pt.global_batch % dp != 0) { setst(TRIOSIM_PT_BAD_BATCH); continue; }
+            // warp-segment kernel only: <= 32 workers on a flow-network topology that fits a segment's links
+            int W = 0, W0 = 2;
+            while (W0 < (int)dp) W0 <<= 1;
+            if (!tp.photonic && tp.max_hops <= MAX_ROUTE_K3)
+                for (int w = W0; w <= 32; w <<= 1)
+                    if ((int)tp.n_links <= lmax_warp(w)) { W = w; break; }
+            if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
+            const uint32_t b_loc = pt.global_batch / dp;
+            auto key = std::make_tuple((int)TRIOSIM_HOP, (int)dp, (int)b_loc, (int)pt.tp_mode, 0, 0, 1, (uint64_t)0,
+                                       (uint32_t)pt.hop, (int)mb, -2);
+            uint32_t c;
+            auto ci = cls_of.find(key);
+            if (ci == cls_of.end()) {
+                ClassDesc cd;
+                std::memset(&cd, 0, sizeof cd);
+                cd.mode = MODE_HOP;
+                cd.strategy = TRIOSIM_HOP;
+                cd.tp_mode = pt.tp_mode;   // the communication graph
+                cd.p = dp;
+                cd.m = mb;
+                cd.tpdeg = 1;
+                cd.dp = 1;
+                cd.b_loc = b_loc;
+                cd.nch = 1;
+                cd.hop = pt.hop;
+                cd.r_b = (double)b_loc / (double)T.b0;
+                c = (uint32_t)S->classes.size();
+                S->classes.push_back(cd);
+                cls_of[key] = c;
+            } else {
+                c = ci->second;
+            }
+            PointDesc &pd = pdesc[i];
+            pd.bw_scale = pt.bw_scale;
+            pd.lat_scale = pt.lat_scale;
+            pd.cls = c;
+            pd.topo = pt.topo;
+            pd.idx = (uint32_t)i;
+            pd.pad = 0;
+            S->width[i] = W;
+            S->mode[i] = MODE_HOP;
+            S->cost[i] = (double)mb * N * 2.0 + (double)mb * 4.0 * 16.0 * dp;
+            continue;
+        }
         if (!bad) {
             if ((pt.strategy == TRIOSIM_DP || pt.strategy == TRIOSIM_DDP) && (tpd != 1 || pp != 1)) bad = true;
             if (pt.strategy == TRIOSIM_TP && (dp != 1 || pp != 1)) bad = true;
@@ -658,7 +715,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         // DataParallel maps to HYBRID with its buckets triggered after the backward pass
         int W = 0;
         bool dp_after = false;
-        if (pt.strategy != TRIOSIM_HYBRID && !tp.photonic)
+        // R27's double binary tree runs in the hybrid kernel (its lanes hold tree B on a spare flow slot)
+        // a warp kernel keeps owner bits for <= MAX_ROUTE_K3 hops: longer routes also go to the hybrid kernel
+        if (pt.strategy != TRIOSIM_HYBRID && !tp.photonic && pt.coll_algo != TRIOSIM_ALGO_DBTREE && tp.max_hops <= MAX_ROUTE_K3)
             for (int w = W0; w <= 32; w <<= 1)
                 if ((int)tp.n_links <= lm(false, w)) { W = w; break; }
         if (W == 0) {
@@ -673,7 +732,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         // photonic tree collectives: a broadcast flow parent -> child lives in the child's lane but needs the
         // parent's logical links (ports are the sender's, R20); not supported by this kernel
         // (a class without collective groups -- dp = tp = 1 -- has no tree to run)
-        if (tp.photonic && pt.coll_algo == TRIOSIM_ALGO_TREE && (dp > 1 || tpd > 1)) W = 0;
+        if (tp.photonic && (pt.coll_algo == TRIOSIM_ALGO_TREE || pt.coll_algo == TRIOSIM_ALGO_DBTREE) && (dp > 1 || tpd > 1)) W = 0;
+        // R27: tree B needs the other group's flow slot -- not with both a TP and a DP group
+        if (pt.coll_algo == TRIOSIM_ALGO_DBTREE && dp > 1 && tpd > 1) W = 0;
         // K2's pipeline / hybrid expansion keeps the layer -> stage map in shared memory (K2P_MAX_LAYERS)
         if ((pt.strategy == TRIOSIM_PP || pt.strategy == TRIOSIM_HYBRID) && T.n_layers > K2P_MAX_LAYERS) W = 0;
         if (W == 0) { setst(TRIOSIM_PT_TOO_LARGE); continue; }
@@ -765,10 +826,11 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     for (uint32_t c = 0; c < S->classes.size(); c++) {
         ClassDesc &cd = S->classes[c];
         cd.dur_off = dur_n; dur_n += N;
-        if (cd.mode == MODE_COLL) {
+        if (cd.mode == MODE_COLL || cd.mode == MODE_HOP) {
             S->coll_list.push_back(c);
             cd.hook_off = hook_n; hook_n += N;
-            cd.coll_cap = (cd.strategy == TRIOSIM_TP) ? T.n_out_total : T.n_wgrad;
+            cd.coll_cap = cd.mode == MODE_HOP ? 0 : (cd.strategy == TRIOSIM_TP) ? T.n_out_total : T.n_wgrad;
+            if (cd.algo == TRIOSIM_ALGO_RSAG) cd.coll_cap *= 2;   // R29: ReduceScatter + AllGather per AllReduce
             cd.coll_off = coll_n; coll_n += cd.coll_cap;
             if (cd.strategy == TRIOSIM_TP) { cd.scratch_off = scr_i; scr_i += NT; }
         } else if (cd.mode == MODE_HYBRID) {
@@ -780,9 +842,9 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             cd.send_off = hsend_n; hsend_n += cd.send_cap;
             cd.recv_cap = T.n_in_total;
             cd.recv_off = recv_n; recv_n += cd.recv_cap;
-            cd.tcol_cap = T.n_out_total;
+            cd.tcol_cap = T.n_out_total * (cd.algo == TRIOSIM_ALGO_RSAG ? 2 : 1);
             cd.tcol_off = coll_n; coll_n += cd.tcol_cap;
-            cd.dcol_cap = T.n_wgrad;
+            cd.dcol_cap = T.n_wgrad * (cd.algo == TRIOSIM_ALGO_RSAG ? 2 : 1);
             cd.dcol_off = coll_n; coll_n += cd.dcol_cap;
             cd.scratch_off = scr_u; scr_u += NT;
         } else {
@@ -916,7 +978,6 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
     PT.mark("wl lists");
     for (int w = 0; w < N_GROUPS; w++) {
         CK(S->d_work[w].upload(S->work[w]));
-        CK(S->d_work_tmp[w].alloc(S->work[w].size()));
     }
     PT.mark("wl uploads");
     CK(S->d_counter.alloc(N_GROUPS));
@@ -972,6 +1033,8 @@ static K3Args k3_args(Sweep &S, int w) {
     a.alg_ops = S.d_alg.p;
     a.lmax = S.lmax[w];
     a.pmax = S.pmax[w];
+    a.rlo = 0;
+    a.rhi = 0xffffffffu;
     return a;
 }
 
@@ -1008,19 +1071,18 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     int launched[N_GROUPS] = {};
     for (int w = 0; w < N_GROUPS; w++) {
         const uint32_t *wl = S.d_work[w].p;
-        uint32_t n = (uint32_t)S.work[w].size();
+        const uint32_t n_all = (uint32_t)S.work[w].size();
+        uint32_t n = n_all;   // points of this group in [first, first + count): the kernel skips the rest
         if (!full) {
-            std::vector<uint32_t> sub;
-            for (uint32_t i : S.work[w]) if (i >= first && i < first + count) sub.push_back(i);
-            n = (uint32_t)sub.size();
-            if (n) CK(cudaMemcpyAsync(S.d_work_tmp[w].p, sub.data(), n * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
-            CK(cudaStreamSynchronize(st));  // sub is a host temporary
-            wl = S.d_work_tmp[w].p;
+            n = 0;
+            for (uint32_t i : S.work[w]) n += (i >= first && i < first + count) ? 1u : 0u;
         }
         if (n == 0) continue;
         const int W = W_OF[w / N_MODES], mode = w % N_MODES;
         K3Args a = k3_args(S, w);
-        a.work = wl; a.n_work = n;
+        a.work = wl; a.n_work = n_all;
+        a.rlo = (uint32_t)first;
+        a.rhi = (uint32_t)(first + count);
         if (S.bd) {
             a.bd = S.d_bd_acc.p;
             a.layer = T.d_layer.p;
@@ -1091,6 +1153,8 @@ triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t firs
     if (out_is_device) {
         CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToDevice, st));
     } else {
+        // the last simulate_batch may have run on another (non-blocking) stream: finish it first
+        if (S.last_stream != st) CK(cudaStreamSynchronize(S.last_stream));
         CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
     }
@@ -1112,6 +1176,9 @@ triosim_status triosim_timeline(triosim_ctx *ctx, int32_t sweep_id, uint64_t poi
     *n_tasks = *n_flows = 0;
     if (S.status[point] >= 0) return TRIOSIM_OK;   // decided on the host (R3): no timeline
     cudaStream_t st = nullptr;
+    // K2's tables, the work counter and the result records are shared with simulate_batch: let its last
+    // call (possibly on a non-blocking stream) finish first
+    CK(cudaStreamSynchronize(S.last_stream));
     CK(enqueue_k1_k2(ctx, S, T, st));
     if (S.d_tl_tasks.n < task_cap || !S.d_tl_tasks.p) CK(S.d_tl_tasks.alloc(task_cap));
     if (S.d_tl_flows.n < flow_cap || !S.d_tl_flows.p) CK(S.d_tl_flows.alloc(flow_cap));

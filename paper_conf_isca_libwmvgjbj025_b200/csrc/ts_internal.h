@@ -7,10 +7,11 @@
 
 namespace ts {
 
-enum { MODE_COLL = 0, MODE_PIPE = 1, MODE_TREE = 2, MODE_HYBRID = 3 };  // K3 variants: ring-only collectives, GPipe, tree-capable collectives, DP x TP x PP
+enum { MODE_COLL = 0, MODE_PIPE = 1, MODE_TREE = 2, MODE_HYBRID = 3, MODE_HOP = 4 };  // K3 variants: ring-only collectives, GPipe, tree-capable collectives, DP x TP x PP, Hop (R28)
 enum { CK_AR = 0, CK_AG = 1, CK_RS = 2 };
 enum { PH_FWD = 0, PH_BWD = 1, PH_OPT = 2 };
-constexpr int MAX_HOPS = 8;
+constexpr int MAX_HOPS = 8;   // route hops cached in registers per flow; longer routes read the rest from rt_links
+constexpr uint32_t MAX_ROUTE_K3 = 32;   // longest route of a warp-kernel (K3) topology (its owner bits); beyond: K3h
 constexpr uint8_t NO_ROUTE = 0xFF;
 #ifndef TS_K3_THREADS
 #define TS_K3_THREADS 128
@@ -128,6 +129,9 @@ struct ClassDesc {
     uint32_t n_coll, need_ring, need_tree, n_prog_max;
     double coll_payload;
     uint64_t n_compute, n_flows;
+    // R28 Hop: backup | staleness << 4 | gap << 8 (host); K2: update bytes, last non-OPT op, first OPT op
+    uint32_t hop, hop_last, hop_first, hop_pad;
+    double hop_S;
 };
 
 struct TopoDev {
@@ -150,6 +154,7 @@ struct K3Args {
     const PointDesc *pts;
     const uint32_t *work;
     uint32_t n_work, lmax;         // lmax: links per segment in dynamic smem (one-point-per-CTA hybrid)
+    uint32_t rlo, rhi;             // simulate only work items (point indices) in [rlo, rhi)
     uint32_t pmax, pad2;           // pmax: photonic ports per lane in dynamic smem (hybrid, R20)
     unsigned int *counter;
     const ClassDesc *cls;
@@ -220,9 +225,9 @@ int k3_max_blocks_per_sm(int W, int mode);
 // links per segment the K3 kernels keep in shared memory
 __host__ __device__ constexpr int lmax_warp(int W) { return 4 * W < 8 ? 8 : 4 * W; }
 __host__ __device__ constexpr int lmax_hybrid(int W) { return 8 * W < 16 ? 16 : 8 * W; }
-constexpr int LMAX_CTA = 12288;         // links of a one-point-per-CTA hybrid segment (dynamic smem, 16 B/link)
+constexpr int LMAX_CTA = 6144;          // links of a one-point-per-CTA hybrid segment (dynamic smem, 28 B/link)
 constexpr int N_WIDTHS = 10;            // W = 2, 4, 8, 16, 32 (warp segments), 64 ... 1024 (hybrid CTAs)
-constexpr int N_MODES = 4;
+constexpr int N_MODES = 5;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups
 constexpr int MAX_PORTS = 8;            // photonic ports per GPU the hybrid kernel holds (R20)
 constexpr uint32_t K2P_MAX_LAYERS = 2048;   // trace layers the PP / HYBRID expansion (K2) stages in shared memory

@@ -80,6 +80,23 @@ struct Route {
     int len;
 };
 
+// R28: neighbours of worker i in Fig. 16a's communication graphs, as a bit set over the n <= 32 workers
+// (so they come out ascending): ring-based -- the ring neighbours and the most distant worker of i's
+// group, the group being all n workers; double ring -- the same inside i's half, plus its counterpart
+// in the other half.  Returns the degree; nb[] receives the ranks.
+__device__ __forceinline__ int hop_nbrs(int n, int graph, int i, int (&nb)[4]) {
+    const int h = graph == 1 ? n / 2 : n, base = i - i % h, j = i % h;
+    uint32_t set = (1u << (base + (j + 1) % h)) | (1u << (base + (j + h - 1) % h)) | (1u << (base + (j + h / 2) % h));
+    if (graph == 1) set |= 1u << ((i + h) % n);
+    set &= ~(1u << i);
+    int d = 0;
+    while (set && d < 4) {
+        nb[d++] = __ffs(set) - 1;
+        set &= set - 1;
+    }
+    return d;
+}
+
 struct TopoRef {
     uint32_t n_gpus, link_off, rt_off, ro_off;
 };
@@ -92,8 +109,9 @@ __device__ __forceinline__ Route get_route(const K3Args &a, const TopoRef &T, ui
     return r;
 }
 
-// route latency: left fold of link latency x lat_scale (R12); caches the link ids (<= 8 hops,
-// 16 bit each) in four registers for the water-filling rounds
+// route latency: left fold of link latency x lat_scale (R12); caches the first MAX_HOPS link ids (16
+// bit each) in four registers for the water-filling rounds -- hops past them (at most MAX_ROUTE_K3) are
+// read from rt_links at the route's offset
 __device__ __forceinline__ double load_route(const K3Args &a, const TopoRef &T, Route r, double lat_scale,
                                              uint32_t (&hl)[4]) {
     double L = 0.0;
@@ -105,6 +123,7 @@ __device__ __forceinline__ double load_route(const K3Args &a, const TopoRef &T, 
             hl[h >> 1] |= e << (16 * (h & 1));
             L = L + a.link_lat[T.link_off + e] * lat_scale;
         }
+    for (int h = MAX_HOPS; h < r.len; h++) L = L + a.link_lat[T.link_off + a.rt_links[r.off + h]] * lat_scale;
     return L;
 }
 __device__ __forceinline__ int hop(const uint32_t (&hl)[4], int h) { return (hl[h >> 1] >> (16 * (h & 1))) & 0xffff; }
@@ -121,12 +140,16 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     constexpr bool LOG = (V & V_LOG) != 0;
     constexpr int NSEG = 32 / W;
     constexpr int LMAX = lmax_warp(W);
-    constexpr bool COLL = MODE != MODE_PIPE;   // DP / DDP / TP collectives
+    constexpr bool HOPM = MODE == MODE_HOP;    // R28 Hop decentralized training (update / token queues)
+    constexpr bool COLL = MODE == MODE_COLL || MODE == MODE_TREE;   // DP / DDP / TP collectives
     constexpr bool TREE = MODE == MODE_TREE;   // ... some of which may be tree AllReduces
     __shared__ double s_res[K3_WARPS][NSEG * LMAX];
     __shared__ int s_n[K3_WARPS][NSEG * LMAX];
     __shared__ int s_k[K3_WARPS][NSEG * LMAX];
     __shared__ uint32_t s_cnt[K3_WARPS][COLL ? 1 : 32];
+    // HOP: per worker lane and neighbour slot q, 1 + the last iteration whose update from that neighbour
+    // was delivered (FIFO streams make it monotone); s_cnt holds each lane's finished backward passes
+    __shared__ uint32_t s_rcv[K3_WARPS][HOPM ? 32 * 4 : 1];
 
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int seg = lane / W, li = lane % W, sbase = seg * W;
@@ -135,6 +158,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     int *ln = &s_n[wid][seg * LMAX];
     int *lk = &s_k[wid][seg * LMAX];
     uint32_t *cnt = &s_cnt[wid][COLL ? 0 : sbase];
+    uint32_t *rcv = &s_rcv[wid][HOPM ? sbase * 4 : 0];
     for (int q = lane; q < NSEG * LMAX; q += 32) { s_n[wid][q] = 0; s_k[wid][q] = 0; }
     __syncwarp();
 
@@ -180,11 +204,21 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     double t_act = 0.0, rem = 0.0, rate = 0.0, t_upd = 0.0, t_drain = 0.0, fbytes = 0.0;
     int flen = 0;
     uint32_t hl[4] = {0, 0, 0, 0};
+    uint32_t froff = 0;       // route offset of the flow in flight (hops past MAX_HOPS)
     uint64_t fcode = 0;
     StageInfo SI;
     SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
     SI.ent_off = SI.send_off = SI.recv_off = 0;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
+    // HOP (R28): neighbours (ranks, ascending) and this lane's slot in each neighbour's list; iteration
+    // structure (ops per iteration, last non-OPT op, first OPT op); finished backward passes; the flow in
+    // flight's destination lane, slot and iteration
+    int hdeg = 0, hb = 0, hs = 0, hg = 0;
+    int hnb[4] = {0, 0, 0, 0}, hsl[4] = {0, 0, 0, 0};
+    uint32_t hN = 1, hlast = 0, hfirst = 0, hbwd = 0;
+    int hdst = 0, hslot = 0;
+    uint32_t hk = 0;
+    double hS = 0.0;
     uint64_t acc = 0;            // this lane's part of the order hash (R19)
     uint32_t alg = 0;            // fp64 operations of the method performed by this lane (wraps per point only beyond 4e9)
     uint64_t tmix = 0;           // mix64(bits(t)) of the current instant
@@ -232,6 +266,8 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
           if (need) {
             if (it >= a.n_work) {
                 exhausted = true;
+            } else if (a.work[it] < a.rlo || a.work[it] >= a.rhi) {
+                // outside [first, first + count) of this simulate_batch call: skipped, refilled next pass
             } else {
                 fresh = have = true;
 #ifdef TS_PROF
@@ -282,11 +318,8 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         nprog = C->n_prog_max;
                         hwait = nprog > 0 ? a.hooks[C->hook_off].wait : -1;
                         rring = get_route(a, TR, gpu, a.ro[TR.ro_off + (li + 1) % p]);
-                        if (C->need_ring) {
-                            if (rring.len == NO_ROUTE) rbad = true;
-                            else if (rring.len > MAX_HOPS) rlong = true;
-                        }
-                        if (rring.len != NO_ROUTE && rring.len <= MAX_HOPS) {
+                        if (C->need_ring && rring.len == NO_ROUTE) rbad = true;
+                        if (rring.len != NO_ROUTE) {
                             Lring = load_route(a, TR, rring, lats, hring);
                             alg += 2 * rring.len;
                             // link-disjoint ring (host-checked): a ring flow is alone on each of its
@@ -299,13 +332,38 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                     const double b = a.link_bw[TR.link_off + hop(hring, h)] * bws;
                                     rbw = b < rbw ? b : rbw;
                                 }
+                            for (int h = MAX_HOPS; h < rring.len; h++) {
+                                const double b = a.link_bw[TR.link_off + a.rt_links[rring.off + h]] * bws;
+                                rbw = b < rbw ? b : rbw;
+                            }
                             alg += 2 * rring.len;
                         }
                         if (C->need_tree && li >= 1) {
                             const uint32_t par = a.ro[TR.ro_off + (li - 1) / 2];
                             const int l1 = get_route(a, TR, gpu, par).len, l2 = get_route(a, TR, par, gpu).len;
                             if (l1 == NO_ROUTE || l2 == NO_ROUTE) rbad = true;
-                            else if (l1 > MAX_HOPS || l2 > MAX_HOPS) rlong = true;
+                        }
+                    } else if constexpr (HOPM) {
+                        hN = C->n_prog_max;
+                        hlast = C->hop_last;
+                        hfirst = C->hop_first;
+                        hS = C->hop_S;
+                        hb = (int)(C->hop & 15u);
+                        hs = (int)((C->hop >> 4) & 15u);
+                        hg = (int)((C->hop >> 8) & 255u);
+                        nprog = m * hN;
+                        hbwd = 0;
+                        hdeg = hop_nbrs(p, (int)C->tp_mode, li, hnb);
+                        nsend_tot = m * (uint32_t)hdeg;
+                        for (int q = 0; q < 4; q++) {
+                            rcv[li * 4 + q] = 0;
+                            if (q < hdeg) {
+                                int o4[4];
+                                const int od = hop_nbrs(p, (int)C->tp_mode, hnb[q], o4);
+                                for (int x = 0; x < od; x++) if (o4[x] == li) hsl[q] = x;
+                                const int l = get_route(a, TR, gpu, a.ro[TR.ro_off + hnb[q]]).len;
+                                if (l == NO_ROUTE) rbad = true;
+                            }
                         }
                     } else {
                         SI = a.stages[C->stage_off + li];
@@ -317,7 +375,6 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             dm &= dm - 1;
                             const int l = get_route(a, TR, gpu, a.ro[TR.ro_off + d]).len;
                             if (l == NO_ROUTE) rbad = true;
-                            else if (l > MAX_HOPS) rlong = true;
                         }
                     }
                 }
@@ -431,24 +488,42 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 }
                             }
                         }
-                        if (used) {
-                            // all eight terms unconditionally (no branches: eight independent chains the
-                            // compiler interleaves), the ones past n masked out of the sum
+                        // order-hash terms (R19).  With spare lanes (W >= 2p) the twin lane li + W/2 hashes
+                        // instants 4..7 of member li and the member lane instants 0..3 (the segment's hash is
+                        // the sum over all its lanes), halving the warp's mix64 work; else the member lane
+                        // takes all eight.  All terms unconditionally (independent chains the compiler
+                        // interleaves), the ones past n masked out of the sum
+                        const bool split = 2 * p <= W;
+                        const bool twin = split && li >= W / 2 && li - W / 2 < p;
+                        if (used || twin) {
+                            const uint64_t cb = ((uint64_t)cur << 32) | (uint64_t)(twin ? li - W / 2 : li);
+                            // instant of parity `odd` (0 activation, 1 delivery + release) of step k
+                            auto term = [&](double tv, bool odd, int kk) -> uint64_t {
+                                const uint64_t m = mix64((uint64_t)__double_as_longlong(tv));
+                                const uint64_t k = (uint64_t)kk;
+                                if (!odd)
+                                    return mix64(m ^ (((uint64_t)EV_ACTIVATE << 60) | cb | (k << 16)));
+                                return mix64(m ^ (((uint64_t)EV_DELIVER << 60) | cb | (k << 16))) +
+                                       mix64(m ^ (((uint64_t)EV_RELEASE << 60) | cb | ((k + 1) << 16)));
+                            };
                             uint64_t add = 0;
+                            if (split) {
+                                const int off = twin ? 4 : 0;
 #pragma unroll
-                            for (int i = 0; i < 8; i++) {
-                                const uint64_t m = mix64((uint64_t)__double_as_longlong(ti[i]));
-                                const uint64_t k = (uint64_t)(D0 + (i >> 1));
-                                uint64_t term;
-                                if ((i & 1) == 0) {
-                                    term = mix64(m ^ (((uint64_t)EV_ACTIVATE << 60) | cbase | (k << 16)));
-                                } else {
-                                    term = mix64(m ^ (((uint64_t)EV_DELIVER << 60) | cbase | (k << 16))) +
-                                           mix64(m ^ (((uint64_t)EV_RELEASE << 60) | cbase | ((k + 1) << 16)));
+                                for (int i = 0; i < 4; i++) {
+                                    const uint64_t tr = term(twin ? ti[i + 4] : ti[i], (i & 1) != 0, D0 + ((i + off) >> 1));
+                                    add += i + off < n ? tr : 0ull;
                                 }
-                                add += i < n ? term : 0ull;
+                            } else {
+#pragma unroll
+                                for (int i = 0; i < 8; i++) {
+                                    const uint64_t tr = term(ti[i], (i & 1) != 0, D0 + (i >> 1));
+                                    add += i < n ? tr : 0ull;
+                                }
                             }
                             acc += add;
+                        }
+                        if (used) {
                             alg += 2u * (uint32_t)((n + 1) >> 1) + (uint32_t)(n >> 1);
                             nflow += (uint32_t)(n >> 1);
                         }
@@ -501,6 +576,12 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             EV(EV_TASK_END, ((uint64_t)gpu << 40) | (pos - 1));
                         }
                         hwait = pos < nprog ? a.hooks[C->hook_off + pos].wait : -1;
+                    } else if constexpr (HOPM) {
+                        // the run ends at the iteration's last non-OPT op: its update goes out (R28)
+                        if ((pos - 1) % hN == hlast) {
+                            hbwd++;
+                            EV(EV_TASK_END, ((uint64_t)gpu << 40) | (pos - 1));
+                        }
                     } else {
                         const uint32_t q = pos - 1;
                         uint32_t P, idx;
@@ -545,9 +626,12 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         }
                     } else {
                         dcnt++;
-                        if constexpr (BD) {   // R22: P2P time of the sending (representative) stage
-                            double *q = a.bd + ((size_t)pidx * 3 + 2) * a.n_layers + bd_l;
-                            *q = *q + (t - bd_t0);
+                        if constexpr (HOPM) rcv[hdst * 4 + hslot] = hk + 1;   // update (hk) reached hdst (R28)
+                        if constexpr (BD) {   // R22: P2P time of the sending (representative) stage / rank 0
+                            if (!HOPM || li == 0) {
+                                double *q = a.bd + ((size_t)pidx * 3 + 2) * a.n_layers + bd_l;
+                                *q = *q + (t - bd_t0);
+                            }
                         }
                     }
                 }
@@ -630,6 +714,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 rel = true;
                                 flen = rring.len;
                                 hl[0] = hring[0]; hl[1] = hring[1]; hl[2] = hring[2]; hl[3] = hring[3];
+                                froff = rring.off;
                                 fbytes = chunk;
                                 t_act = t + Lring;
                                 alg += 1;
@@ -646,6 +731,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 const Route r = get_route(a, TR, gpu, par);
                                 flen = r.len;
                                 t_act = t + load_route(a, TR, r, lats, hl);
+                                froff = r.off;
                                 fcode = ((uint64_t)cur << 32) | (uint64_t)li;
                                 fup = uprel = rel = true;
                                 if constexpr (LOG) { fbytes = cS; tl_release(gpu, par); }
@@ -656,6 +742,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 const Route r = get_route(a, TR, par, gpu);
                                 flen = r.len;
                                 t_act = t + load_route(a, TR, r, lats, hl);
+                                froff = r.off;
                                 fcode = ((uint64_t)cur << 32) | (1ull << 16) | (uint64_t)li;
                                 fup = false;
                                 dnrel = rel = true;
@@ -669,6 +756,37 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         if (rel) {
                             fst = FS_LAT;
                             EV(EV_RELEASE, fcode);
+                            if (t_act == t) more = true;
+                        }
+                    }
+                } else if constexpr (HOPM) {
+                    // (d) R28 update queues: the lane's FIFO send stream -- iteration k's update to each
+                    // neighbour in turn, once the iteration's backward pass is done
+                    cnt[li] = hbwd;
+                    __syncwarp();
+                    if (used && fst == FS_NONE && sq < nsend_tot) {
+                        const uint32_t k = sq / (uint32_t)hdeg, q = sq % (uint32_t)hdeg;
+                        if (hbwd > k) {
+                            const int j = hnb[q];
+                            const uint32_t dg = a.ro[TR.ro_off + j];
+                            const Route r = get_route(a, TR, gpu, dg);
+                            flen = r.len;
+                            fst = FS_LAT;
+                            fbytes = hS;
+                            t_act = t + load_route(a, TR, r, lats, hl);
+                                froff = r.off;
+                            alg += 2 * flen + 1;
+                            fcode = (1ull << 58) | ((uint64_t)k << 32) | ((uint64_t)li << 16) | (uint64_t)j;
+                            hdst = j;
+                            hslot = hsl[q];
+                            hk = k;
+                            EV(EV_RELEASE, fcode);
+                            if constexpr (LOG) tl_release(gpu, dg);
+                            if constexpr (BD) {
+                                bd_t0 = t;
+                                bd_l = a.layer[hlast];
+                            }
+                            sq++;
                             if (t_act == t) more = true;
                         }
                     }
@@ -693,6 +811,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             fst = FS_LAT;
                             fbytes = se.bytes;
                             t_act = t + load_route(a, TR, r, lats, hl);
+                                froff = r.off;
                             alg += 2 * flen + 1;
                             fcode = (1ull << 59) | ((uint64_t)se.x << 32) | ((uint64_t)j << 16) | (uint64_t)dg;
                             EV(EV_RELEASE, fcode);
@@ -708,7 +827,50 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 }
                 // (e) an idle GPU starts its head operator once its inputs are present
                 if (used && cst == CS_IDLE && pos < nprog) {
-                    if constexpr (COLL) {
+                    if constexpr (HOPM) {
+                        const uint32_t k = pos / hN, o = pos % hN;
+                        bool ok = true, ev = false;
+                        if (o == 0 && hg > 0 && (int)k >= hg) {
+                            // token queues: every neighbour finished computing iteration k - g
+                            ev = true;
+                            for (int q = 0; q < hdeg; q++)
+                                if (cnt[hnb[q]] < k - (uint32_t)hg + 1) ok = false;
+                        }
+                        if (o == hfirst && (int)k >= hs && hdeg > hb) {
+                            // update queues: deg - b neighbours' updates of iteration k - s arrived
+                            ev = true;
+                            int got = 0;
+                            for (int q = 0; q < hdeg; q++) got += rcv[li * 4 + q] >= k - (uint32_t)hs + 1 ? 1 : 0;
+                            if (got < hdeg - hb) ok = false;
+                        }
+                        if (ok) {
+                            if (ev) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
+                            run_start = pos;
+                            // fold (R16) to the next boundary: through the iteration's last non-OPT op (its
+                            // completion sends the update), or up to an op that waits (the first OPT op of an
+                            // iteration that applies updates, the first op of a gated iteration)
+                            double te = t;
+                            uint32_t q = pos;
+                            for (;;) {
+                                const uint32_t oo = q % hN;
+                                const double dd = a.dur[C->dur_off + oo];
+                                if constexpr (LOG) tl_task(gpu, q, oo, q / hN, te, te + dd);
+                                te = te + dd;
+                                busy = busy + dd;
+                                q++;
+                                if (oo == hlast || q >= nprog) break;
+                                const uint32_t no = q % hN, nk = q / hN;
+                                if (no == hfirst && (int)nk >= hs && hdeg > hb) break;
+                                if (no == 0 && hg > 0 && (int)nk >= hg) break;
+                            }
+                            ntask += q - pos;
+                            alg += 2 * (q - pos);
+                            run_end = q;
+                            t_end = te;
+                            cst = CS_RUN;
+                            if (te == t) more = true;
+                        }
+                    } else if constexpr (COLL) {
                         if (hwait < 0 || (int)donec > hwait) {
                             const OpHook *HK = a.hooks + C->hook_off;
                             const OpHook h = HK[pos];
@@ -820,15 +982,31 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             atomicAdd(&ln[e], 1);
                             lres[e] = a.link_bw[TR.link_off + e] * bws;
                         }
+                    for (int h = MAX_HOPS; h < flen; h++) {   // long routes
+                        const int e = a.rt_links[froff + h];
+                        atomicAdd(&ln[e], 1);
+                        lres[e] = a.link_bw[TR.link_off + e] * bws;
+                    }
                 }
                 __syncwarp();
             }
             if (act && fast) rate = rbw;
             // uniform link-disjoint ring: one round at rate rbw, nothing to reduce
             const bool uni = fast && ring_uni;
-            bool unf = act && !uni;
             const bool segany = (__ballot_sync(FULL, act) & smask) != 0;
             uint32_t rounds = (uni && segany) ? 1u : 0u;
+            // link-disjoint ring with different rates: progressive filling freezes, round after round, the
+            // flows at the smallest remaining rate, so its rounds are the distinct rates of the active
+            // flows -- counted at once (a lane leads its value if it is the lowest segment lane holding it)
+            if (__any_sync(FULL, fast && !uni && segany)) {
+                const unsigned long long key = act ? (unsigned long long)__double_as_longlong(rate)
+                                                   : ~(unsigned long long)lane;   // NaN patterns, never a rate
+                const unsigned mm = __match_any_sync(FULL, key) & smask;
+                const bool lead = act && (__ffs(mm) - 1) == lane;
+                const uint32_t nd = __popc(__ballot_sync(FULL, lead) & smask);
+                if (fast && !uni) rounds = nd;
+            }
+            bool unf = act && !fast;
             if (__any_sync(FULL, unf)) {   // guard: keeps the loop's hoisted address math off the fast path
                 while (__any_sync(FULL, unf)) {
                     const bool segact = (__ballot_sync(FULL, unf) & smask) != 0;
@@ -844,6 +1022,11 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                     const double sh = lres[e] / (double)ln[e];
                                     my = sh < my ? sh : my;
                                 }
+                            for (int h = MAX_HOPS; h < flen; h++) {
+                                const int e = a.rt_links[froff + h];
+                                const double sh = lres[e] / (double)ln[e];
+                                my = sh < my ? sh : my;
+                            }
                             alg += 2 * flen;
                         }
                     }
@@ -855,6 +1038,8 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
                             if (h < flen && atomicAdd(&lk[hop(hl, h)], 1) == 0) own |= 1u << h;
+                        for (int h = MAX_HOPS; h < flen; h++)   // (flen <= MAX_ROUTE_K3 = 32: host-checked)
+                            if (atomicAdd(&lk[a.rt_links[froff + h]], 1) == 0) own |= 1u << h;
                     }
                     if (anygen) __syncwarp();
                     if (inF && !fast) {
@@ -862,6 +1047,16 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         for (int h = 0; h < MAX_HOPS; h++)
                             if ((own >> h) & 1u) {
                                 const int e = hop(hl, h);
+                                const int kk = lk[e];
+                                const double r = lres[e] - s * (double)kk;
+                                lres[e] = r > 0.0 ? r : 0.0;
+                                ln[e] -= kk;
+                                lk[e] = 0;
+                                alg += 3;
+                            }
+                        for (int h = MAX_HOPS; h < flen; h++)
+                            if ((own >> h) & 1u) {
+                                const int e = a.rt_links[froff + h];
                                 const int kk = lk[e];
                                 const double r = lres[e] - s * (double)kk;
                                 lres[e] = r > 0.0 ? r : 0.0;
@@ -965,6 +1160,7 @@ static cudaError_t launch_w(int mode, const K3Args &a, int grid, cudaStream_t s)
     switch (mode) {
     case MODE_COLL: return launch_wm<W, MODE_COLL>(a, grid, s);
     case MODE_TREE: return launch_wm<W, MODE_TREE>(a, grid, s);
+    case MODE_HOP: return launch_wm<W, MODE_HOP>(a, grid, s);
     default: return launch_wm<W, MODE_PIPE>(a, grid, s);
     }
 }
@@ -985,6 +1181,7 @@ static int occ_w(int mode) {
     int nb = 0;
     if (mode == MODE_COLL) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_COLL, 0>, K3_THREADS, 0);
     else if (mode == MODE_TREE) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_TREE, 0>, K3_THREADS, 0);
+    else if (mode == MODE_HOP) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_HOP, 0>, K3_THREADS, 0);
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k3_timeline<W, MODE_PIPE, 0>, K3_THREADS, 0);
     return nb;
 }

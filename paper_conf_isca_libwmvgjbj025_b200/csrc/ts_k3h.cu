@@ -62,7 +62,8 @@ struct Flow {
     int st;
     double t_act, rem, rate, t_upd, t_drain, bytes;
     int len;
-    uint32_t hl[4];
+    uint32_t hl[4];               // the first MAX_HOPS link ids (16 bit each) ...
+    uint32_t roff;                // ... and where the route sits in rt_links, for the hops beyond them
     uint64_t code;
     uint32_t src, dst;            // endpoints (R23 timeline records only)
     unsigned long long tl;        // R23 (LOG): record slot
@@ -91,6 +92,7 @@ struct Group {
     uint64_t gid;
     uint32_t ncoll, trig, donec, cur;
     bool running, tree_cur, ldone, uprel, upd, dnrel, dnd, fup;
+    bool dbt_cur, uprel2, upd2, dnrel2, dnd2, fup2;   // R27 double binary tree: the mirrored tree B's edge state
     bool rb_cur;              // R26: the running AllReduce is a ring Reduce + ring Broadcast
     int K, D, Kp;             // this member's / its predecessor's sends in the running collective
     double cS, chunk;
@@ -139,6 +141,8 @@ __device__ __forceinline__ void release(const K3Args &a, const Topo &T, Flow &f,
             f.hl[h >> 1] |= e << (16 * (h & 1));
             L = L + a.link_lat[T.link_off + e] * lats;
         }
+    for (int h = MAX_HOPS; h < len; h++) L = L + a.link_lat[T.link_off + a.rt_links[off + h]] * lats;   // long routes
+    f.roff = off;
     f.len = len;
     f.st = FS_LAT;
     f.bytes = bytes;
@@ -161,26 +165,41 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     constexpr int LMAXW = lmax_hybrid(W);               // warp segments: static link arrays
     constexpr int NSLOT = NW == 1 ? K3_WARPS : 1;       // segment-array slots of the block
     // warp segments keep their link arrays in static smem; a one-point CTA sizes them to the sweep's
-    // largest topology (a.lmax links, dynamic smem: residual f64, unfrozen and frozen counts)
+    // largest topology (a.lmax links, dynamic smem: residual f64, share f64, unfrozen and frozen counts)
     __shared__ double s_res[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
+    __shared__ double s_sh[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
     __shared__ int s_n[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
     __shared__ int s_k[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];
+    __shared__ int s_own[NW == 1 ? NSLOT : 1][NW == 1 ? NSEG * LMAXW : 1];   // owner of a link reached past MAX_HOPS
     extern __shared__ double s_dyn[];
     const int LMAX = NW == 1 ? LMAXW : (int)a.lmax;
     // photonic tables (R20) after the CTA link arrays: per lane a.pmax logical links {dst GPU, state
     // 0 none / 1 setup / 2 up, t = ready time or last use} and per flow slot its buffer request
     constexpr int NTHR = NW == 1 ? K3_THREADS : 32 * NW;
     const int PM = (int)a.pmax;
-    double *p_t = s_dyn + (NW == 1 ? 0 : 2 * LMAX);
-    int *p_dst = (int *)(p_t + NTHR * PM);
-    int *p_st = p_dst + NTHR * PM;
-    double *q_t = (double *)(p_st + NTHR * PM);               // [3 * NTHR] request key time
-    unsigned long long *q_code = (unsigned long long *)(q_t + 3 * NTHR);
-    int *q_dst = (int *)(q_code + 3 * NTHR);                   // destination GPU or -1
-    uint8_t *q_st = (uint8_t *)(q_dst + 3 * NTHR);             // 1 waiting for a buffer, 2 transferring
-    uint8_t *q_g = q_st + 3 * NTHR;                            // granted
+    // A one-point CTA keeps them at the start of dynamic smem while it runs a photonic point (which has
+    // no link arrays), after the link arrays otherwise; dynamic smem = the larger of the two (k3h_dyn_smem)
+    double *p_t;
+    int *p_dst, *p_st;
+    double *q_t;                    // [3 * NTHR] request key time
+    unsigned long long *q_code;
+    int *q_dst;                     // destination GPU or -1
+    uint8_t *q_st, *q_g;            // 1 waiting for a buffer / 2 transferring; granted
+    auto ph_tables = [&](bool phot) {
+        p_t = s_dyn + ((NW == 1 || phot) ? 0 : (7 * LMAX + 1) / 2);   // after lres, lsh, ln, lk, lown
+        p_dst = (int *)(p_t + NTHR * PM);
+        p_st = p_dst + NTHR * PM;
+        q_t = (double *)(p_st + NTHR * PM);
+        q_code = (unsigned long long *)(q_t + 3 * NTHR);
+        q_dst = (int *)(q_code + 3 * NTHR);
+        q_st = (uint8_t *)(q_dst + 3 * NTHR);
+        q_g = q_st + 3 * NTHR;
+    };
+    ph_tables(false);
+    bool last_phot = false;   // CTA: the previous point ran photonic (its tables overlaid the link arrays)
     __shared__ uint32_t s_cnt[NSLOT][NW == 1 ? 32 : SL];
     __shared__ double s_red[2][NW];
+    __shared__ unsigned s_fl3[2][NW];                  // CTA: per-warp end-of-instant votes
     __shared__ unsigned long long s_red64[2][NW];
     __shared__ int s_xch[2][NW == 1 ? 1 : SL];
     __shared__ int s_gc[3][NW == 1 ? 1 : SL];          // cross-warp group counters (rotating triple buffer)
@@ -194,8 +213,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     const unsigned smask = NW == 1 ? ((W == 32 ? FULL : ((1u << (W & 31)) - 1u)) << sbase) : FULL;
     const int slot = NW == 1 ? wid : 0;
     double *lres = NW == 1 ? &s_res[slot][seg * LMAX] : s_dyn;
-    int *ln = NW == 1 ? &s_n[slot][seg * LMAX] : (int *)(s_dyn + LMAX);
-    int *lk = NW == 1 ? &s_k[slot][seg * LMAX] : (int *)(s_dyn + LMAX) + LMAX;
+    double *lsh = NW == 1 ? &s_sh[slot][seg * LMAX] : s_dyn + LMAX;   // share res / n of links with n > 0
+    int *ln = NW == 1 ? &s_n[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX);
+    int *lk = NW == 1 ? &s_k[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + LMAX;
+    int *lown = NW == 1 ? &s_own[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + 2 * LMAX;
     uint32_t *cnt = &s_cnt[slot][sbase];                     // indexed by segment lane
     for (int q = (NW == 1 ? lane : (int)threadIdx.x); q < NSEG * LMAX; q += (NW == 1 ? 32 : 32 * NW)) {
         ln[q - seg * LMAX] = 0;   // (NW == 1: each lane clears its warp's slot through segment 0's base)
@@ -322,7 +343,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     int ports = 0, bufs = 0;
     int R = 1, S = 1, tp = 1, dp = 1;
     uint32_t m = 1;
-    bool tree_algo = false;
+    bool tree_algo = false, dbt_algo = false;   // binary-tree AllReduce (R10) / double binary tree (R27)
     const ClassDesc *C = nullptr;
     Topo TR = {0, 0, 0, 0, false};
     uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
@@ -403,6 +424,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         G.ncoll = ncoll;
         G.trig = G.donec = G.cur = 0;
         G.running = G.tree_cur = G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = G.fup = false;
+        G.dbt_cur = G.uprel2 = G.upd2 = G.dnrel2 = G.dnd2 = G.fup2 = false;
         G.K = G.D = G.Kp = 0;
         G.rb_cur = false;
         G.cS = G.chunk = 0.0;
@@ -416,15 +438,22 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     };
 
     // R10 for one group: done on this member, finish, start, releases (all lanes call it)
-    auto grp_pass = [&](Group &G, Flow &F, bool is_tp, bool &more) {
-        const int Dp = xch(G.D, G.pred);
+    auto grp_pass = [&](Group &G, Flow &F, Flow &F2, bool is_tp, bool &more) {
+        // the predecessor's progress: a shuffle when every group of this kind lies inside one warp (TP groups;
+        // segment-uniform), a shared-memory exchange across warps otherwise
+        const int Dp = (NW > 1 && !G.cross) ? __shfl_sync(FULL, G.D, G.pred & 31) : xch(G.D, G.pred);
         LF upb, dnb, zero;
         upb.bits = dnb.bits = zero.bits = 0;
         upb.p = dnb.p = zero.p = nullptr;
         upb.sel = dnb.sel = zero.sel = 1;
-        if (vany(G.tree_cur)) flags2(G.upd, G.dnd, upb, dnb);
+        if ((tree_algo || dbt_algo) && vany(G.tree_cur)) flags2(G.upd, G.dnd, upb, dnb);   // (segment-uniform)
+        LF upb2 = zero, dnb2 = zero;
+        if (dbt_algo && vany(G.dbt_cur)) flags2(G.upd2, G.dnd2, upb2, dnb2);
         auto mb = [&](const LF &b, int k) -> bool { return b.test(G.lane0 + k * G.stride); };
         const int c1 = 2 * G.i + 1, c2 = 2 * G.i + 2;
+        // R27's tree B: member i sits at heap position p - 1 - i
+        const int hB = G.p - 1 - G.i, b1 = 2 * hB + 1, b2 = 2 * hB + 2;
+        auto memB = [&](int h) { return G.p - 1 - h; };
         if (G.member && G.running && !G.ldone) {
             bool dn;
             if (!G.tree_cur) {
@@ -433,6 +462,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 const bool ku = (c1 >= G.p || mb(upb, c1)) && (c2 >= G.p || mb(upb, c2));
                 const bool kd = (c1 >= G.p || mb(dnb, c1)) && (c2 >= G.p || mb(dnb, c2));
                 dn = (G.i == 0 || (G.upd && G.dnd)) && ku && kd;
+                if (G.dbt_cur) {
+                    const bool kuB = (b1 >= G.p || mb(upb2, memB(b1))) && (b2 >= G.p || mb(upb2, memB(b2)));
+                    const bool kdB = (b1 >= G.p || mb(dnb2, memB(b1))) && (b2 >= G.p || mb(dnb2, memB(b2)));
+                    dn = dn && (hB == 0 || (G.upd2 && G.dnd2)) && kuB && kdB;
+                }
             }
             if (dn) {
                 G.ldone = true;
@@ -461,8 +495,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 ce = a.colls[HS.dcol_off + G.cur];
             }
             G.running = started = true;
-            G.tree_cur = tree_algo && ce.kind == CK_AR;
-            G.cS = ce.S;
+            G.tree_cur = (tree_algo || dbt_algo) && ce.kind == CK_AR;
+            G.dbt_cur = dbt_algo && ce.kind == CK_AR;
+            G.cS = G.dbt_cur ? ce.S / 2.0 : ce.S;   // R27: each tree carries half the payload
             G.chunk = ce.S / (double)G.p / (double)C->nch;   // R25
             G.K = (ce.kind == CK_AR ? 2 * (G.p - 1) : (G.p - 1)) * (int)C->nch;
             G.Kp = G.K;
@@ -476,6 +511,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             }
             G.D = 0;
             G.ldone = G.uprel = G.upd = G.dnrel = G.dnd = false;
+            G.uprel2 = G.upd2 = G.dnrel2 = G.dnd2 = false;
             if (G.i == 0) {
                 EV(EV_COLL_START, (G.gid << 20) | G.cur);
                 alg += 1;
@@ -521,6 +557,30 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 if (F.t_act == t) more = true;
             }
         }
+        // R27 tree B (mirrored heap positions, steps 2 up / 3 down) on the lane's second slot
+        if (G.member && G.running && G.dbt_cur && hB >= 1 && F2.st == FS_NONE) {
+            const uint64_t cc = (G.gid << 20) | G.cur;
+            const LF ub = started ? zero : upb2, db = started ? zero : dnb2;
+            const bool ku = (b1 >= G.p || mb(ub, memB(b1))) && (b2 >= G.p || mb(ub, memB(b2)));
+            const int parh = (hB - 1) / 2, par = memB(parh);
+            bool rel = false;
+            if (!G.uprel2 && ku) {
+                release(a, TR, F2, gpu, gpu_of_member(G, par), G.cS, (cc << 32) | (2ull << 16) | (uint64_t)G.i, t, lats,
+                        alg);
+                G.fup2 = G.uprel2 = rel = true;
+            } else if (G.uprel2 && G.upd2 && !G.dnrel2 &&
+                       (parh == 0 ? ((G.p <= 1 || mb(ub, memB(1))) && (G.p <= 2 || mb(ub, memB(2)))) : mb(db, par))) {
+                release(a, TR, F2, gpu_of_member(G, par), gpu, G.cS, (cc << 32) | (3ull << 16) | (uint64_t)G.i, t, lats,
+                        alg);
+                G.fup2 = false;
+                G.dnrel2 = rel = true;
+            }
+            if (rel) {
+                EV(EV_RELEASE, F2.code);
+                if constexpr (LOG) tl_release(F2);
+                if (F2.t_act == t) more = true;
+            }
+        }
     };
     // (b)/(c) for one flow slot; returns true if delivered
     auto flow_step = [&](Flow &F, bool &dirty) -> bool {
@@ -558,6 +618,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             G.D++;
         }
     };
+    auto grp_delivered2 = [&](Group &G) {   // R27: a tree-B edge of G (on the lane's second slot)
+        G.flow_deliv++;
+        if (G.fup2) G.upd2 = true; else G.dnd2 = true;
+    };
     // decode program position q of this stage -> (phase, micro-batch, index in phase list)
     auto decode = [&](uint32_t q, uint32_t &P, uint32_t &j, uint32_t &idx) {
         if (q < m * SI.nF) { P = 0; j = q / SI.nF; idx = q % SI.nF; }
@@ -592,6 +656,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             if (need) {
                 if (it >= a.n_work) {
                     exhausted = true;
+                } else if (a.work[it] < a.rlo || a.work[it] >= a.rhi) {
+                    // outside [first, first + count) of this simulate_batch call: skipped, refilled next pass
                 } else {
                     fresh = have = true;
                     const PointDesc pd = a.pts[a.work[it]];
@@ -615,6 +681,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     R = dp * S * tp;
                     m = C->m;
                     tree_algo = C->algo == TRIOSIM_ALGO_TREE;
+                    dbt_algo = C->algo == TRIOSIM_ALGO_DBTREE;
                     t = 0.0;
                     tmix = mix64(0ull);
                     ninst = nwf = nrounds = maxact = 0;
@@ -644,14 +711,21 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     grp_init(GT, used && tp > 1, tp, tt, (d * S + s) * tp, 1, (uint64_t)(d * S + s), ntp, d * S + s);
                     grp_init(GD, used && dp > 1, dp, d, s * tp + tt, S * tp,
                              (uint64_t)((tp > 1 ? dp * S : 0) + s * tp + tt), ndp, s * tp + tt);
-                    if (TR.phot)
+                    if constexpr (NW > 1) {
+                        ph_tables(TR.phot);
+                        if (!TR.phot && last_phot)   // the link counters must start at 0 again
+                            for (int q = (int)threadIdx.x; q < LMAX; q += NTHR) { ln[q] = 0; lk[q] = 0; }
+                        last_phot = TR.phot;
+                    }
+                    if (TR.phot) {
                         for (int k = 0; k < ports; k++) p_st[k * NTHR + threadIdx.x] = 0;
+                        for (int k = 0; k < 3; k++) q_g[threadIdx.x * 3 + k] = 0;
+                    }
                     if (used && !TR.phot) {
                         // route checks of every pair this rank's flows will use (R3)
                         auto chk = [&](uint32_t x, uint32_t y) {
                             const int l = route_len(a, TR, x, y);
-                            if (l == NO_ROUTE) rbad = true;
-                            else if (l > MAX_HOPS) rlong = true;
+                            if (l == NO_ROUTE) rbad = true;   // (any length: hops past MAX_HOPS are read from rt_links)
                         };
                         for (int gk = 0; gk < 2; gk++) {
                             const Group &G = gk == 0 ? GT : GD;
@@ -659,6 +733,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             if (C->need_ring) chk(gpu, gpu_of_member(G, (G.i + 1) % G.p));
                             if (C->need_tree && G.i >= 1) {
                                 const uint32_t par = gpu_of_member(G, (G.i - 1) / 2);
+                                chk(gpu, par);
+                                chk(par, gpu);
+                            }
+                            if (C->need_tree && dbt_algo && G.p - 1 - G.i >= 1) {   // R27 tree B's edge to its parent
+                                const uint32_t par = gpu_of_member(G, G.p - 1 - (G.p - 2 - G.i) / 2);
                                 chk(gpu, par);
                                 chk(par, gpu);
                             }
@@ -709,8 +788,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 }
                 // (b) / (c) for the three flow slots
                 if (used) {
-                    if (flow_step(FT, dirty)) { nflow++; grp_delivered(GT); }
-                    if (flow_step(FD, dirty)) { nflow++; grp_delivered(GD); }
+                    // R27: with a double binary tree, the group's tree B runs on the other group's (absent) slot
+                    if (flow_step(FT, dirty)) { nflow++; if (dbt_algo && dp > 1) grp_delivered2(GD); else grp_delivered(GT); }
+                    if (flow_step(FD, dirty)) { nflow++; if (dbt_algo && tp > 1) grp_delivered2(GT); else grp_delivered(GD); }
                     if (flow_step(FP, dirty)) {
                         nflow++; np2p++; dcnt++;
                         if constexpr (BD)
@@ -720,8 +800,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 cnt[li] = dcnt;
                 ssync();
                 // (d) both groups, then this rank's next P2P send
-                grp_pass(GT, FT, true, more);
-                grp_pass(GD, FD, false, more);
+                grp_pass(GT, FT, FD, true, more);
+                grp_pass(GD, FD, FT, false, more);
                 if (used && FP.st == FS_NONE && sq < nsend_tot) {
                     uint32_t P, j, e;
                     if (sq < m * SI.SF) { P = 0; j = sq / SI.SF; e = sq % SI.SF; }
@@ -812,7 +892,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             // (f') R20 photonic network: (i) a logical link per request, (ii) link heads ask for a
             // receive buffer, (iii) destinations grant buffers in (release time, code) order
             const bool phw = TR.phot && used && (FT.st >= PS_REQ || FD.st >= PS_REQ || FP.st >= PS_REQ);
-            if (vany(phw)) {
+            if ((NW == 1 || TR.phot) && vany(phw)) {   // (a CTA segment runs one point: TR.phot is uniform)
                 const int me = (int)threadIdx.x;
                 auto onlink = [&](int k) -> bool {   // a transfer of this lane is queued on / using link k
                     auto u = [&](const Flow &F) { return (F.st >= PS_LINKQ || F.st == FS_ACT) && (int)F.hl[1] == k; };
@@ -821,14 +901,19 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 auto klt = [](double ta, uint64_t ca, double tb, uint64_t cb) { return ta < tb || (ta == tb && ca < cb); };
                 if (phw) {
                     // (i) requests in key order: existing link, free port, else tear down the link idle longest
+                    // (the slots are chosen by index, never by address: a Flow whose address is taken would
+                    // live in local memory for the whole kernel)
+                    auto with_slot = [&](int k, auto &&fn) { if (k == 0) fn(FT); else if (k == 1) fn(FD); else fn(FP); };
                     for (int r = 0; r < 3; r++) {
-                        Flow *best = nullptr;
-                        auto pick = [&](Flow &F) {
-                            if (F.st == PS_REQ && F.len == 0 && (!best || klt(F.t_upd, F.code, best->t_upd, best->code))) best = &F;
+                        int bi = -1;
+                        double bt = 0.0;
+                        uint64_t bc = 0;
+                        auto pick = [&](const Flow &F, int k) {
+                            if (F.st == PS_REQ && F.len == 0 && (bi < 0 || klt(F.t_upd, F.code, bt, bc))) { bi = k; bt = F.t_upd; bc = F.code; }
                         };
-                        pick(FT); pick(FD); pick(FP);
-                        if (!best) break;
-                        Flow &F = *best;
+                        pick(FT, 0); pick(FD, 1); pick(FP, 2);
+                        if (bi < 0) break;
+                        with_slot(bi, [&](Flow &F) {
                         F.len = 1;   // visited in this pass
                         const int dg = (int)F.hl[0];
                         int k = -1;
@@ -854,24 +939,27 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             }
                         }
                         if (k >= 0) { F.st = PS_LINKQ; F.hl[1] = (uint32_t)k; }
+                        });
                     }
                     FT.len = FT.st == PS_REQ ? 0 : FT.len;
                     FD.len = FD.st == PS_REQ ? 0 : FD.len;
                     FP.len = FP.st == PS_REQ ? 0 : FP.len;
                     // (ii) an up link with nothing waiting for a buffer or moving passes its queue head on
                     for (int r = 0; r < 3; r++) {
-                        Flow *head = nullptr;
-                        auto hd = [&](Flow &F) {
+                        int hi = -1;
+                        double ht = 0.0;
+                        uint64_t hc = 0;
+                        auto hd = [&](const Flow &F, int q) {
                             if (F.st != PS_LINKQ) return;
                             const int k = (int)F.hl[1];
                             if (p_st[k * NTHR + me] != 2) return;
                             auto busy = [&](const Flow &G) { return (G.st == PS_BUFW || G.st == FS_ACT) && (int)G.hl[1] == k; };
                             if (busy(FT) || busy(FD) || busy(FP)) return;
-                            if (!head || klt(F.t_upd, F.code, head->t_upd, head->code)) head = &F;
+                            if (hi < 0 || klt(F.t_upd, F.code, ht, hc)) { hi = q; ht = F.t_upd; hc = F.code; }
                         };
-                        hd(FT); hd(FD); hd(FP);
-                        if (!head) break;
-                        head->st = PS_BUFW;
+                        hd(FT, 0); hd(FD, 1); hd(FP, 2);
+                        if (hi < 0) break;
+                        with_slot(hi, [&](Flow &F) { F.st = PS_BUFW; });
                     }
                 }
                 // (iii) publish buffer requests and transfers, each destination grants in key order
@@ -952,123 +1040,117 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             progress(FT, aT);
             progress(FD, aD);
             progress(FP, aP);
-            // link counters are 0 here: every complete progressive filling returns them to 0
-            auto count = [&](const Flow &F, bool on) {
+            // link counters are 0 here: every complete progressive filling returns them to 0.  The first
+            // flow to count a link owns it for this call: it sets the residual, computes the share and
+            // updates both whenever flows on the link freeze (R14's single per-link expression)
+            unsigned lo = 0;   // owned links: bit slot * 8 + hop (the first MAX_HOPS hops)
+            unsigned lt = 0;   // bit slot: this slot owns links past MAX_HOPS (marked in lown)
+            auto count = [&](const Flow &F, bool on, int slot) {
                 if (on) {
                     alg += F.len;
 #pragma unroll
                     for (int h = 0; h < MAX_HOPS; h++)
                         if (h < F.len) {
                             const int e = hop(F.hl, h);
-                            atomicAdd(&ln[e], 1);
+                            if (atomicAdd(&ln[e], 1) == 0) {
+                                lo |= 1u << (slot * 8 + h);
+                                lres[e] = a.link_bw[TR.link_off + e] * bws;
+                            }
+                        }
+                    for (int h = MAX_HOPS; h < F.len; h++) {   // long routes
+                        const int e = a.rt_links[F.roff + h];
+                        if (atomicAdd(&ln[e], 1) == 0) {
+                            lown[e] = li * 4 + slot;
+                            lt |= 1u << slot;
                             lres[e] = a.link_bw[TR.link_off + e] * bws;
                         }
+                    }
                 }
             };
-            count(FT, aT);
-            count(FD, aD);
-            count(FP, aP);
+            count(FT, aT, 0);
+            count(FD, aD, 1);
+            count(FP, aP, 2);
             ssync();
-            // if no link carries two active flows, R14 is exactly "rate = smallest residual on the
-            // route" (n_e = 1: res_e / 1.0 == res_e) and the rounds are the distinct rates
-            auto alone = [&](const Flow &F, bool on) -> bool {
-                bool ok = true;
-                if (on) {
+            auto owned = [&](auto &&fn) {   // fn(link) for every link this lane owns
+                auto one = [&](const Flow &F, int slot) {
 #pragma unroll
                     for (int h = 0; h < MAX_HOPS; h++)
-                        if (h < F.len && ln[hop(F.hl, h)] != 1) ok = false;
-                }
-                return ok;
+                        if ((lo >> (slot * 8 + h)) & 1u) fn(hop(F.hl, h));
+                    if ((lt >> slot) & 1u)
+                        for (int h = MAX_HOPS; h < F.len; h++) {
+                            const int e = a.rt_links[F.roff + h];
+                            if (lown[e] == li * 4 + slot) fn(e);
+                        }
+                };
+                if (lo | lt) { one(FT, 0); one(FD, 1); one(FP, 2); }
             };
-            const bool disj = !sany(!(alone(FT, aT) && alone(FD, aD) && alone(FP, aP)));
+            owned([&](int e) { lsh[e] = lres[e] / (double)ln[e]; alg += 2; });
+            ssync();
+            // progressive filling: each round freezes every unfrozen flow crossing a link whose share is
+            // the minimum s; the owners then update those links' residual, count and share
             auto fmin = [&](const Flow &F, bool on) -> double {
                 double my = dinf();
                 if (on) {
 #pragma unroll
                     for (int h = 0; h < MAX_HOPS; h++)
                         if (h < F.len) {
-                            const int e = hop(F.hl, h);
-                            const double sh = lres[e] / (double)ln[e];
+                            const double sh = lsh[hop(F.hl, h)];
                             my = sh < my ? sh : my;
                         }
-                    alg += 2 * F.len;
+                    for (int h = MAX_HOPS; h < F.len; h++) {
+                        const double sh = lsh[a.rt_links[F.roff + h]];
+                        my = sh < my ? sh : my;
+                    }
                 }
                 return my;
             };
-            if (disj) {
-                auto solo = [&](Flow &F, bool on) {
-                    if (on) {
-                        F.rate = fmin(F, true);
-#pragma unroll
-                        for (int h = 0; h < MAX_HOPS; h++)
-                            if (h < F.len) ln[hop(F.hl, h)] = 0;
-                    }
-                };
-                solo(FT, aT);
-                solo(FD, aD);
-                solo(FP, aP);
-            }
-            ssync();
             bool uT = aT, uD = aD, uP = aP;
             uint32_t rounds = 0;
-            while (vany(uT || uD || uP)) {
-                const bool segact = sany(uT || uD || uP);
-                double mT, mD, mP;
-                if (disj) {
-                    mT = uT ? FT.rate : dinf();
-                    mD = uD ? FD.rate : dinf();
-                    mP = uP ? FP.rate : dinf();
-                } else {
-                    mT = fmin(FT, uT);
-                    mD = fmin(FD, uD);
-                    mP = fmin(FP, uP);
-                }
+            for (;;) {
+                const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
                 double my = mT < mD ? mT : mD;
                 my = mP < my ? mP : my;
-                const double sm = smin(my);
+                const double sm = smin(my);   // segment-uniform; +inf: nothing left to freeze
+                const bool segact = sm < dinf();
+                if constexpr (NW == 1) {
+                    if (!__any_sync(FULL, segact)) break;
+                } else {
+                    if (!segact) break;
+                }
                 const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
-                unsigned own = 0;
-                {
-                    // (disj is per segment: every lane still reaches both __syncwarp()s)
-                    auto freeze = [&](Flow &F, bool in, int slot) {
-                        if (in) {
-                            F.rate = sm;
-#pragma unroll
-                            for (int h = 0; h < MAX_HOPS; h++)
-                                if (h < F.len && atomicAdd(&lk[hop(F.hl, h)], 1) == 0) own |= 1u << (slot * 8 + h);
-                        }
-                    };
-                    if (!disj) {
-                        freeze(FT, iT, 0);
-                        freeze(FD, iD, 1);
-                        freeze(FP, iP, 2);
-                    }
-                    ssync();
-                    auto update = [&](const Flow &F, int slot) {
+                auto freeze = [&](Flow &F, bool in) {
+                    if (in) {
+                        F.rate = sm;
 #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
-                            if ((own >> (slot * 8 + h)) & 1u) {
-                                const int e = hop(F.hl, h);
-                                const int kk = lk[e];
-                                const double r = lres[e] - sm * (double)kk;
-                                lres[e] = r > 0.0 ? r : 0.0;
-                                ln[e] -= kk;
-                                lk[e] = 0;
-                                alg += 3;
-                            }
-                    };
-                    if (own) {
-                        update(FT, 0);
-                        update(FD, 1);
-                        update(FP, 2);
+                            if (h < F.len) atomicAdd(&lk[hop(F.hl, h)], 1);
+                        for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&lk[a.rt_links[F.roff + h]], 1);
                     }
-                }
+                };
+                freeze(FT, iT);
+                freeze(FD, iD);
+                freeze(FP, iP);
+                ssync();
+                owned([&](int e) {
+                    const int kk = lk[e];
+                    if (kk) {
+                        const double r = lres[e] - sm * (double)kk;
+                        const double rr = r > 0.0 ? r : 0.0;
+                        const int nn = ln[e] - kk;
+                        lres[e] = rr;
+                        ln[e] = nn;
+                        lk[e] = 0;
+                        if (nn > 0) lsh[e] = rr / (double)nn;
+                        alg += 5;
+                    }
+                });
                 ssync();
                 if (segact) rounds++;
                 uT = uT && !iT;
                 uD = uD && !iD;
                 uP = uP && !iP;
             }
+            // every link's count is back to 0 (all its flows froze)
             const uint32_t nact = scount(aT) + scount(aD) + scount(aP);
             if (segdirty) {
                 nwf++;
@@ -1089,19 +1171,12 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         }
 
         // ------------------------------ end of instant ------------------------------
-        const bool any_ev = sany(nev);
-        if (have && any_ev) ninst++;
-        nev = false;
-        const bool infl = sany(used && (FT.st != FS_NONE || FD.st != FS_NONE || FP.st != FS_NONE));
-        if (have) {
-            if (infl && !bon) { bon = true; bstart = t; }
-            else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
-        }
+        // the instant's end: did anything happen (R19 n_instants), is a flow in flight (R18 comm_busy),
+        // is every lane done, and the next event time -- one exchange in a CTA, segment votes in a warp
+        const bool myinfl = used && (FT.st != FS_NONE || FD.st != FS_NONE || FP.st != FS_NONE);
         const bool lane_done = !used || (cst == CS_IDLE && pos >= nprog && FT.st == FS_NONE && FD.st == FS_NONE &&
                                          FP.st == FS_NONE && sq >= nsend_tot && GT.cur >= GT.ncoll * (GT.member ? 1u : 0u) &&
                                          GD.cur >= GD.ncoll * (GD.member ? 1u : 0u) && !GT.running && !GD.running);
-        const bool alldone = !sany(!lane_done);
-        const bool fin = have && alldone;
         double cand = dinf();
         if (used) {
             if (cst == CS_RUN) cand = t_end;
@@ -1116,9 +1191,44 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 for (int k = 0; k < ports; k++)
                     if (p_st[k * NTHR + threadIdx.x] == 1 && p_t[k * NTHR + threadIdx.x] < cand) cand = p_t[k * NTHR + threadIdx.x];
         }
-        const double tn = smin(cand);
+        bool any_ev, infl, alldone;
+        double tn;
+        if constexpr (NW == 1) {
+            any_ev = sany(nev);
+            infl = sany(myinfl);
+            alldone = !sany(!lane_done);
+            tn = smin(cand);
+        } else {
+            const double wmin = seg_min<32>(cand);
+            const unsigned f = (__any_sync(FULL, nev) ? 1u : 0u) | (__any_sync(FULL, myinfl) ? 2u : 0u) |
+                               (__any_sync(FULL, !lane_done) ? 4u : 0u);
+            if (lane == 0) {
+                s_red[bb][wid] = wmin;
+                s_fl3[bb][wid] = f;
+            }
+            __syncthreads();
+            double r = s_red[bb][0];
+            unsigned fa = s_fl3[bb][0];
+#pragma unroll
+            for (int i = 1; i < NW; i++) {
+                r = s_red[bb][i] < r ? s_red[bb][i] : r;
+                fa |= s_fl3[bb][i];
+            }
+            bb ^= 1;
+            any_ev = (fa & 1u) != 0;
+            infl = (fa & 2u) != 0;
+            alldone = (fa & 4u) == 0;
+            tn = r;
+        }
+        if (have && any_ev) ninst++;
+        nev = false;
+        if (have) {
+            if (infl && !bon) { bon = true; bstart = t; }
+            else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
+        }
+        const bool fin = have && alldone;
         const bool stuck = have && !fin && !(tn < dinf());
-        if (vany(fin || stuck)) {
+        if ((NW > 1) ? (fin || stuck) : vany(fin || stuck)) {   // (a CTA segment: uniform, no vote needed)
             const double bmax = smax(used ? busy : 0.0);
             const unsigned long long ntk = ssum(ntask);
             const unsigned long long nfl = ssum(nflow);
@@ -1161,7 +1271,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
 size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
     const size_t nthr = W <= 32 ? K3_THREADS : (size_t)W;
     const size_t ph = pmax ? nthr * pmax * 16 + nthr * 3 * (8 + 8 + 4 + 1 + 1) : 0;
-    return (W <= 32 ? 0 : (size_t)lmax * 16) + ph;
+    if (W <= 32) return ph;
+    const size_t links = (size_t)lmax * 28 + 8;
+    return links > ph ? links : ph;   // a one-point CTA runs either a flow-network or a photonic point
 }
 
 template <int W, int NW, int V>

@@ -147,6 +147,26 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
         H[o].wait = -1;
         H[o].nsig = 0;
     }
+    if (C.strategy == TRIOSIM_HOP) {
+        // R28: the update every worker sends each neighbour per iteration -- the left fold of its weight
+        // gradients' bytes' in production order -- and the iteration's boundaries
+        if (tid == 0) {
+            double S = 0.0;
+            for (int i = 0; i < T.scal[0]; i++) S = S + tensor_bytes(T, T.wgrad[i], C.r_b, 1, C.tp_mode);
+            const uint32_t n = C.p, h = C.tp_mode == TRIOSIM_HOP_DOUBLE_RING ? n / 2 : n;
+            const uint32_t deg = (h > 2 ? 3u : h == 2 ? 1u : 0u) + (C.tp_mode == TRIOSIM_HOP_DOUBLE_RING ? 1u : 0u);
+            C.hop_S = S;
+            C.hop_last = (uint32_t)T.scal[2];
+            C.hop_first = (uint32_t)T.scal[1];
+            C.n_coll = 0;
+            C.coll_payload = 0.0;
+            C.need_ring = C.need_tree = 0;
+            C.n_prog_max = T.n_ops;
+            C.n_compute = (uint64_t)n * C.m * T.n_ops;
+            C.n_flows = (uint64_t)n * C.m * deg;
+        }
+        return;
+    }
     const bool is_dp = C.strategy == TRIOSIM_DP || C.strategy == TRIOSIM_DDP;
     int32_t *coll_of = scratch + C.scratch_off;
     if (!is_dp)
@@ -154,14 +174,14 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
     __syncthreads();
     if (is_dp) {
         if (tid == 0) {
-            uint32_t nc = 0;
+            uint32_t nc = 0, nb = 0;   // collectives, gradient buckets
             double payload = 0.0;
             const int nw = T.scal[0], first_opt = T.scal[1], last_nonopt = T.scal[2];
             if (C.p > 1) {
                 int i = 0;
                 while (i < nw) {
                     // gradient bucket (reading Q5): greedy on the u64 byte sum, first cap per R24
-                    const uint64_t cap = bucket_cap(C, nc);
+                    const uint64_t cap = bucket_cap(C, nb);
                     uint64_t sum = 0;
                     double S = 0.0;
                     int j = i;
@@ -173,12 +193,17 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         if (cap == 0 || sum >= cap || j == nw) break;
                     }
                     int trig = (C.strategy == TRIOSIM_DDP) ? T.prod[T.wgrad[j - 1]] : last_nonopt;
-                    CE[nc].S = S;
-                    CE[nc].kind = CK_AR;
-                    CE[nc].layer = T.layer[trig];
-                    H[trig].nsig += 1;
-                    payload = payload + S;
-                    nc++;
+                    // R29: an AllReduce, or its ReduceScatter + AllGather pair (two collectives)
+                    const int parts = C.algo == TRIOSIM_ALGO_RSAG ? 2 : 1;
+                    for (int h = 0; h < parts; h++) {
+                        CE[nc].S = S;
+                        CE[nc].kind = parts == 1 ? CK_AR : h == 0 ? CK_RS : CK_AG;
+                        CE[nc].layer = T.layer[trig];
+                        H[trig].nsig += 1;
+                        payload = payload + S;
+                        nc++;
+                    }
+                    nb++;
                     i = j;
                 }
                 if (nc > 0 && first_opt != INT_MAX) H[first_opt].wait = (int32_t)nc - 1;
@@ -188,9 +213,9 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
             C.need_ring = nc > 0 && C.algo != TRIOSIM_ALGO_TREE;
             C.need_tree = nc > 0 && C.algo == TRIOSIM_ALGO_TREE;
             C.n_compute = (uint64_t)C.p * T.n_ops;
-            uint64_t fl = C.algo == TRIOSIM_ALGO_RING ? 2ull * (C.p - 1) * C.p * C.nch
+            uint64_t fl = (C.algo == TRIOSIM_ALGO_RING || C.algo == TRIOSIM_ALGO_RSAG) ? 2ull * (C.p - 1) * C.p * C.nch
                         : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (C.p - 1) * C.nch : 2ull * (C.p - 1);
-            C.n_flows = fl * nc;
+            C.n_flows = fl * nb;
             C.n_prog_max = T.n_ops;
         }
     } else {
@@ -216,6 +241,16 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         if (kind < 0) continue;
                         double S = (double)T.ts[x].bytes_b0;
                         if (T.ts[x].batch_scaled) S = S * C.r_b;
+                        const bool split = kind == CK_AR && C.algo == TRIOSIM_ALGO_RSAG;
+                        if (split) {   // R29: ReduceScatter, then AllGather
+                            CE[nc].S = S;
+                            CE[nc].kind = CK_RS;
+                            CE[nc].layer = T.layer[o];
+                            H[o].nsig += 1;
+                            payload = payload + S;
+                            nc++;
+                            kind = CK_AG;
+                        }
                         CE[nc].S = S;
                         CE[nc].kind = (uint32_t)kind;
                         CE[nc].layer = T.layer[o];
@@ -225,7 +260,7 @@ __global__ void __launch_bounds__(256) k2_coll(ClassDesc *cls, const uint32_t *l
                         if (kind == CK_AG) any_ag = 1; else any_ar = 1;
                         if (kind == CK_AR && C.algo == TRIOSIM_ALGO_TREE) nfl += 2ull * (C.p - 1);
                         else if (kind == CK_AR && C.algo == TRIOSIM_ALGO_REDBCAST) nfl += 2ull * (C.p - 1) * C.nch;
-                        else nfl += (kind == CK_AR ? 2ull : 1ull) * (C.p - 1) * C.p * C.nch;
+                        else nfl += (kind == CK_AR || split ? 2ull : 1ull) * (C.p - 1) * C.p * C.nch;
                         nc++;
                     }
                 }
@@ -485,7 +520,10 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                 const unsigned long long r = readers[x] & ~(1ull << s);
                 sn[op.phase] += __popcll(r);
                 dmask |= r;
-                if (tp > 1 && tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode) >= 0) tn[op.phase]++;
+                if (tp > 1) {
+                    const int kd = tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode);
+                    if (kd >= 0) tn[op.phase] += (kd == CK_AR && C.algo == TRIOSIM_ALGO_RSAG) ? 2 : 1;   // R29 pairs
+                }
             }
             for (uint32_t k = 0; k < op.n_in; k++) {
                 const int32_t po = T.prod[T.io[op.io_off + k]];
@@ -510,6 +548,7 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
         SI[s].nF = n[0]; SI[s].nB = n[1]; SI[s].nO = n[2];
         SI[s].SF = sn[0]; SI[s].SB = sn[1]; SI[s].SO = sn[2];
         SI[s].dst_mask = dmask;
+        if (C.algo == TRIOSIM_ALGO_RSAG) nb *= 2;   // R29: each bucket's ReduceScatter + AllGather
         HS[s].TF = tn[0]; HS[s].TB = tn[1]; HS[s].TO = tn[2];
         HS[s].ndp = nb;
         HS[s].first_opt = n[2] > 0 ? 0u : 0xffffffffu;
@@ -563,15 +602,23 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     nsend++;
                 }
                 if (tp > 1) {
-                    const int kind = tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode);
+                    int kind = tp_kind_dev(op.tp_role, op.phase, T.ts[x].category, C.tp_mode);
                     if (kind >= 0) {
                         CollEnt ce;
                         ce.S = (double)T.ts[x].bytes_b0;
                         if (T.ts[x].batch_scaled) ce.S = ce.S * C.r_b;
-                        ce.kind = (uint32_t)kind;
-                        ce.pad = x;
                         ce.layer = op.layer;
                         ce.pad2 = 0;
+                        if (kind == CK_AR && C.algo == TRIOSIM_ALGO_RSAG) {
+                            // R29: the ReduceScatter half (no reader waits on it: pad = no tensor), then the AllGather
+                            ce.kind = CK_RS;
+                            ce.pad = 0xffffffffu;
+                            colls[toff[P] + tj[P]++] = ce;
+                            ntp++;
+                            kind = CK_AG;
+                        }
+                        ce.kind = (uint32_t)kind;
+                        ce.pad = x;
                         colls[toff[P] + tj[P]++] = ce;
                         ntp++;
                     }
@@ -607,7 +654,7 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     last_prod = T.prod[x];
                     open = true;
                 }
-                const uint64_t cap = bucket_cap(C, b);
+                const uint64_t cap = bucket_cap(C, C.algo == TRIOSIM_ALGO_RSAG ? b / 2 : b);   // b counts collectives (R29: 2 per bucket)
                 if (open && (end || cap == 0 || sum >= cap)) {
                     CollEnt ce;
                     ce.S = Sb;
@@ -617,15 +664,21 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                     ce.pad2 = 0;
                     // trigger: (producer of the bucket's last gradient, micro-batch 0); the HYBRID form
                     // of DataParallel (R6) triggers every bucket after the stage's last non-OPT op
+                    const uint16_t parts = C.algo == TRIOSIM_ALGO_RSAG ? 2 : 1;   // R29: RS + AG pair
                     if (C.dp_after_bwd && (si.nB > 0 || si.nF > 0)) {
                         HEnt &te = ents[si.nB > 0 ? eoff[1] + si.nB - 1 : eoff[0] + si.nF - 1];
-                        te.dp_nsig++;
+                        te.dp_nsig += parts;
                         ce.layer = T.layer[te.op];
                     } else {
                         const int P = (int)(T.info[last_prod] & INFO_PHASE_MASK);
                         const uint32_t cntP = P == 0 ? si.nF : P == 1 ? si.nB : si.nO;
                         for (uint32_t q = 0; q < cntP; q++)
-                            if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig++; break; }
+                            if (ents[eoff[P] + q].op == (uint32_t)last_prod) { ents[eoff[P] + q].dp_nsig += parts; break; }
+                    }
+                    if (parts == 2) {
+                        ce.kind = CK_RS;
+                        colls[hs.dcol_off + b++] = ce;
+                        ce.kind = CK_AG;
                     }
                     colls[hs.dcol_off + b++] = ce;
                     sum = 0;
@@ -736,8 +789,9 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                 for (uint32_t e = 0; e < hs.TF + hs.TB + hs.TO; e++) {
                     const uint32_t kind = colls[hs.tcol_off + e].kind;
                     const uint64_t reps = e < hs.TF + hs.TB ? m : 1;
-                    const uint64_t per = kind == CK_AG ? (uint64_t)(tp - 1) * tp * C.nch
+                    const uint64_t per = (kind == CK_AG || kind == CK_RS) ? (uint64_t)(tp - 1) * tp * C.nch
                                        : C.algo == TRIOSIM_ALGO_TREE ? 2ull * (tp - 1)
+                                       : C.algo == TRIOSIM_ALGO_DBTREE ? 4ull * (tp - 1)
                                        : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (tp - 1) * C.nch : 2ull * (tp - 1) * tp * C.nch;
                     nflow += reps * per;
                     ncoll += reps;
@@ -749,7 +803,9 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
                 for (uint32_t b = 0; b < HS[s].ndp; b++) {
                     payload = payload + colls[HS[s].dcol_off + b].S;
                     nflow += C.algo == TRIOSIM_ALGO_TREE ? 2ull * (dp - 1)
-                           : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (dp - 1) * C.nch : 2ull * (dp - 1) * dp * C.nch;
+                           : C.algo == TRIOSIM_ALGO_DBTREE ? 4ull * (dp - 1)
+                           : C.algo == TRIOSIM_ALGO_REDBCAST ? 2ull * (dp - 1) * C.nch
+                           : C.algo == TRIOSIM_ALGO_RSAG ? 1ull * (dp - 1) * dp * C.nch : 2ull * (dp - 1) * dp * C.nch;
                     ncoll++;
                     any_ar = 1;
                 }
@@ -758,8 +814,8 @@ __global__ void __launch_bounds__(K2P_THREADS) k2_hybrid(ClassDesc *cls, const u
         C.n_coll = (uint32_t)ncoll;
         C.coll_payload = payload;
         C.n_prog_max = pmax;
-        C.need_ring = any_ag || (any_ar && C.algo != TRIOSIM_ALGO_TREE);
-        C.need_tree = any_ar && C.algo == TRIOSIM_ALGO_TREE;
+        C.need_ring = any_ag || (any_ar && C.algo != TRIOSIM_ALGO_TREE && C.algo != TRIOSIM_ALGO_DBTREE);
+        C.need_tree = any_ar && (C.algo == TRIOSIM_ALGO_TREE || C.algo == TRIOSIM_ALGO_DBTREE);
     }
 }
 
@@ -790,6 +846,10 @@ __global__ void __launch_bounds__(128) k4_layer_compute(const ClassDesc *cls, Tr
         if (C.mode == MODE_COLL || C.mode == MODE_TREE) {
             for (uint32_t o = 0; o < T.n_ops; o++)
                 if (T.layer[o] == l) acc = acc + du[o];
+        } else if (C.mode == MODE_HOP) {   // R28: rank 0 runs every operator once per iteration
+            for (uint32_t k = 0; k < C.m; k++)
+                for (uint32_t o = 0; o < T.n_ops; o++)
+                    if (T.layer[o] == l) acc = acc + du[o];
         } else {
             const bool hyb = C.mode == MODE_HYBRID;
             auto op_at = [&](uint32_t e) -> uint32_t { return hyb ? hents[e].op : ents[e].op; };

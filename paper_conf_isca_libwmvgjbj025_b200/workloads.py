@@ -63,7 +63,7 @@ OPF_BATCH_SCALED = 1
 ST_DP, ST_DDP, ST_TP, ST_PP, ST_HYBRID, ST_HOP = range(6)
 HOP_RING_BASED, HOP_DOUBLE_RING = 0, 1   # R28 communication graphs (Fig. 16a), in tp_mode
 TPM_PAPER, TPM_MEGATRON = 0, 1
-ALG_RING, ALG_TREE, ALG_REDBCAST, ALG_DBTREE = 0, 1, 2, 3
+ALG_RING, ALG_TREE, ALG_REDBCAST, ALG_DBTREE, ALG_RSAG = 0, 1, 2, 3, 4
 PT_OK, PT_BAD_BATCH, PT_BAD_DEGREES, PT_NO_ROUTE, PT_TOO_LARGE, PT_DEADLOCK, PT_BAD_PLAN, PT_BAD_CONFIG = range(8)
 
 MiB = 1 << 20
@@ -395,6 +395,38 @@ def resnet50_trace(b0=128, seed=2) -> Trace:
     tb.backward()
     tb.optimizer()
     return tb.build(model="resnet50")
+
+
+def vgg11_trace(b0=128, seed=6) -> Trace:
+    """VGG-11 (224x224, fp32): 8 conv + ReLU (max pools after conv 1, 2, 4, 6, 8), 3 linear layers -> 14
+    parameter tensors (bias-free convolutions, as TraceBuilder.conv), 132.9 M parameters; the Hop case study's
+    model at its batch size 128."""
+    tb = TraceBuilder("vgg11", b0, seed)
+    tb.start()
+    img = tb.tensor(b0 * 3 * 224 * 224 * 4, CAT_INPUT, True)
+    labels = tb.tensor(b0 * 8, CAT_INPUT, True)
+    h, hw, cin = img, 224, 3
+    layer = 0
+    for cout, pool in ((64, True), (128, True), (256, False), (256, True), (512, False), (512, True),
+                       (512, False), (512, True)):
+        tb.layer = layer
+        h, hw = tb.conv(h, cin, cout, 3, 1, hw, b0)
+        h = tb.pointwise(h, "relu")
+        if pool:
+            hw //= 2
+            h = tb.resize(h, b0 * cout * hw * hw * 4, "max_pool2d")
+        cin = cout
+        layer += 1
+    for fin, fout in ((512 * 7 * 7, 4096), (4096, 4096), (4096, 1000)):
+        tb.layer = layer
+        h = tb.linear(h, fin, fout, b0)
+        if fout != 1000:
+            h = tb.pointwise(h, "relu")
+        layer += 1
+    tb.loss(h, labels)
+    tb.backward()
+    tb.optimizer()
+    return tb.build(model="vgg11")
 
 
 def transformer_trace(name, n_layers, hidden, heads, ffn, seq, vocab, b0, seed, causal_head=True,
@@ -831,7 +863,8 @@ def c5_parity_index(full: Sweep, per_n=20, heavy=4, seed=55) -> np.ndarray:
     simulated-GPU count N, `heavy` points of the heavy classes -- data x tensor parallel degree
     dp * tp = 64 (the verdict's "dp x tp >= 64" at its smallest product, which keeps each point at
     1e6-1e7 instants), on the perturbed (slow-link subset) topology at 4:1 oversubscription, with 8
-    micro-batches -- plus seeded random points with 8 micro-batches."""
+    micro-batches -- plus seeded random points with 8 micro-batches and dp * tp <= 64 (none heavier than
+    the heavy class)."""
     P = full.points
     N = P["dp"].astype(np.int64) * P["tp"] * P["pp"]
     rng = np.random.Generator(np.random.PCG64(seed))
@@ -842,7 +875,7 @@ def c5_parity_index(full: Sweep, per_n=20, heavy=4, seed=55) -> np.ndarray:
         hv = np.flatnonzero(sel & (P["dp"].astype(np.int64) * P["tp"] == 64) & (P["topo"] % 2 == 1)
                             & (np.char.find(topo_ov[P["topo"]].astype(str), "o4") >= 0))
         hv = hv[rng.permutation(len(hv))][:heavy]
-        rest = np.setdiff1d(np.flatnonzero(sel), hv)
+        rest = np.setdiff1d(np.flatnonzero(sel & (P["dp"].astype(np.int64) * P["tp"] <= 64)), hv)
         idx += hv.tolist() + rest[rng.permutation(len(rest))][:per_n - len(hv)].tolist()
     return np.asarray(sorted(idx), np.int64)
 
@@ -851,6 +884,38 @@ def sweep_c5_parity() -> Sweep:
     """The C5 parity / bench subset: c5_parity_index over the full configs[4] sweep (100 points)."""
     full = sweep_c5()
     return Sweep(full.name + "_parity", full.trace, full.topos, full.points[c5_parity_index(full)])
+
+
+def sweep_hop(trace=None, seed=7, groups=8, n_bw=5, n_lat=2) -> Sweep:
+    """NEXT 4: the Hop case study (Fig. 16).  VGG-11 at batch 128 per worker on 8
+    A100-class workers; communication graphs ring-based and double ring (Fig. 16a), each a topology whose
+    links are exactly the graph's edges; `groups` random slowdown scenarios that divide every GPU's link
+    bandwidth by U[1, 10]; without and with one backup worker (and bounded staleness 0 / 1, token
+    gap 0 / 2); 10 iterations; n_bw bandwidth x n_lat latency scales -> 8 x 2 x 2 x 2 x 5 x 2 = 640 points
+    (seeded order)."""
+    tr = trace if trace is not None else vgg11_trace()
+    rng = np.random.Generator(np.random.PCG64(seed))
+    topos = []
+    for g in range(groups):
+        u = rng.uniform(1.0, 10.0, 8)
+        for graph, mk in ((HOP_RING_BASED, ring_graph), (HOP_DOUBLE_RING, double_ring)):
+            t = mk(8, bw=50e9, lat=2e-6)
+            links = t.links.copy()
+            links["bw_Bps"] = links["bw_Bps"] / u[links["src"]]
+            topos.append((graph, Topology(f"{t.name}~g{g}", t.n_nodes, t.n_gpus, links, np.arange(8, dtype=np.uint32))))
+    bws = np.logspace(np.log10(0.25), np.log10(4.0), n_bw)
+    lats = np.logspace(np.log10(0.5), np.log10(2.0), n_lat)
+    pts = []
+    for ti, (graph, _) in enumerate(topos):
+        for b in (0, 1):
+            for st, gap in ((0, 0), (1, 2)):
+                for bw in bws:
+                    for lat in lats:
+                        pts.append(make_point(ti, ST_HOP, dp=8, m=10, B=8 * 128, tp_mode=graph, bw=float(bw),
+                                              lat=float(lat), hop=(b, st, gap)))
+    arr = points_array(pts)
+    perm = np.random.Generator(np.random.PCG64(seed + 1)).permutation(len(arr))
+    return Sweep("hop_vgg11_fig16", tr, [t for _, t in topos], arr[perm])
 
 
 def sweep_wafer(trace=None, seed=6, n_bw=10, n_lat=5) -> Sweep:

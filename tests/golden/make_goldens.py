@@ -39,7 +39,9 @@ SWEEPS = {"c1": W.sweep_c1, "c2": W.sweep_c2, "c3": W.sweep_c3, "c4": W.sweep_c4
 
 def sweep_digest(sw) -> str:
     h = hashlib.sha256()
-    for a in (sw.trace.ops, sw.trace.tensors, sw.trace.io, sw.points):
+    ops = np.array(sw.trace.ops, copy=True)
+    ops["kind"] = 0   # informational operator-name ids, numbered in first-use order per process
+    for a in (ops, sw.trace.tensors, sw.trace.io, sw.points):
         h.update(np.ascontiguousarray(a).tobytes())
     for t in sw.topos:
         h.update(np.ascontiguousarray(t.links).tobytes())
@@ -72,15 +74,41 @@ def make(name, procs):
     chunks = [list(range(a, min(n, a + chunk))) for a in range(0, n, chunk)]
     rec = np.zeros(n, W.RESULT_DTYPE)
     secs = np.zeros(n)
+    # resumable: finished points are appended to <name>.partial (point bytes -> record), reused on a rerun
+    part = os.path.join(HERE, f"{name}.partial.npz")
+    cache = {}
+    if os.path.exists(part):
+        z = np.load(part)
+        for pb, rb, sc in zip(z["points"], z["records"], z["secs"]):
+            cache[pb.tobytes()] = (rb, float(sc))
+    todo = []
+    for c in chunks:
+        hit = [cache.get(sw.points[i].tobytes()) for i in c]
+        if all(h is not None for h in hit):
+            for i, h in zip(c, hit):
+                rec[i] = h[0].view(W.RESULT_DTYPE)[0]
+                secs[i] = h[1]
+        else:
+            todo.append(c)
+    if name == "c5":   # the heaviest-looking first, so the long points start at once
+        todo.sort(key=lambda c: -float(sw.points[c[0]]["dp"]) * float(sw.points[c[0]]["tp"]) * float(sw.points[c[0]]["pp"]))
+
+    def save_partial():
+        done = [i for i in range(n) if secs[i] > 0 or rec[i]["status"] != 0 or rec[i]["n_instants"] > 0]
+        np.savez(part, points=sw.points[done].view(np.uint8).reshape(len(done), -1),
+                 records=rec[done].view(np.uint8).reshape(len(done), -1), secs=secs[done])
     t0 = time.perf_counter()
     with mp.get_context("spawn").Pool(procs) as pool:
-        for k, (idx, r, dt) in enumerate(pool.imap_unordered(_work, [(name, c) for c in chunks])):
+        for k, (idx, r, dt) in enumerate(pool.imap_unordered(_work, [(name, c) for c in todo])):
             rec[idx] = r
-            secs[idx] = dt / len(idx)
+            secs[idx] = max(dt / len(idx), 1e-9)
             if name == "c5":
                 print(f"  {name} point {idx[0]}: {dt:.1f} s, {int(r['n_instants'][0])} instants", flush=True)
+                save_partial()
     out = os.path.join(HERE, f"{name}.npz")
     np.savez_compressed(out, records=rec.view(np.uint8), n=n, digest=sweep_digest(sw), oracle_s=secs)
+    if os.path.exists(part):
+        os.remove(part)
     print(f"{name}: {n} points in {time.perf_counter() - t0:.1f} s -> {out} "
           f"({os.path.getsize(out)} B); statuses {np.bincount(rec['status'])}", flush=True)
 

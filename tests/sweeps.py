@@ -156,7 +156,21 @@ def random_chunked(seed):
 def random_redbcast(seed):
     """R26 AllReduce as ring Reduce + ring Broadcast (0-6 chunks) for DP / DDP / TP / HYBRID on uniform and
     asymmetric rings, a star, random graphs, a photonic net and 64-rank points (CTA kernel)."""
-    rng = np.random.Generator(np.random.PCG64(2600 + seed))
+    return _random_algo(seed, W.ALG_REDBCAST, 2600, "redbcast")
+
+
+def random_rsag(seed):
+    """R29 AllReduce as ring ReduceScatter + ring AllGather (0-6 chunks), the same mix as random_redbcast."""
+    return _random_algo(seed, W.ALG_RSAG, 3600, "rsag")
+
+
+def random_dbtree(seed):
+    """R27 double binary tree AllReduce (chunks ignored) on the GPU, the same mix as random_redbcast."""
+    return _random_algo(seed, W.ALG_DBTREE, 4600, "dbtree")
+
+
+def _random_algo(seed, algo, base, name):
+    rng = np.random.Generator(np.random.PCG64(base + seed))
     tr = W.random_trace(rng, n_layers=int(rng.integers(3, 6)), max_ops_per_layer=3, b0=2)
     topos = [W.ring(8, 50e9, 1e-6), W.ring(16, 100e9, 2e-6), W.star(8, 80e9, 1e-6),
              W.random_topology(rng, n_gpus=6, n_switch=1, p_edge=0.3), W.perturb(W.ring_graph(8, 90e9, 1e-6), seed),
@@ -171,7 +185,7 @@ def random_redbcast(seed):
         c = int(rng.integers(0, 7))
         bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
         full = G == 64 or rng.random() < 0.5
-        kw = dict(algo=W.ALG_REDBCAST, bw=bw, lat=lat, chunks=c)
+        kw = dict(algo=algo, bw=bw, lat=lat, chunks=c)
         if st in (W.ST_DP, W.ST_DDP):
             dp = G if full else int(rng.integers(1, G + 1))
             pts.append(P(ti, st, dp=dp, B=dp * 2, bucket=int(rng.choice([0, 1 << 12, 1 << 30])), **kw))
@@ -186,5 +200,49 @@ def random_redbcast(seed):
             m = int(rng.integers(1, 3))
             pts.append(P(ti, st, dp=dp, tp=tpd, pp=pp, m=m, B=dp * m * 2, bucket=int(rng.choice([0, 1 << 12, 1 << 30])),
                          tp_mode=int(rng.integers(0, 2)), **kw))
-    pts.append(P(0, W.ST_DDP, dp=8, B=16, algo=4))   # unknown algorithm -> BAD_CONFIG
-    return W.Sweep("redbcast", tr, topos, W.points_array(pts))
+    pts.append(P(0, W.ST_DDP, dp=8, B=16, algo=7))   # unknown algorithm -> BAD_CONFIG
+    return W.Sweep(name, tr, topos, W.points_array(pts))
+
+
+def random_hop(seed):
+    """R28 Hop points: both Fig. 16a graphs, 2-32 workers, backup workers / staleness / iteration gap, on
+    topologies with dedicated links (ring-based, double ring), shared links (star, mesh, random) and the
+    paper's 1-10x per-GPU slowdowns (P:356), mixed with DDP points so both kernels' segments share warps;
+    the last point is invalid (odd worker count)."""
+    rng = np.random.Generator(np.random.PCG64(2100 + seed))
+    tr = W.random_trace(rng, n_layers=int(rng.integers(2, 6)), max_ops_per_layer=3, b0=2)
+    if not (tr.ops["phase"] == W.PH_OPT).any():
+        tr = W.random_trace(np.random.Generator(np.random.PCG64(1)), n_layers=3, max_ops_per_layer=3, b0=2)
+
+    def ident(t):
+        return W.Topology(t.name, t.n_nodes, t.n_gpus, t.links.copy(), np.arange(t.n_gpus, dtype=np.uint32))
+
+    def slow(t, s):
+        r = np.random.Generator(np.random.PCG64(s))
+        u = r.uniform(1.0, 10.0, t.n_nodes)
+        t = ident(t)
+        t.links["bw_Bps"] = t.links["bw_Bps"] / u[t.links["src"]]
+        return t
+    topos = [ident(W.ring_graph(8, 25e9, 2e-6)), ident(W.double_ring(8, 25e9, 2e-6)),
+             slow(W.ring_graph(8, 25e9, 2e-6), seed), slow(W.double_ring(8, 25e9, 2e-6), seed + 7),
+             W.star(8, 40e9, 1e-6), W.mesh(2, 4, 30e9, 1e-6), ident(W.ring_graph(16, 30e9, 1e-6)),
+             W.star(32, 60e9, 1e-6), W.random_topology(rng, n_gpus=4, n_switch=1, p_edge=0.4),
+             slow(W.ring_graph(4, 20e9, 3e-6), seed + 3)]
+    pts = []
+    for _ in range(300):
+        ti = int(rng.integers(len(topos)))
+        G = topos[ti].n_gpus
+        bw, lat = float(rng.uniform(0.3, 3.0)), float(rng.uniform(0.0, 2.0))
+        if rng.random() < 0.15:
+            dp = int(rng.integers(1, G + 1))
+            pts.append(W.make_point(ti, W.ST_DDP, dp=dp, B=dp * 2, bw=bw, lat=lat))
+            continue
+        graph = int(rng.integers(0, 2))
+        cand = [n for n in (2, 4, 8, 16, 32) if n <= G and (graph == 0 or n % 4 == 0)]
+        n = int(rng.choice(cand))
+        K = int(rng.integers(1, 6))
+        hop = (int(rng.integers(0, 3)), int(rng.integers(0, 3)), int(rng.choice([0, 0, 1, 2])))
+        pts.append(W.make_point(ti, W.ST_HOP, dp=n, m=K, B=n * int(rng.integers(1, 4)), tp_mode=graph, bw=bw,
+                                lat=lat, hop=hop))
+    pts.append(W.make_point(0, W.ST_HOP, dp=7, m=2, B=7))
+    return W.Sweep("rand_hop", tr, topos, W.points_array(pts))

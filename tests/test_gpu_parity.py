@@ -317,3 +317,35 @@ def test_double_tree_rejected_until_implemented(ctx):
     assert got["status"][1] == 0
     check(got, sw, [1])
     assert oracle.run_point(tr, topos[0], pts[0])["status"] == 0
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_reduce_scatter_all_gather(ctx, seed):
+    """R29 AllReduce as ring ReduceScatter + ring AllGather (0-6 chunks) in the warp, hybrid, photonic and
+    64-rank CTA kernels, against the oracle point by point."""
+    sw = S.random_rsag(seed)
+    got = ctx.run_sweep(sw)
+    assert got["status"][-1] == W.PT_BAD_CONFIG
+    assert (got["status"][:-1] == 0).sum() > 170
+    assert (got["status"] == W.PT_TOO_LARGE).sum() <= 10
+    check(got, sw, list(range(len(sw.points))), allow_too_large=True)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_double_binary_tree(ctx, seed):
+    """R27 double binary tree AllReduce on the GPU (the hybrid kernel holds tree B on a spare flow slot):
+    every point against the oracle.  The documented limits (include/triosim.h TRIOSIM_ALGO_DBTREE) are the
+    only PT_TOO_LARGE points: HYBRID with both dp > 1 and tp > 1, and collectives over photonic links."""
+    sw = S.random_dbtree(seed)
+    got = ctx.run_sweep(sw)
+    assert got["status"][-1] == W.PT_BAD_CONFIG
+    P = sw.points[:-1]
+    phot = np.array([getattr(sw.topos[int(p["topo"])], "photonic", None) is not None for p in P])
+    both = (P["strategy"] == W.ST_HYBRID) & (P["dp"] > 1) & (P["tp"] > 1)
+    coll = np.where(P["strategy"] == W.ST_TP, P["tp"] > 1,
+                    np.where(P["strategy"] == W.ST_HYBRID, (P["dp"] > 1) | (P["tp"] > 1), P["dp"] > 1))
+    expect = np.flatnonzero(both | (phot & coll))
+    assert np.flatnonzero(got["status"][:-1] == W.PT_TOO_LARGE).tolist() == expect.tolist()
+    ok = [i for i in range(len(P)) if i not in set(expect.tolist())]
+    assert len(ok) > 100
+    check(got, sw, ok)

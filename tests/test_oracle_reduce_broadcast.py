@@ -88,7 +88,7 @@ def test_allgather_keeps_the_ring_and_limits():
     assert r_ring["status"] == 0 and r_rb["status"] == 0
     assert r_rb["coll_payload_bytes"] == r_ring["coll_payload_bytes"]
     assert r_rb["n_collectives"] == r_ring["n_collectives"]
-    assert oracle.run_point(tr, topo, W.make_point(0, W.ST_DDP, dp=4, B=64, algo=4))["status"] == W.PT_BAD_CONFIG
+    assert oracle.run_point(tr, topo, W.make_point(0, W.ST_DDP, dp=4, B=64, algo=7))["status"] == W.PT_BAD_CONFIG
 
 
 def test_hybrid_and_degenerate_groups():
