@@ -45,7 +45,9 @@ typedef int32_t triosim_status;
 #define TRIOSIM_PT_BAD_BATCH 1   /* global_batch not divisible by dp * microbatches (Q3, Q12) */
 #define TRIOSIM_PT_BAD_DEGREES 2 /* zero / inconsistent degrees, dp*tp*pp > GPUs, pp > layers or > 64 */
 #define TRIOSIM_PT_NO_ROUTE 3    /* a needed (src, dst) GPU pair has no path */
-#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits (> 1024 ranks, > 8192 links, > 8 hops) */
+#define TRIOSIM_PT_TOO_LARGE 4   /* exceeds this GPU kernel's limits: > 1024 ranks, > 6144 links on a > 32-rank point,
+                                    tree collectives over photonic links, a double binary tree on a HYBRID
+                                    point with both TP and DP groups, Hop beyond 32 workers (R3) */
 #define TRIOSIM_PT_DEADLOCK 5    /* the task graph cannot make progress */
 #define TRIOSIM_PT_BAD_PLAN 6    /* explicit stage plan invalid for this point */
 #define TRIOSIM_PT_BAD_CONFIG 7  /* unknown enum, topology index out of range, bw_scale <= 0, lat_scale < 0 */

@@ -574,7 +574,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             if (plans->off[k + 1] < plans->off[k]) return fail(ctx, TRIOSIM_EINVAL, "bad plan offsets");
 
     PhaseTimer PT;
-    static const int widen_from = getenv("TS_WIDEN_FROM") ? atoi(getenv("TS_WIDEN_FROM")) : 16;
+    static const int widen_from = getenv("TS_WIDEN_FROM") ? atoi(getenv("TS_WIDEN_FROM")) : 8;
     std::vector<HostTopo> HT(n_topos);
     for (uint32_t i = 0; i < n_topos; i++) {
         triosim_status st = prep_topology(ctx, topos[i], i, HT[i]);
@@ -706,9 +706,11 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto lm = [&](bool h, int w) { return !h ? lmax_warp(w) : w <= 32 ? lmax_hybrid(w) : LMAX_CTA; };
         int W0 = 2;
         while (W0 < (int)lanes) W0 <<= 1;
-        // DP / DDP / TP points of 9-16 GPUs run one per warp (W = 32) instead of two per warp: the two
-        // segments of a warp diverge on every event, and these heaviest points set the step (C2 3.18 ->
-        // 3.04 ms measured; results are identical for any W >= lanes).  TS_WIDEN_FROM=0 turns it off.
+        // DP / DDP / TP points of 5-16 GPUs run on twice their segment width (9-16: one per warp): the
+        // segments of a warp diverge on every event, and the spare lanes hash half of the ring
+        // fast-forward's events (R19) -- C2 3.69 -> 3.59 ms per step with 5-8 widened too (round 2; round 1,
+        // before the full-strength hash, measured 9-16 only as the better choice).  Results are identical
+        // for any W >= lanes.  TS_WIDEN_FROM=16 restores round 1's choice, 0 turns widening off.
         if (widen_from > 0 && W0 >= widen_from && W0 < 32 && pt.strategy != TRIOSIM_PP && pt.strategy != TRIOSIM_HYBRID)
             W0 <<= 1;
         // photonic points (R20) always run in the HYBRID kernel, whose lanes own their logical links;

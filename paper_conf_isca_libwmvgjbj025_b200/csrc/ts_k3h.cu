@@ -225,7 +225,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     if constexpr (NW > 1) {
         s_gc[0][threadIdx.x] = s_gc[1][threadIdx.x] = s_gc[2][threadIdx.x] = 0;
     }
-    if (PM > 0) {
+    if (NW == 1 && PM > 0) {   // (a CTA overlays its tables on the link arrays: set up per photonic point)
         for (int k = 0; k < PM; k++) p_st[k * NTHR + threadIdx.x] = 0;
         for (int k = 0; k < 3; k++) q_g[threadIdx.x * 3 + k] = 0;
     }
@@ -365,6 +365,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
     Group GT, GD;
     GT.member = GD.member = false;
+    GT.cross = GD.cross = false;
+    GT.tree_cur = GD.tree_cur = GT.dbt_cur = GD.dbt_cur = false;
     Flow FT, FD, FP;
     FT.st = FD.st = FP.st = FS_NONE;
     uint64_t acc = 0, alg = 0, tmix = 0;
@@ -446,9 +448,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         upb.bits = dnb.bits = zero.bits = 0;
         upb.p = dnb.p = zero.p = nullptr;
         upb.sel = dnb.sel = zero.sel = 1;
-        if ((tree_algo || dbt_algo) && vany(G.tree_cur)) flags2(G.upd, G.dnd, upb, dnb);   // (segment-uniform)
+        // (the vote / ballots must be warp-uniform: the segments of a warp may run different algorithms; a
+        // CTA segment skips the vote when its point runs no tree)
+        if ((NW == 1 || tree_algo || dbt_algo) && vany(G.tree_cur)) flags2(G.upd, G.dnd, upb, dnb);
         LF upb2 = zero, dnb2 = zero;
-        if (dbt_algo && vany(G.dbt_cur)) flags2(G.upd2, G.dnd2, upb2, dnb2);
+        if ((NW == 1 || dbt_algo) && vany(G.dbt_cur)) flags2(G.upd2, G.dnd2, upb2, dnb2);
         auto mb = [&](const LF &b, int k) -> bool { return b.test(G.lane0 + k * G.stride); };
         const int c1 = 2 * G.i + 1, c2 = 2 * G.i + 2;
         // R27's tree B: member i sits at heap position p - 1 - i
@@ -1054,6 +1058,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             const int e = hop(F.hl, h);
                             if (atomicAdd(&ln[e], 1) == 0) {
                                 lo |= 1u << (slot * 8 + h);
+                                lown[e] = li * 4 + slot;   // (so no stale owner mark of an earlier call matches)
                                 lres[e] = a.link_bw[TR.link_off + e] * bws;
                             }
                         }
@@ -1072,17 +1077,29 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             count(FP, aP, 2);
             ssync();
             auto owned = [&](auto &&fn) {   // fn(link) for every link this lane owns
-                auto one = [&](const Flow &F, int slot) {
-#pragma unroll
-                    for (int h = 0; h < MAX_HOPS; h++)
-                        if ((lo >> (slot * 8 + h)) & 1u) fn(hop(F.hl, h));
-                    if ((lt >> slot) & 1u)
-                        for (int h = MAX_HOPS; h < F.len; h++) {
-                            const int e = a.rt_links[F.roff + h];
-                            if (lown[e] == li * 4 + slot) fn(e);
-                        }
-                };
-                if (lo | lt) { one(FT, 0); one(FD, 1); one(FP, 2); }
+                // the cached hops: one bit scan (one copy of fn); the slot's words are selected, not
+                // addressed, so the flow slots stay in registers
+                for (unsigned m = lo; m; m &= m - 1) {
+                    const int b = __ffs(m) - 1, sl = b >> 3, h = b & 7, q = h >> 1;
+                    const uint32_t x0 = sl == 0 ? FT.hl[0] : sl == 1 ? FD.hl[0] : FP.hl[0];
+                    const uint32_t x1 = sl == 0 ? FT.hl[1] : sl == 1 ? FD.hl[1] : FP.hl[1];
+                    const uint32_t x2 = sl == 0 ? FT.hl[2] : sl == 1 ? FD.hl[2] : FP.hl[2];
+                    const uint32_t x3 = sl == 0 ? FT.hl[3] : sl == 1 ? FD.hl[3] : FP.hl[3];
+                    const uint32_t w = q == 0 ? x0 : q == 1 ? x1 : q == 2 ? x2 : x3;
+                    fn((int)((w >> (16 * (h & 1))) & 0xffffu));
+                }
+                if (lt) {   // hops past the cache (long routes): the owner marks
+                    auto tail = [&](const Flow &F, int slot) {
+                        if ((lt >> slot) & 1u)
+                            for (int h = MAX_HOPS; h < F.len; h++) {
+                                const int e = a.rt_links[F.roff + h];
+                                if (lown[e] == li * 4 + slot) fn(e);
+                            }
+                    };
+                    tail(FT, 0);
+                    tail(FD, 1);
+                    tail(FP, 2);
+                }
             };
             owned([&](int e) { lsh[e] = lres[e] / (double)ln[e]; alg += 2; });
             ssync();

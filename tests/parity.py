@@ -29,3 +29,20 @@ def compare(got, ref, idx=None, allow_too_large=False):
             elif a != b:
                 ulp += 1
     return bad, ulp
+
+
+def expected_too_large(sw):
+    """Indices of the points the library documents as beyond its kernels (include/triosim.h
+    TRIOSIM_PT_TOO_LARGE) that the oracle still simulates: tree / double-tree collectives over photonic
+    links (for points that have a collective group) and double binary trees on HYBRID points with both a
+    TP and a DP group."""
+    P = sw.points
+    phot = np.array([getattr(sw.topos[int(p["topo"])], "photonic", None) is not None if p["topo"] < len(sw.topos)
+                     else False for p in P], bool)
+    coll = np.where(P["strategy"] == W.ST_TP, P["tp"] > 1,
+                    np.where(P["strategy"] == W.ST_HYBRID, (P["dp"] > 1) | (P["tp"] > 1),
+                             np.where(P["strategy"] == W.ST_PP, False, P["dp"] > 1)))
+    trees = (P["coll_algo"] == W.ALG_TREE) | (P["coll_algo"] == W.ALG_DBTREE)
+    both = (P["strategy"] == W.ST_HYBRID) & (P["dp"] > 1) & (P["tp"] > 1) & (P["coll_algo"] == W.ALG_DBTREE)
+    valid = P["strategy"] <= W.ST_HOP
+    return np.flatnonzero(valid & ((phot & coll & trees) | both)).tolist()
