@@ -266,7 +266,8 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
 /* Copy result records [first, first+count) to out.  out_is_device == 0: host memory; the call first
  * synchronises the stream of the sweep's last simulate_batch (if it is not cuda_stream), then copies on
  * cuda_stream and synchronises it.  out_is_device != 0: a device pointer on the context's GPU; the copy
- * is enqueued on `cuda_stream` (stream-ordered, asynchronous: order it after simulate_batch yourself). */
+ * is enqueued on `cuda_stream`, after an event the sweep's last simulate_batch recorded on its own stream
+ * (so the copy is ordered after that batch on any stream; asynchronous, no host synchronisation). */
 triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t first, uint64_t count,
                                triosim_result *out, int out_is_device, void *cuda_stream);
 

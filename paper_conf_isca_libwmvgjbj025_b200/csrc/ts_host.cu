@@ -150,7 +150,10 @@ struct Trace {
 };
 
 struct Sweep {
-    ~Sweep() { cudaDeviceSynchronize(); }   // before the members' blocks go back to the cache
+    ~Sweep() {
+        cudaDeviceSynchronize();   // before the members' blocks go back to the cache
+        if (ev_done) cudaEventDestroy(ev_done);
+    }
     int trace_handle = -1;
     uint64_t n_pts = 0;
     std::vector<int32_t> status;            // host-side status per point (-1 = simulate)
@@ -191,6 +194,7 @@ struct Sweep {
     DevBuf<unsigned int> d_counter;
     DevBuf<unsigned long long> d_alg;
     cudaStream_t last_stream = nullptr;
+    cudaEvent_t ev_done = nullptr;           // recorded on last_stream after the last simulate_batch's K3 joins
     // R22 per-layer breakdown (triosim_set_breakdown): per-class layer compute, per-point [3][L]
     // communication accumulators, staging for host-bound copies
     bool bd = false;
@@ -1100,15 +1104,26 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         }
         const uint64_t cap = (uint64_t)ctx->n_sms * (uint64_t)((S.lmax[w] || S.pmax[w]) ? S.occ[w] : ctx->occ[w]);
         if (blocks > cap) blocks = cap;
-        CK(cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0));
-        if (mode == MODE_HYBRID) CK(launch_k3_hybrid(W, a, (int)blocks, ctx->side[w]));
-        else CK(launch_k3(W, mode, a, (int)blocks, ctx->side[w]));
-        ctx->n_k3++;
-        CK(cudaEventRecord(ctx->ev_join[w], ctx->side[w]));
-        launched[w] = 1;
+        cudaError_t e = cudaStreamWaitEvent(ctx->side[w], ctx->ev_fork, 0);
+        if (e == cudaSuccess)
+            e = mode == MODE_HYBRID ? launch_k3_hybrid(W, a, (int)blocks, ctx->side[w])
+                                    : launch_k3(W, mode, a, (int)blocks, ctx->side[w]);
+        if (e == cudaSuccess) {
+            ctx->n_k3++;
+            e = cudaEventRecord(ctx->ev_join[w], ctx->side[w]);
+            if (e == cudaSuccess) launched[w] = 1;
+        }
+        if (e != cudaSuccess) {
+            // join the groups already running back into the caller's stream before reporting
+            for (int v = 0; v < w; v++)
+                if (launched[v]) cudaStreamWaitEvent(st, ctx->ev_join[v], 0);
+            CK(e);
+        }
     }
     for (int w = 0; w < N_GROUPS; w++)
         if (launched[w]) CK(cudaStreamWaitEvent(st, ctx->ev_join[w], 0));
+    if (!S.ev_done) CK(cudaEventCreateWithFlags(&S.ev_done, cudaEventDisableTiming));
+    CK(cudaEventRecord(S.ev_done, st));
     if (slot >= 0) {
         CK(cudaEventRecord(ctx->t_end[slot], st));
         ctx->n_timed++;
@@ -1153,6 +1168,8 @@ triosim_status triosim_results(triosim_ctx *ctx, int32_t sweep_id, uint64_t firs
     if (count == 0) return TRIOSIM_OK;
     cudaStream_t st = (cudaStream_t)cuda_stream;
     if (out_is_device) {
+        // stream-ordered after the last simulate_batch even when that ran on another stream
+        if (S.ev_done && S.last_stream != st) CK(cudaStreamWaitEvent(st, S.ev_done, 0));
         CK(cudaMemcpyAsync(out, S.d_res.p + first, count * sizeof(triosim_result), cudaMemcpyDeviceToDevice, st));
     } else {
         // the last simulate_batch may have run on another (non-blocking) stream: finish it first
