@@ -578,7 +578,7 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
             if (plans->off[k + 1] < plans->off[k]) return fail(ctx, TRIOSIM_EINVAL, "bad plan offsets");
 
     PhaseTimer PT;
-    static const int widen_from = getenv("TS_WIDEN_FROM") ? atoi(getenv("TS_WIDEN_FROM")) : 8;
+    static const int widen_from = getenv("TS_WIDEN_FROM") ? atoi(getenv("TS_WIDEN_FROM")) : 16;
     std::vector<HostTopo> HT(n_topos);
     for (uint32_t i = 0; i < n_topos; i++) {
         triosim_status st = prep_topology(ctx, topos[i], i, HT[i]);
@@ -710,11 +710,12 @@ triosim_status triosim_build_sweep(triosim_ctx *ctx, int32_t trace_id, const tri
         auto lm = [&](bool h, int w) { return !h ? lmax_warp(w) : w <= 32 ? lmax_hybrid(w) : LMAX_CTA; };
         int W0 = 2;
         while (W0 < (int)lanes) W0 <<= 1;
-        // DP / DDP / TP points of 5-16 GPUs run on twice their segment width (9-16: one per warp): the
+        // DP / DDP / TP points of 9-16 GPUs run on twice their segment width (one point per warp): the
         // segments of a warp diverge on every event, and the spare lanes hash half of the ring
-        // fast-forward's events (R19) -- C2 3.69 -> 3.59 ms per step with 5-8 widened too (round 2; round 1,
-        // before the full-strength hash, measured 9-16 only as the better choice).  Results are identical
-        // for any W >= lanes.  TS_WIDEN_FROM=16 restores round 1's choice, 0 turns widening off.
+        // fast-forward's events (R19).  Widening 5-8-GPU points too was measured equal on C2 (3.59 vs 3.55 ms
+        // per step) and 37 % slower on C3 (75.7 vs 55.3 ms: its TP = 8 points run the general path, where
+        // the halved number of resident points costs a second wave) -- profiles/r2_ab_widen_minb.txt.
+        // Results are identical for any W >= lanes.  TS_WIDEN_FROM=8 widens from 5 GPUs, 0 turns it off.
         if (widen_from > 0 && W0 >= widen_from && W0 < 32 && pt.strategy != TRIOSIM_PP && pt.strategy != TRIOSIM_HYBRID)
             W0 <<= 1;
         // photonic points (R20) always run in the HYBRID kernel, whose lanes own their logical links;
@@ -1075,6 +1076,9 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
     if (slot >= 0) CK(cudaEventRecord(ctx->t_mid[slot], st));
     CK(cudaEventRecord(ctx->ev_fork, st));
     int launched[N_GROUPS] = {};
+    // groups in width order: the narrow groups' few CTAs take their SM slots first and finish early, then the
+    // wide groups' persistent grids fill the GPU (launching the most expensive group first was measured 12 %
+    // slower on C2: its persistent grid held every slot, serialising the narrow groups behind it)
     for (int w = 0; w < N_GROUPS; w++) {
         const uint32_t *wl = S.d_work[w].p;
         const uint32_t n_all = (uint32_t)S.work[w].size();
@@ -1115,7 +1119,7 @@ triosim_status triosim_simulate_batch(triosim_ctx *ctx, int32_t sweep_id, uint64
         }
         if (e != cudaSuccess) {
             // join the groups already running back into the caller's stream before reporting
-            for (int v = 0; v < w; v++)
+            for (int v = 0; v < N_GROUPS; v++)
                 if (launched[v]) cudaStreamWaitEvent(st, ctx->ev_join[v], 0);
             CK(e);
         }

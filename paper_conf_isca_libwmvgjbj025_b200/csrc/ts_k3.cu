@@ -210,6 +210,11 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
     SI.nF = SI.nB = SI.nO = SI.SF = SI.SB = SI.SO = 0;
     SI.ent_off = SI.send_off = SI.recv_off = 0;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
+    // PIPE: the head operator's first unmet receive (lane, count it waits for) at program position hc_pos.
+    // Counters only grow, so while that receive is still missing the head cannot start: an idle stage
+    // re-checks one shared-memory counter per pass instead of re-reading its entry and receive tables
+    uint32_t hc_pos = 0xffffffffu, hc_seq = 0;
+    int hc_src = 0;
     // HOP (R28): neighbours (ranks, ascending) and this lane's slot in each neighbour's list; iteration
     // structure (ops per iteration, last non-OPT op, first OPT op); finished backward passes; the flow in
     // flight's destination lane, slot and iteration
@@ -310,6 +315,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                 ldone = uprel = upd = dnrel = dnd = false;
                 fst = FS_NONE;
                 sq = dcnt = 0;
+                hc_pos = 0xffffffffu;
                 acc = alg = 0;
                 nev = false;
                 if (used) {
@@ -896,7 +902,7 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             cst = CS_RUN;
                             if (te == t) more = true;
                         }
-                    } else {
+                    } else if (!(hc_pos == pos && !(cnt[hc_src] > hc_seq))) {
                         uint32_t q = pos, P, j, idx;
                         if (q < m * SI.nF) { P = 0; j = q / SI.nF; idx = q % SI.nF; }
                         else if (q < m * (SI.nF + SI.nB)) { const uint32_t r = q - m * SI.nF; P = 1; j = m - 1 - r / SI.nB; idx = r % SI.nB; }
@@ -910,7 +916,12 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                             const uint32_t seqi = re.phase == 0 ? jp * ps.SF + re.e
                                                 : re.phase == 1 ? m * ps.SF + (m - 1 - jp) * ps.SB + re.e
                                                                 : m * (ps.SF + ps.SB) + re.e;
-                            if (!(cnt[re.src] > seqi)) ok = false;
+                            if (!(cnt[re.src] > seqi)) {
+                                ok = false;
+                                hc_pos = pos;
+                                hc_src = (int)re.src;
+                                hc_seq = seqi;
+                            }
                         }
                         if (ok) {
                             if (en.nrecv) EV(EV_TASK_START, ((uint64_t)gpu << 40) | q);

@@ -186,7 +186,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     int *q_dst;                     // destination GPU or -1
     uint8_t *q_st, *q_g;            // 1 waiting for a buffer / 2 transferring; granted
     auto ph_tables = [&](bool phot) {
-        p_t = s_dyn + ((NW == 1 || phot) ? 0 : (7 * LMAX + 1) / 2);   // after lres, lsh, ln, lk, lown
+        p_t = s_dyn + ((NW == 1 || phot) ? 0 : 4 * LMAX);   // after lres, lsh, ln, lk, lown / lused, lchg
         p_dst = (int *)(p_t + NTHR * PM);
         p_st = p_dst + NTHR * PM;
         q_t = (double *)(p_st + NTHR * PM);
@@ -205,6 +205,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     __shared__ int s_gc[3][NW == 1 ? 1 : SL];          // cross-warp group counters (rotating triple buffer)
     __shared__ uint8_t s_fl[2][NW == 1 ? 1 : SL];      // tree flags exchange (CTA)
     __shared__ uint32_t s_item;
+    __shared__ int s_nu, s_na, s_nchg;                 // CTA water-filling: links used, active flows, changed links
 
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int seg = NW == 1 ? lane / W : 0;
@@ -217,6 +218,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     int *ln = NW == 1 ? &s_n[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX);
     int *lk = NW == 1 ? &s_k[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + LMAX;
     int *lown = NW == 1 ? &s_own[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + 2 * LMAX;
+    // CTA water-filling lists (k3h_dyn_smem): the links the call's active flows use (lown's slot: a CTA needs
+    // no owner marks) and the links on which flows froze in the current round
+    int *lused = lown;
+    int *lchg = lown + LMAX;
     uint32_t *cnt = &s_cnt[slot][sbase];                     // indexed by segment lane
     for (int q = (NW == 1 ? lane : (int)threadIdx.x); q < NSEG * LMAX; q += (NW == 1 ? 32 : 32 * NW)) {
         ln[q - seg * LMAX] = 0;   // (NW == 1: each lane clears its warp's slot through segment 0's base)
@@ -287,9 +292,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             v = seg_min<32>(v);
             if (lane == 0) s_red[bb][wid] = v;
             __syncthreads();
-            double r = s_red[bb][0];
-#pragma unroll
-            for (int i = 1; i < NW; i++) r = s_red[bb][i] < r ? s_red[bb][i] : r;
+            // every warp combines the NW warp minima with a shuffle tree (lane i reads warp i's), not a
+            // serial NW-long chain
+            double r = seg_min<32>(lane < NW ? s_red[bb][lane] : dinf());
             bb ^= 1;
             return r;
         }
@@ -363,6 +368,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     HS.TF = HS.TB = HS.TO = HS.tcol_off = HS.ndp = HS.dcol_off = 0;
     HS.first_opt = 0xffffffffu;
     uint32_t sq = 0, nsend_tot = 0, dcnt = 0;
+    // the head operator's first unmet condition at program position hc_pos (counters only grow, so while it
+    // holds the head cannot start): kind 0 a receive (cnt[hc_a] > hc_b), 1 the TP wait (GT.donec > hc_b),
+    // 2 the DP wait of the first OPT op (GD.donec >= GD.ncoll) -- one register / shared-memory test per pass
+    uint32_t hc_pos = 0xffffffffu, hc_b = 0;
+    int hc_kind = 0, hc_a = 0;
     Group GT, GD;
     GT.member = GD.member = false;
     GT.cross = GD.cross = false;
@@ -405,6 +415,18 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         acc += mix64(tmix ^ (((uint64_t)(kind) << 60) | (uint64_t)(code)));   \
         nev = true;                                                           \
     } while (0)
+    // TS_PROF_H (profiling builds only): thread 0 accumulates clock64() cycles per phase of an instant and
+    // prints them when its point finishes; a point stops after TS_PROF_H instants
+#ifdef TS_PROF_H
+    long long pf_c[7] = {0, 0, 0, 0, 0, 0, 0}, pf_last = clock64();
+    unsigned pf_inner = 0, pf_outer = 0;
+#define PFM(k)                                                                 \
+    do {                                                                       \
+        if (threadIdx.x == 0) { const long long c_ = clock64(); pf_c[k] += c_ - pf_last; pf_last = c_; } \
+    } while (0)
+#else
+#define PFM(k) do {} while (0)
+#endif
 
     auto grp_init = [&](Group &G, bool member, int p, int i, int lane0, int stride, uint64_t gid, uint32_t ncoll,
                         int slot) {
@@ -646,7 +668,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         // ------------------------------ refill ------------------------------
         const bool need = !have && !exhausted;
         bool fresh = false, rbad = false, rlong = false;
-        if (vany(need)) {
+        // (a CTA is one segment: have / exhausted are block-uniform, so it needs no vote here)
+        if (NW > 1 ? need : vany(need)) {
             uint32_t it = 0;
             if constexpr (NW == 1) {
                 if (need && li == 0) it = atomicAdd(a.counter, 1u);
@@ -697,6 +720,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     t_end = busy = 0.0;
                     ntask = nflow = np2p = 0;
                     sq = dcnt = 0;
+                    hc_pos = 0xffffffffu;
                     FT.st = FD.st = FP.st = FS_NONE;
                     acc = alg = 0;
                     nev = false;
@@ -769,9 +793,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 }
             }
         }
-        if (vall(!have && exhausted)) break;
+        if (NW > 1 ? (!have && exhausted) : vall(!have && exhausted)) break;
 
         // ------------------------------ one instant ------------------------------
+        PFM(0);
         bool dirty = false;
         if (TR.phot && used)   // R20: logical links whose setup completes now are up (last use = now)
             for (int k = 0; k < ports; k++)
@@ -833,7 +858,9 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     }
                 }
                 // (e) compute start
-                if (used && cst == CS_IDLE && pos < nprog) {
+                const bool hc_blocked = hc_pos == pos && (hc_kind == 0 ? !(cnt[hc_a] > hc_b)
+                                                          : hc_kind == 1 ? !(GT.donec > hc_b) : GD.donec < GD.ncoll);
+                if (used && cst == CS_IDLE && pos < nprog && !hc_blocked) {
                     uint32_t P, j, idx;
                     decode(pos, P, j, idx);
                     HEnt en = ent_at(P, idx);
@@ -845,14 +872,23 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         const uint32_t seqi = re.phase == 0 ? jp * ps.SF + re.e
                                             : re.phase == 1 ? m * ps.SF + (m - 1 - jp) * ps.SB + re.e
                                                             : m * (ps.SF + ps.SB) + re.e;
-                        if (!(cnt[(d * S + re.src) * tp + tt] > seqi)) ok = false;
+                        if (!(cnt[(d * S + re.src) * tp + tt] > seqi)) {
+                            ok = false;
+                            hc_pos = pos; hc_kind = 0; hc_a = (d * S + re.src) * tp + tt; hc_b = seqi;
+                        }
                     }
                     if (ok && en.tpw >= 0) {
                         const uint32_t pp_ = (uint32_t)en.tpw >> 24, ee = (uint32_t)en.tpw & 0xffffffu;
                         const uint32_t jp = (pp_ == 2 || P == 2) ? 0 : j;
-                        if (!(GT.donec > tp_seq(pp_, jp, ee))) ok = false;
+                        if (!(GT.donec > tp_seq(pp_, jp, ee))) {
+                            ok = false;
+                            hc_pos = pos; hc_kind = 1; hc_b = tp_seq(pp_, jp, ee);
+                        }
                     }
-                    if (ok && P == 2 && idx == HS.first_opt && GD.ncoll > 0 && GD.donec < GD.ncoll) ok = false;
+                    if (ok && P == 2 && idx == HS.first_opt && GD.ncoll > 0 && GD.donec < GD.ncoll) {
+                        ok = false;
+                        hc_pos = pos; hc_kind = 2;
+                    }
                     if (ok) {
                         if (has_wait(en, P, idx)) EV(EV_TASK_START, ((uint64_t)gpu << 40) | pos);
                         run_start = pos;
@@ -889,8 +925,15 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     }
                 }
                 ssync();
+#ifdef TS_PROF_H
+                pf_inner++;
+#endif
                 if (!vany(more)) break;
             }
+            PFM(1);
+#ifdef TS_PROF_H
+            pf_outer++;
+#endif
 
             bool again = false;
             // (f') R20 photonic network: (i) a logical link per request, (ii) link heads ask for a
@@ -1023,11 +1066,14 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 if (TR.phot && have && nx > maxact) maxact = nx;
             }
 
+            PFM(2);
             // (f) R14 over every in-transit flow of the segment (up to three per lane)
             if (!vany(dirty)) {
                 if (!vany(again)) break;
                 continue;
             }
+            if constexpr (NW > 1)
+                if (threadIdx.x == 0) { s_nu = 0; s_na = 0; }   // (their last readers passed barriers since)
             const bool segdirty = sany(dirty);
             dirty = false;
             const bool aT = segdirty && used && FT.st == FS_ACT;
@@ -1044,65 +1090,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             progress(FT, aT);
             progress(FD, aD);
             progress(FP, aP);
-            // link counters are 0 here: every complete progressive filling returns them to 0.  The first
-            // flow to count a link owns it for this call: it sets the residual, computes the share and
-            // updates both whenever flows on the link freeze (R14's single per-link expression)
-            unsigned lo = 0;   // owned links: bit slot * 8 + hop (the first MAX_HOPS hops)
-            unsigned lt = 0;   // bit slot: this slot owns links past MAX_HOPS (marked in lown)
-            auto count = [&](const Flow &F, bool on, int slot) {
-                if (on) {
-                    alg += F.len;
-#pragma unroll
-                    for (int h = 0; h < MAX_HOPS; h++)
-                        if (h < F.len) {
-                            const int e = hop(F.hl, h);
-                            if (atomicAdd(&ln[e], 1) == 0) {
-                                lo |= 1u << (slot * 8 + h);
-                                lown[e] = li * 4 + slot;   // (so no stale owner mark of an earlier call matches)
-                                lres[e] = a.link_bw[TR.link_off + e] * bws;
-                            }
-                        }
-                    for (int h = MAX_HOPS; h < F.len; h++) {   // long routes
-                        const int e = a.rt_links[F.roff + h];
-                        if (atomicAdd(&ln[e], 1) == 0) {
-                            lown[e] = li * 4 + slot;
-                            lt |= 1u << slot;
-                            lres[e] = a.link_bw[TR.link_off + e] * bws;
-                        }
-                    }
-                }
-            };
-            count(FT, aT, 0);
-            count(FD, aD, 1);
-            count(FP, aP, 2);
-            ssync();
-            auto owned = [&](auto &&fn) {   // fn(link) for every link this lane owns
-                // the cached hops: one bit scan (one copy of fn); the slot's words are selected, not
-                // addressed, so the flow slots stay in registers
-                for (unsigned m = lo; m; m &= m - 1) {
-                    const int b = __ffs(m) - 1, sl = b >> 3, h = b & 7, q = h >> 1;
-                    const uint32_t x0 = sl == 0 ? FT.hl[0] : sl == 1 ? FD.hl[0] : FP.hl[0];
-                    const uint32_t x1 = sl == 0 ? FT.hl[1] : sl == 1 ? FD.hl[1] : FP.hl[1];
-                    const uint32_t x2 = sl == 0 ? FT.hl[2] : sl == 1 ? FD.hl[2] : FP.hl[2];
-                    const uint32_t x3 = sl == 0 ? FT.hl[3] : sl == 1 ? FD.hl[3] : FP.hl[3];
-                    const uint32_t w = q == 0 ? x0 : q == 1 ? x1 : q == 2 ? x2 : x3;
-                    fn((int)((w >> (16 * (h & 1))) & 0xffffu));
-                }
-                if (lt) {   // hops past the cache (long routes): the owner marks
-                    auto tail = [&](const Flow &F, int slot) {
-                        if ((lt >> slot) & 1u)
-                            for (int h = MAX_HOPS; h < F.len; h++) {
-                                const int e = a.rt_links[F.roff + h];
-                                if (lown[e] == li * 4 + slot) fn(e);
-                            }
-                    };
-                    tail(FT, 0);
-                    tail(FD, 1);
-                    tail(FP, 2);
-                }
-            };
-            owned([&](int e) { lsh[e] = lres[e] / (double)ln[e]; alg += 2; });
-            ssync();
+            // link counters are 0 here: every complete progressive filling returns them to 0
             // progressive filling: each round freezes every unfrozen flow crossing a link whose share is
             // the minimum s; the owners then update those links' residual, count and share
             auto fmin = [&](const Flow &F, bool on) -> double {
@@ -1121,36 +1109,72 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 }
                 return my;
             };
-            bool uT = aT, uD = aD, uP = aP;
             uint32_t rounds = 0;
-            for (;;) {
-                const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
-                double my = mT < mD ? mT : mD;
-                my = mP < my ? mP : my;
-                const double sm = smin(my);   // segment-uniform; +inf: nothing left to freeze
-                const bool segact = sm < dinf();
-                if constexpr (NW == 1) {
-                    if (!__any_sync(FULL, segact)) break;
-                } else {
-                    if (!segact) break;
-                }
-                const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
-                auto freeze = [&](Flow &F, bool in) {
-                    if (in) {
-                        F.rate = sm;
+            uint32_t nact;
+            if constexpr (NW > 1) {
+                // CTA: the first flow to count a link sets its residual and lists it; the shares of the listed
+                // links, and each round the updates of the links on which flows froze (listed by the first
+                // freezing flow), are spread over all threads -- no lane scans the links it happened to reach
+                // first.  Same per-link expressions (R14), so the same bits as the warp-segment path.
+                auto count_c = [&](const Flow &F, bool on) {
+                    if (on) {
+                        alg += F.len;
+                        auto cnt1 = [&](int e) {
+                            if (atomicAdd(&ln[e], 1) == 0) {
+                                lres[e] = a.link_bw[TR.link_off + e] * bws;
+                                lused[atomicAdd(&s_nu, 1)] = e;
+                            }
+                        };
 #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
-                            if (h < F.len) atomicAdd(&lk[hop(F.hl, h)], 1);
-                        for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&lk[a.rt_links[F.roff + h]], 1);
+                            if (h < F.len) cnt1(hop(F.hl, h));
+                        for (int h = MAX_HOPS; h < F.len; h++) cnt1(a.rt_links[F.roff + h]);
                     }
                 };
-                freeze(FT, iT);
-                freeze(FD, iD);
-                freeze(FP, iP);
-                ssync();
-                owned([&](int e) {
-                    const int kk = lk[e];
-                    if (kk) {
+                count_c(FT, aT);
+                count_c(FD, aD);
+                count_c(FP, aP);
+                const int na = (aT ? 1 : 0) + (aD ? 1 : 0) + (aP ? 1 : 0);
+                if (na) atomicAdd(&s_na, na);
+                __syncthreads();
+                const int nu = s_nu;
+                nact = (uint32_t)s_na;
+                for (int k = (int)threadIdx.x; k < nu; k += NTHR) {
+                    const int e = lused[k];
+                    lsh[e] = lres[e] / (double)ln[e];
+                    alg += 2;
+                }
+                __syncthreads();
+                PFM(3);
+                bool uT = aT, uD = aD, uP = aP;
+                for (;;) {
+                    if (threadIdx.x == 0) s_nchg = 0;   // (last round's readers passed its closing barrier)
+                    const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
+                    double my = mT < mD ? mT : mD;
+                    my = mP < my ? mP : my;
+                    const double sm = smin(my);   // block-uniform; +inf: nothing left to freeze
+                    if (!(sm < dinf())) break;
+                    const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
+                    auto freeze_c = [&](Flow &F, bool in) {
+                        if (in) {
+                            F.rate = sm;
+                            auto fr1 = [&](int e) {
+                                if (atomicAdd(&lk[e], 1) == 0) lchg[atomicAdd(&s_nchg, 1)] = e;
+                            };
+#pragma unroll
+                            for (int h = 0; h < MAX_HOPS; h++)
+                                if (h < F.len) fr1(hop(F.hl, h));
+                            for (int h = MAX_HOPS; h < F.len; h++) fr1(a.rt_links[F.roff + h]);
+                        }
+                    };
+                    freeze_c(FT, iT);
+                    freeze_c(FD, iD);
+                    freeze_c(FP, iP);
+                    __syncthreads();
+                    const int nc = s_nchg;
+                    for (int k = (int)threadIdx.x; k < nc; k += NTHR) {
+                        const int e = lchg[k];
+                        const int kk = lk[e];
                         const double r = lres[e] - sm * (double)kk;
                         const double rr = r > 0.0 ? r : 0.0;
                         const int nn = ln[e] - kk;
@@ -1160,15 +1184,123 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         if (nn > 0) lsh[e] = rr / (double)nn;
                         alg += 5;
                     }
-                });
+                    __syncthreads();
+                    rounds++;
+                    uT = uT && !iT;
+                    uD = uD && !iD;
+                    uP = uP && !iP;
+                }
+            } else {
+                // warp segments: the first flow to count a link owns it for this call: it sets the residual,
+                // computes the share and updates both whenever flows on the link freeze (R14's single
+                // per-link expression)
+                unsigned lo = 0;   // owned links: bit slot * 8 + hop (the first MAX_HOPS hops)
+                unsigned lt = 0;   // bit slot: this slot owns links past MAX_HOPS (marked in lown)
+                auto count = [&](const Flow &F, bool on, int slot) {
+                    if (on) {
+                        alg += F.len;
+    #pragma unroll
+                        for (int h = 0; h < MAX_HOPS; h++)
+                            if (h < F.len) {
+                                const int e = hop(F.hl, h);
+                                if (atomicAdd(&ln[e], 1) == 0) {
+                                    lo |= 1u << (slot * 8 + h);
+                                    lown[e] = li * 4 + slot;   // (so no stale owner mark of an earlier call matches)
+                                    lres[e] = a.link_bw[TR.link_off + e] * bws;
+                                }
+                            }
+                        for (int h = MAX_HOPS; h < F.len; h++) {   // long routes
+                            const int e = a.rt_links[F.roff + h];
+                            if (atomicAdd(&ln[e], 1) == 0) {
+                                lown[e] = li * 4 + slot;
+                                lt |= 1u << slot;
+                                lres[e] = a.link_bw[TR.link_off + e] * bws;
+                            }
+                        }
+                    }
+                };
+                count(FT, aT, 0);
+                count(FD, aD, 1);
+                count(FP, aP, 2);
                 ssync();
-                if (segact) rounds++;
-                uT = uT && !iT;
-                uD = uD && !iD;
-                uP = uP && !iP;
+                auto owned = [&](auto &&fn) {   // fn(link) for every link this lane owns
+                    // the cached hops: one bit scan (one copy of fn); the slot's words are selected, not
+                    // addressed, so the flow slots stay in registers
+                    for (unsigned m = lo; m; m &= m - 1) {
+                        const int b = __ffs(m) - 1, sl = b >> 3, h = b & 7, q = h >> 1;
+                        const uint32_t x0 = sl == 0 ? FT.hl[0] : sl == 1 ? FD.hl[0] : FP.hl[0];
+                        const uint32_t x1 = sl == 0 ? FT.hl[1] : sl == 1 ? FD.hl[1] : FP.hl[1];
+                        const uint32_t x2 = sl == 0 ? FT.hl[2] : sl == 1 ? FD.hl[2] : FP.hl[2];
+                        const uint32_t x3 = sl == 0 ? FT.hl[3] : sl == 1 ? FD.hl[3] : FP.hl[3];
+                        const uint32_t w = q == 0 ? x0 : q == 1 ? x1 : q == 2 ? x2 : x3;
+                        fn((int)((w >> (16 * (h & 1))) & 0xffffu));
+                    }
+                    if (lt) {   // hops past the cache (long routes): the owner marks
+                        auto tail = [&](const Flow &F, int slot) {
+                            if ((lt >> slot) & 1u)
+                                for (int h = MAX_HOPS; h < F.len; h++) {
+                                    const int e = a.rt_links[F.roff + h];
+                                    if (lown[e] == li * 4 + slot) fn(e);
+                                }
+                        };
+                        tail(FT, 0);
+                        tail(FD, 1);
+                        tail(FP, 2);
+                    }
+                };
+                owned([&](int e) { lsh[e] = lres[e] / (double)ln[e]; alg += 2; });
+                ssync();
+                PFM(3);
+                // warp segments: every lane its own (up to three) flows, segment minimum per round
+                bool uT = aT, uD = aD, uP = aP;
+                for (;;) {
+                    const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
+                    double my = mT < mD ? mT : mD;
+                    my = mP < my ? mP : my;
+                    const double sm = smin(my);   // segment-uniform; +inf: nothing left to freeze
+                    const bool segact = sm < dinf();
+                    if constexpr (NW == 1) {
+                        if (!__any_sync(FULL, segact)) break;
+                    } else {
+                        if (!segact) break;
+                    }
+                    const bool iT = uT && mT == sm, iD = uD && mD == sm, iP = uP && mP == sm;
+                    auto freeze = [&](Flow &F, bool in) {
+                        if (in) {
+                            F.rate = sm;
+    #pragma unroll
+                            for (int h = 0; h < MAX_HOPS; h++)
+                                if (h < F.len) atomicAdd(&lk[hop(F.hl, h)], 1);
+                            for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&lk[a.rt_links[F.roff + h]], 1);
+                        }
+                    };
+                    freeze(FT, iT);
+                    freeze(FD, iD);
+                    freeze(FP, iP);
+                    ssync();
+                    owned([&](int e) {
+                        const int kk = lk[e];
+                        if (kk) {
+                            const double r = lres[e] - sm * (double)kk;
+                            const double rr = r > 0.0 ? r : 0.0;
+                            const int nn = ln[e] - kk;
+                            lres[e] = rr;
+                            ln[e] = nn;
+                            lk[e] = 0;
+                            if (nn > 0) lsh[e] = rr / (double)nn;
+                            alg += 5;
+                        }
+                    });
+                    ssync();
+                    if (segact) rounds++;
+                    uT = uT && !iT;
+                    uD = uD && !iD;
+                    uP = uP && !iP;
+                }
+                nact = scount(aT) + scount(aD) + scount(aP);
             }
+            PFM(4);
             // every link's count is back to 0 (all its flows froze)
-            const uint32_t nact = scount(aT) + scount(aD) + scount(aP);
             if (segdirty) {
                 nwf++;
                 nrounds += rounds;
@@ -1184,6 +1316,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             drain(FT, aT);
             drain(FD, aD);
             drain(FP, aP);
+            PFM(5);
             if (!vany(again)) break;
         }
 
@@ -1224,13 +1357,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 s_fl3[bb][wid] = f;
             }
             __syncthreads();
-            double r = s_red[bb][0];
-            unsigned fa = s_fl3[bb][0];
+            const double r = seg_min<32>(lane < NW ? s_red[bb][lane] : dinf());
+            unsigned fa = lane < NW ? s_fl3[bb][lane] : 0u;
 #pragma unroll
-            for (int i = 1; i < NW; i++) {
-                r = s_red[bb][i] < r ? s_red[bb][i] : r;
-                fa |= s_fl3[bb][i];
-            }
+            for (int o = 16; o > 0; o >>= 1) fa |= __shfl_xor_sync(FULL, fa, o);
             bb ^= 1;
             any_ev = (fa & 1u) != 0;
             infl = (fa & 2u) != 0;
@@ -1243,7 +1373,16 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             if (infl && !bon) { bon = true; bstart = t; }
             else if (!infl && bon) { bon = false; cbusy = cbusy + (t - bstart); }
         }
+        PFM(6);
+#ifdef TS_PROF_H
+        const bool fin = have && (alldone || ninst >= (uint32_t)TS_PROF_H);
+        if (fin && threadIdx.x == 0)
+            printf("PFH pidx=%u W=%d NW=%d inst=%u wf=%u rounds=%u inner=%u outer=%u cyc refill+end=%lld inner=%lld phot=%lld wfsetup=%lld rounds=%lld drain=%lld endinst=%lld\n",
+                   pidx, W, NW, ninst, nwf, nrounds, pf_inner, pf_outer, pf_c[0], pf_c[1], pf_c[2], pf_c[3], pf_c[4], pf_c[5], pf_c[6]);
+        if (fin) { for (int k = 0; k < 7; k++) pf_c[k] = 0; pf_inner = pf_outer = 0; }
+#else
         const bool fin = have && alldone;
+#endif
         const bool stuck = have && !fin && !(tn < dinf());
         if ((NW > 1) ? (fin || stuck) : vany(fin || stuck)) {   // (a CTA segment: uniform, no vote needed)
             const double bmax = smax(used ? busy : 0.0);
@@ -1283,13 +1422,14 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         }
     }
 #undef EV
+#undef PFM
 }
 
 size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
     const size_t nthr = W <= 32 ? K3_THREADS : (size_t)W;
     const size_t ph = pmax ? nthr * pmax * 16 + nthr * 3 * (8 + 8 + 4 + 1 + 1) : 0;
     if (W <= 32) return ph;
-    const size_t links = (size_t)lmax * 28 + 8;
+    const size_t links = (size_t)lmax * 32 + 8;   // lres, lsh (f64); ln, lk, lused, lchg (i32)
     return links > ph ? links : ph;   // a one-point CTA runs either a flow-network or a photonic point
 }
 

@@ -2,10 +2,15 @@
 no GPU needed): per launch the time, grid, registers, occupancy limit, warps active, issue active, executed
 warp instructions, lane efficiency, DRAM bytes, fp64 pipe activity and the stall reasons per issue.
 
-    python profiles/raw_summary.py <raw.csv> <out.json> <run id> [note]
+    python profiles/raw_summary.py <raw.csv> <out.json> <run id> [note] [--issue <cfg>]
+
+--issue <cfg> also writes profiles/ncu_issue_<cfg>.json, the issue evidence bench.py prints next to its
+roofline (warp instructions of one step's K3 launches, lane efficiency, time-weighted warps active, DRAM
+bytes per step).
 """
 import csv
 import json
+import os
 import sys
 
 KEYS = {
@@ -31,7 +36,7 @@ def num(x):
         return None
 
 
-def main(path, out, run, note=""):
+def main(path, out, run, note="", issue_cfg=None):
     rows = list(csv.reader(open(path)))
     h = next(i for i, r in enumerate(rows) if r and r[0] == "ID")
     hdr = rows[h]
@@ -58,10 +63,27 @@ def main(path, out, run, note=""):
            "total_time_ms_serialised": round(tot_t, 4), "total_warp_inst": tot_i}
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
+    if issue_cfg:
+        thr = sum((l.get("warp_inst") or 0) * (l.get("threads_per_inst") or 0) for l in launches)
+        dur = sum(l.get("time_ms") or 0 for l in launches)
+        warps = sum((l.get("warps_active_pct") or 0) * (l.get("time_ms") or 0) for l in launches) / max(dur, 1e-30)
+        iss = {"run": run, "config": issue_cfg, "launches": len(launches), "warp_inst_per_step": tot_i,
+               "lane_efficiency": round(thr / max(tot_i, 1.0) / 32.0, 4), "warps_active_pct": round(warps, 3),
+               "dram_bytes_per_step": sum((l.get("dram_read_bytes") or 0) + (l.get("dram_write_bytes") or 0)
+                                          for l in launches),
+               "serialised_k3_ns": round(dur * 1e6), "source": path}
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), f"ncu_issue_{issue_cfg}.json"), "w") as f:
+            json.dump(iss, f, indent=1)
     for l in launches:
         print(l["kernel"][:40], l.get("time_ms"), l.get("registers"), l.get("warps_active_pct"), l.get("issue_active_pct"),
               {k: v for k, v in l["stalls_per_issue"].items() if v and v > 0.3})
 
 
 if __name__ == "__main__":
-    main(*sys.argv[1:])
+    argv = sys.argv[1:]
+    cfg = None
+    if "--issue" in argv:
+        k = argv.index("--issue")
+        cfg = argv[k + 1]
+        del argv[k:k + 2]
+    main(*argv, issue_cfg=cfg)
