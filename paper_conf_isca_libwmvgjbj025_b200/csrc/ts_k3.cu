@@ -1009,11 +1009,24 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
             // link-disjoint ring with different rates: progressive filling freezes, round after round, the
             // flows at the smallest remaining rate, so its rounds are the distinct rates of the active
             // flows -- counted at once (a lane leads its value if it is the lowest segment lane holding it)
-            if (__any_sync(FULL, fast && !uni && segany)) {
+            if (COLL && __any_sync(FULL, fast && !uni && segany)) {   // (ring fast path: COLL classes only)
                 const unsigned long long key = act ? (unsigned long long)__double_as_longlong(rate)
                                                    : ~(unsigned long long)lane;   // NaN patterns, never a rate
-                const unsigned mm = __match_any_sync(FULL, key) & smask;
-                const bool lead = act && (__ffs(mm) - 1) == lane;
+                bool lead;
+                if constexpr (W <= 16) {
+                    // W - 1 independent shuffles beat one 64-bit match.any here (its issue latency was 14 % of
+                    // the C3 K3 stall samples, profiles/r2_c3_k3_lines.txt)
+                    bool dup = false;
+#pragma unroll
+                    for (int d = 1; d < W; d++) {
+                        const unsigned long long o = __shfl_up_sync(FULL, key, d, W);
+                        dup = dup || (li >= d && o == key);
+                    }
+                    lead = act && !dup;
+                } else {
+                    const unsigned mm = __match_any_sync(FULL, key) & smask;
+                    lead = act && (__ffs(mm) - 1) == lane;
+                }
                 const uint32_t nd = __popc(__ballot_sync(FULL, lead) & smask);
                 if (fast && !uni) rounds = nd;
             }

@@ -292,9 +292,16 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             v = seg_min<32>(v);
             if (lane == 0) s_red[bb][wid] = v;
             __syncthreads();
-            // every warp combines the NW warp minima with a shuffle tree (lane i reads warp i's), not a
-            // serial NW-long chain
-            double r = seg_min<32>(lane < NW ? s_red[bb][lane] : dinf());
+            // every warp combines the NW warp minima: serially for a few warps, with a shuffle tree (lane i
+            // reads warp i's) for many -- not an NW-long chain
+            double r;
+            if constexpr (NW <= 4) {
+                r = s_red[bb][0];
+#pragma unroll
+                for (int i = 1; i < NW; i++) r = s_red[bb][i] < r ? s_red[bb][i] : r;
+            } else {
+                r = seg_min<32>(lane < NW ? s_red[bb][lane] : dinf());
+            }
             bb ^= 1;
             return r;
         }
