@@ -5,6 +5,11 @@ from the CUDA path.  Each file stores the sweep's point indices, the records and
 trace / topology / point bytes, so a test can prove it rebuilt the same inputs.
 
     python tests/golden/make_goldens.py [c1 c2 c3 c4 c5] [--procs N]
+    python tests/golden/make_goldens.py c5 --finalize-partial   (while a long run is still going)
+
+--finalize-partial writes <name>.npz from the points the (still running) oracle has finished so far, with a
+boolean `have` mask; the GPU test compares exactly those points and names the rest.  A finished run
+overwrites the file with every record (no mask).
 """
 from __future__ import annotations
 
@@ -113,13 +118,38 @@ def make(name, procs):
           f"({os.path.getsize(out)} B); statuses {np.bincount(rec['status'])}", flush=True)
 
 
+def finalize_partial(name):
+    """<name>.npz from <name>.partial.npz: the finished points' oracle records plus the `have` mask."""
+    sw = SWEEPS[name]()
+    n = len(sw.points)
+    z = np.load(os.path.join(HERE, f"{name}.partial.npz"))
+    cache = {pb.tobytes(): (rb, float(sc)) for pb, rb, sc in zip(z["points"], z["records"], z["secs"])}
+    rec = np.zeros(n, W.RESULT_DTYPE)
+    secs = np.zeros(n)
+    have = np.zeros(n, bool)
+    for i in range(n):
+        h = cache.get(sw.points[i].tobytes())
+        if h is not None:
+            rec[i] = h[0].view(W.RESULT_DTYPE)[0]
+            secs[i] = h[1]
+            have[i] = True
+    out = os.path.join(HERE, f"{name}.npz")
+    np.savez_compressed(out, records=rec.view(np.uint8), n=n, digest=sweep_digest(sw), oracle_s=secs, have=have)
+    print(f"{name}: {int(have.sum())} of {n} points finished by the oracle -> {out}; pending: "
+          f"{np.flatnonzero(~have).tolist()}", flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("names", nargs="*", default=["c1", "c2", "c3", "c4"])
     ap.add_argument("--procs", type=int, default=os.cpu_count() or 1)
+    ap.add_argument("--finalize-partial", action="store_true")
     a = ap.parse_args()
     for name in a.names:
-        make(name, a.procs)
+        if a.finalize_partial:
+            finalize_partial(name)
+        else:
+            make(name, a.procs)
 
 
 if __name__ == "__main__":

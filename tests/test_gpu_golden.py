@@ -40,15 +40,20 @@ def load(name):
     if not os.path.exists(path):
         pytest.fail(f"missing golden file {path}: run tests/golden/make_goldens.py {name}")
     z = np.load(path)
-    return z["records"].view(W.RESULT_DTYPE), str(z["digest"])
+    have = z["have"] if "have" in z.files else np.ones(int(z["n"]), bool)
+    return z["records"].view(W.RESULT_DTYPE), str(z["digest"]), have
 
 
 def _compare_full(ctx, name, select=None):
-    ref, digest = load(name)
+    ref, digest, have = load(name)
     sw = G.SWEEPS[name]()
     assert G.sweep_digest(sw) == digest, "the seeded generator no longer reproduces the golden sweep"
     assert len(ref) == len(sw.points)
-    idx = np.arange(len(sw.points)) if select is None else np.flatnonzero(select(sw.points))
+    sel = np.ones(len(sw.points), bool) if select is None else np.asarray(select(sw.points), bool)
+    pending = np.flatnonzero(sel & ~have).tolist()
+    if pending:   # points the oracle had not finished when the file was written (make_goldens --finalize-partial)
+        print(f"{name}: no oracle record yet for points {pending}; compared the other {int((sel & have).sum())}")
+    idx = np.flatnonzero(sel & have)
     sub = W.Sweep(sw.name, sw.trace, sw.topos, sw.points[idx], sw.plans)
     got = ctx.run_sweep(sub)
     too_large = np.flatnonzero(got["status"] == W.PT_TOO_LARGE).tolist()
