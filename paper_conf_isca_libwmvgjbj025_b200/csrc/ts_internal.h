@@ -225,7 +225,7 @@ int k3_max_blocks_per_sm(int W, int mode);
 // links per segment the K3 kernels keep in shared memory
 __host__ __device__ constexpr int lmax_warp(int W) { return 4 * W < 8 ? 8 : 4 * W; }
 __host__ __device__ constexpr int lmax_hybrid(int W) { return 8 * W < 16 ? 16 : 8 * W; }
-constexpr int LMAX_CTA = 6144;          // links of a one-point-per-CTA hybrid segment (dynamic smem, 32 B/link)
+constexpr int LMAX_CTA = 6144;          // links of a one-point-per-CTA hybrid segment (dynamic smem, 28 B/link)
 constexpr int N_WIDTHS = 10;            // W = 2, 4, 8, 16, 32 (warp segments), 64 ... 1024 (hybrid CTAs)
 constexpr int N_MODES = 5;
 constexpr int N_GROUPS = N_MODES * N_WIDTHS;  // (width, mode) launch groups

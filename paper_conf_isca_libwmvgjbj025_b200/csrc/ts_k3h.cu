@@ -54,7 +54,7 @@ __device__ __forceinline__ unsigned long long seg_sum_u64(unsigned long long v) 
 }
 
 struct Topo {
-    uint32_t n_gpus, link_off, rt_off, ro_off;
+    uint32_t n_gpus, link_off, rt_off, ro_off, n_links;
     bool phot;
 };
 
@@ -186,7 +186,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     int *q_dst;                     // destination GPU or -1
     uint8_t *q_st, *q_g;            // 1 waiting for a buffer / 2 transferring; granted
     auto ph_tables = [&](bool phot) {
-        p_t = s_dyn + ((NW == 1 || phot) ? 0 : 4 * LMAX);   // after lres, lsh, ln, lk, lown / lused, lchg
+        p_t = s_dyn + ((NW == 1 || phot) ? 0 : (7 * LMAX + 1) / 2);   // after lres, lsh, ln, lk, lown
         p_dst = (int *)(p_t + NTHR * PM);
         p_st = p_dst + NTHR * PM;
         q_t = (double *)(p_st + NTHR * PM);
@@ -201,11 +201,15 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     __shared__ double s_red[2][NW];
     __shared__ unsigned s_fl3[2][NW];                  // CTA: per-warp end-of-instant votes
     __shared__ unsigned long long s_red64[2][NW];
-    __shared__ int s_xch[2][NW == 1 ? 1 : SL];
-    __shared__ int s_gc[3][NW == 1 ? 1 : SL];          // cross-warp group counters (rotating triple buffer)
+    // CTA: each lane's group progress D (TP, DP), published with an event-loop pass's first barrier
+    __shared__ int s_dx[2][NW == 1 ? 1 : SL];
+    // CTA: one round of cross-warp group votes per pass and group -- members done, and ready under either
+    // outcome (21-bit fields) -- in a rotating triple buffer indexed by group slot (a group that spans warps
+    // has >= 2 members, so its slot is < SL / 2)
+    __shared__ unsigned long long s_gc3[3][NW == 1 ? 1 : SL / 2];
     __shared__ uint8_t s_fl[2][NW == 1 ? 1 : SL];      // tree flags exchange (CTA)
     __shared__ uint32_t s_item;
-    __shared__ int s_nu, s_na, s_nchg;                 // CTA water-filling: links used, active flows, changed links
+    __shared__ int s_na;                               // CTA water-filling: active flows of the call
 
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int seg = NW == 1 ? lane / W : 0;
@@ -218,17 +222,13 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     int *ln = NW == 1 ? &s_n[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX);
     int *lk = NW == 1 ? &s_k[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + LMAX;
     int *lown = NW == 1 ? &s_own[slot][seg * LMAX] : (int *)(s_dyn + 2 * LMAX) + 2 * LMAX;
-    // CTA water-filling lists (k3h_dyn_smem): the links the call's active flows use (lown's slot: a CTA needs
-    // no owner marks) and the links on which flows froze in the current round
-    int *lused = lown;
-    int *lchg = lown + LMAX;
     uint32_t *cnt = &s_cnt[slot][sbase];                     // indexed by segment lane
     for (int q = (NW == 1 ? lane : (int)threadIdx.x); q < NSEG * LMAX; q += (NW == 1 ? 32 : 32 * NW)) {
         ln[q - seg * LMAX] = 0;   // (NW == 1: each lane clears its warp's slot through segment 0's base)
         lk[q - seg * LMAX] = 0;
     }
     if constexpr (NW > 1) {
-        s_gc[0][threadIdx.x] = s_gc[1][threadIdx.x] = s_gc[2][threadIdx.x] = 0;
+        if (threadIdx.x < SL / 2) s_gc3[0][threadIdx.x] = s_gc3[1][threadIdx.x] = s_gc3[2][threadIdx.x] = 0ull;
     }
     if (NW == 1 && PM > 0) {   // (a CTA overlays its tables on the link arrays: set up per photonic point)
         for (int k = 0; k < PM; k++) p_st[k * NTHR + threadIdx.x] = 0;
@@ -236,7 +236,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     }
     int bb = 0;   // double-buffer toggle of the block-level exchanges (NW > 1)
     int fb = 0;   // double-buffer toggle of the tree-flag exchange (NW > 1)
-    int gcb = 0;  // rotating buffer of the cross-warp group counters (NW > 1)
+    int gcb3 = 0;  // rotating buffer of the cross-warp group votes (NW > 1)
 
     // ---- segment primitives: a segment is W lanes of a warp, or the whole CTA ----
     auto ssync = [&]() {
@@ -271,19 +271,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         fu.sel = 1;
         fd.sel = 2;
     };
-    // every member of G satisfies pred (called by all lanes; non-members pass anything)
+    // every member of G satisfies pred (called by all lanes; non-members pass anything) -- groups inside a
+    // warp; a CTA's cross-warp groups vote in grp_pass
     auto gall = [&](const Group &G, bool pred) -> bool {
-        if (NW == 1 || !G.cross) {
-            const unsigned b = __ballot_sync(FULL, !G.member || pred);
-            return (b & G.wmask) == G.wmask;
-        } else {
-            const int cb = gcb;
-            gcb = gcb == 2 ? 0 : gcb + 1;
-            s_gc[gcb][threadIdx.x] = 0;    // next call's buffer: its last readers passed a barrier since
-            if (G.member && pred) atomicAdd(&s_gc[cb][G.slot], 1);
-            __syncthreads();
-            return !G.member || s_gc[cb][G.slot] == G.p;
-        }
+        const unsigned b = __ballot_sync(FULL, !G.member || pred);
+        return (b & G.wmask) == G.wmask;
     };
     auto smin = [&](double v) -> double {
         if constexpr (NW == 1) {
@@ -334,16 +326,8 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             return r;
         }
     };
-    auto xch = [&](int v, int src) -> int {    // value of segment lane src
-        if constexpr (NW == 1) {
-            return __shfl_sync(FULL, v, sbase + src);
-        } else {
-            s_xch[bb][threadIdx.x] = v;
-            __syncthreads();
-            const int r = s_xch[bb][src];
-            bb ^= 1;
-            return r;
-        }
+    auto xch = [&](int v, int src) -> int {    // value of segment lane src (warp segments)
+        return __shfl_sync(FULL, v, sbase + src);
     };
     ssync();
 
@@ -357,7 +341,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     uint32_t m = 1;
     bool tree_algo = false, dbt_algo = false;   // binary-tree AllReduce (R10) / double binary tree (R27)
     const ClassDesc *C = nullptr;
-    Topo TR = {0, 0, 0, 0, false};
+    Topo TR = {0, 0, 0, 0, 0, false};
     uint32_t ninst = 0, nwf = 0, nrounds = 0, maxact = 0;
     bool bon = false;
     double bstart = 0.0, cbusy = 0.0;
@@ -472,7 +456,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     auto grp_pass = [&](Group &G, Flow &F, Flow &F2, bool is_tp, bool &more) {
         // the predecessor's progress: a shuffle when every group of this kind lies inside one warp (TP groups;
         // segment-uniform), a shared-memory exchange across warps otherwise
-        const int Dp = (NW > 1 && !G.cross) ? __shfl_sync(FULL, G.D, G.pred & 31) : xch(G.D, G.pred);
+        // (a cross-warp group reads it from s_dx, written before the pass's first barrier: G.D does not change
+        // between that barrier and here)
+        const int Dp = NW == 1 ? xch(G.D, G.pred)
+                     : !G.cross ? __shfl_sync(FULL, G.D, G.pred & 31) : s_dx[is_tp ? 0 : 1][G.pred];
         LF upb, dnb, zero;
         upb.bits = dnb.bits = zero.bits = 0;
         upb.p = dnb.p = zero.p = nullptr;
@@ -508,12 +495,36 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     if (bd_rep) bd_add(is_tp ? 0u : 1u, G.bd_l, t - G.bd_t0);
             }
         }
-        const bool allfin = gall(G, G.ldone);
-        if (G.member && G.running && allfin) {
-            G.running = false;
-            G.cur++;
+        bool allfin, allrdy;
+        if (NW > 1 && G.cross) {
+            // one barrier for both votes: a group's members start and finish collectives together (running
+            // is group-uniform), so each member also reports readiness for the next collective
+            const int cb = gcb3;
+            gcb3 = gcb3 == 2 ? 0 : gcb3 + 1;
+            if (threadIdx.x < SL / 2) s_gc3[gcb3][threadIdx.x] = 0ull;   // next call's buffer (its last readers
+                                                                          // passed a barrier since)
+            if (G.member) {
+                const unsigned long long v = (G.ldone ? 1ull : 0ull) | (G.trig > G.cur ? (1ull << 21) : 0ull) |
+                                             (G.trig > G.cur + 1 ? (1ull << 42) : 0ull);
+                if (v) atomicAdd(&s_gc3[cb][G.slot], v);
+            }
+            __syncthreads();
+            const unsigned long long c = s_gc3[cb][G.slot], M = (1ull << 21) - 1ull, P = (unsigned long long)G.p;
+            allfin = !G.member || (c & M) == P;
+            const bool adv = G.member && G.running && allfin;
+            if (adv) {
+                G.running = false;
+                G.cur++;
+            }
+            allrdy = !G.member || ((c >> (adv ? 42 : 21)) & M) == P;
+        } else {
+            allfin = gall(G, G.ldone);
+            if (G.member && G.running && allfin) {
+                G.running = false;
+                G.cur++;
+            }
+            allrdy = gall(G, G.trig > G.cur);
         }
-        const bool allrdy = gall(G, G.trig > G.cur);
         bool started = false;
         if (G.member && !G.running && G.cur < G.ncoll && allrdy) {
             CollEnt ce;
@@ -702,6 +713,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     {
                         const TopoDev td = a.topo[pd.topo];
                         TR.n_gpus = td.n_gpus; TR.link_off = td.link_off; TR.rt_off = td.rt_off; TR.ro_off = td.ro_off;
+                        TR.n_links = td.n_links;
                         TR.phot = td.net == TRIOSIM_NET_PHOTONIC;
                         ports = (int)td.ports;
                         bufs = (int)td.buf_slots;
@@ -834,6 +846,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     }
                 }
                 cnt[li] = dcnt;
+                if constexpr (NW > 1) {
+                    s_dx[0][threadIdx.x] = GT.D;
+                    s_dx[1][threadIdx.x] = GD.D;
+                }
                 ssync();
                 // (d) both groups, then this rank's next P2P send
                 grp_pass(GT, FT, FD, true, more);
@@ -931,7 +947,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         if (te == t) more = true;
                     }
                 }
-                ssync();
+                if constexpr (NW == 1) ssync();   // (a CTA's vote below is a barrier itself)
 #ifdef TS_PROF_H
                 pf_inner++;
 #endif
@@ -1080,7 +1096,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 continue;
             }
             if constexpr (NW > 1)
-                if (threadIdx.x == 0) { s_nu = 0; s_na = 0; }   // (their last readers passed barriers since)
+                if (threadIdx.x == 0) s_na = 0;   // (its last readers passed barriers since)
             const bool segdirty = sany(dirty);
             dirty = false;
             const bool aT = segdirty && used && FT.st == FS_ACT;
@@ -1119,23 +1135,17 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             uint32_t rounds = 0;
             uint32_t nact;
             if constexpr (NW > 1) {
-                // CTA: the first flow to count a link sets its residual and lists it; the shares of the listed
-                // links, and each round the updates of the links on which flows froze (listed by the first
-                // freezing flow), are spread over all threads -- no lane scans the links it happened to reach
-                // first.  Same per-link expressions (R14), so the same bits as the warp-segment path.
+                // CTA: flows count their links with fire-and-forget shared-memory adds (no returned value on
+                // the critical path); then the topology's links are spread over all threads, which set
+                // residual and share of every counted link, and after each round's freezes update every link
+                // with frozen flows.  Same per-link expressions (R14), so the same bits as the warp path.
                 auto count_c = [&](const Flow &F, bool on) {
                     if (on) {
                         alg += F.len;
-                        auto cnt1 = [&](int e) {
-                            if (atomicAdd(&ln[e], 1) == 0) {
-                                lres[e] = a.link_bw[TR.link_off + e] * bws;
-                                lused[atomicAdd(&s_nu, 1)] = e;
-                            }
-                        };
 #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
-                            if (h < F.len) cnt1(hop(F.hl, h));
-                        for (int h = MAX_HOPS; h < F.len; h++) cnt1(a.rt_links[F.roff + h]);
+                            if (h < F.len) atomicAdd(&ln[hop(F.hl, h)], 1);
+                        for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&ln[a.rt_links[F.roff + h]], 1);
                     }
                 };
                 count_c(FT, aT);
@@ -1144,18 +1154,21 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 const int na = (aT ? 1 : 0) + (aD ? 1 : 0) + (aP ? 1 : 0);
                 if (na) atomicAdd(&s_na, na);
                 __syncthreads();
-                const int nu = s_nu;
                 nact = (uint32_t)s_na;
-                for (int k = (int)threadIdx.x; k < nu; k += NTHR) {
-                    const int e = lused[k];
-                    lsh[e] = lres[e] / (double)ln[e];
-                    alg += 2;
+                const int nl = (int)TR.n_links;
+                for (int e = (int)threadIdx.x; e < nl; e += NTHR) {
+                    const int c = ln[e];
+                    if (c > 0) {
+                        const double r0 = a.link_bw[TR.link_off + e] * bws;
+                        lres[e] = r0;
+                        lsh[e] = r0 / (double)c;
+                        alg += 2;
+                    }
                 }
                 __syncthreads();
                 PFM(3);
                 bool uT = aT, uD = aD, uP = aP;
                 for (;;) {
-                    if (threadIdx.x == 0) s_nchg = 0;   // (last round's readers passed its closing barrier)
                     const double mT = fmin(FT, uT), mD = fmin(FD, uD), mP = fmin(FP, uP);
                     double my = mT < mD ? mT : mD;
                     my = mP < my ? mP : my;
@@ -1165,31 +1178,28 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     auto freeze_c = [&](Flow &F, bool in) {
                         if (in) {
                             F.rate = sm;
-                            auto fr1 = [&](int e) {
-                                if (atomicAdd(&lk[e], 1) == 0) lchg[atomicAdd(&s_nchg, 1)] = e;
-                            };
 #pragma unroll
                             for (int h = 0; h < MAX_HOPS; h++)
-                                if (h < F.len) fr1(hop(F.hl, h));
-                            for (int h = MAX_HOPS; h < F.len; h++) fr1(a.rt_links[F.roff + h]);
+                                if (h < F.len) atomicAdd(&lk[hop(F.hl, h)], 1);
+                            for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&lk[a.rt_links[F.roff + h]], 1);
                         }
                     };
                     freeze_c(FT, iT);
                     freeze_c(FD, iD);
                     freeze_c(FP, iP);
                     __syncthreads();
-                    const int nc = s_nchg;
-                    for (int k = (int)threadIdx.x; k < nc; k += NTHR) {
-                        const int e = lchg[k];
+                    for (int e = (int)threadIdx.x; e < nl; e += NTHR) {
                         const int kk = lk[e];
-                        const double r = lres[e] - sm * (double)kk;
-                        const double rr = r > 0.0 ? r : 0.0;
-                        const int nn = ln[e] - kk;
-                        lres[e] = rr;
-                        ln[e] = nn;
-                        lk[e] = 0;
-                        if (nn > 0) lsh[e] = rr / (double)nn;
-                        alg += 5;
+                        if (kk) {
+                            const double r = lres[e] - sm * (double)kk;
+                            const double rr = r > 0.0 ? r : 0.0;
+                            const int nn = ln[e] - kk;
+                            lres[e] = rr;
+                            ln[e] = nn;
+                            lk[e] = 0;
+                            if (nn > 0) lsh[e] = rr / (double)nn;
+                            alg += 5;
+                        }
                     }
                     __syncthreads();
                     rounds++;
@@ -1436,7 +1446,7 @@ size_t k3h_dyn_smem(int W, uint32_t lmax, uint32_t pmax) {
     const size_t nthr = W <= 32 ? K3_THREADS : (size_t)W;
     const size_t ph = pmax ? nthr * pmax * 16 + nthr * 3 * (8 + 8 + 4 + 1 + 1) : 0;
     if (W <= 32) return ph;
-    const size_t links = (size_t)lmax * 32 + 8;   // lres, lsh (f64); ln, lk, lused, lchg (i32)
+    const size_t links = (size_t)lmax * 28 + 8;   // lres, lsh (f64); ln, lk, lown (i32)
     return links > ph ? links : ph;   // a one-point CTA runs either a flow-network or a photonic point
 }
 
