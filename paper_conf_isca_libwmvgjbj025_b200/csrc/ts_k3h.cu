@@ -1096,7 +1096,13 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 continue;
             }
             if constexpr (NW > 1)
+            {
                 if (threadIdx.x == 0) s_na = 0;   // (its last readers passed barriers since)
+                // the call's link masks (s_dx's words: the event loop's progress exchange is over): bit j of
+                // thread i's word = link j * NTHR + i is counted / has flows frozen in this round
+                s_dx[0][threadIdx.x] = 0;
+                s_dx[1][threadIdx.x] = 0;
+            }
             const bool segdirty = sany(dirty);
             dirty = false;
             const bool aT = segdirty && used && FT.st == FS_ACT;
@@ -1139,13 +1145,20 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 // the critical path); then the topology's links are spread over all threads, which set
                 // residual and share of every counted link, and after each round's freezes update every link
                 // with frozen flows.  Same per-link expressions (R14), so the same bits as the warp path.
+                const int nl = (int)TR.n_links;
+                const bool lmask = nl <= 32 * NTHR;   // block-uniform: the links fit the per-thread masks
+                unsigned *um = reinterpret_cast<unsigned *>(s_dx[0]), *dm = reinterpret_cast<unsigned *>(s_dx[1]);
+                auto mark = [&](unsigned *mk, int e) {
+                    if (lmask) atomicOr(&mk[e & (NTHR - 1)], 1u << (e / NTHR));
+                };
                 auto count_c = [&](const Flow &F, bool on) {
                     if (on) {
                         alg += F.len;
+                        auto c1 = [&](int e) { atomicAdd(&ln[e], 1); mark(um, e); };
 #pragma unroll
                         for (int h = 0; h < MAX_HOPS; h++)
-                            if (h < F.len) atomicAdd(&ln[hop(F.hl, h)], 1);
-                        for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&ln[a.rt_links[F.roff + h]], 1);
+                            if (h < F.len) c1(hop(F.hl, h));
+                        for (int h = MAX_HOPS; h < F.len; h++) c1(a.rt_links[F.roff + h]);
                     }
                 };
                 count_c(FT, aT);
@@ -1155,8 +1168,7 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                 if (na) atomicAdd(&s_na, na);
                 __syncthreads();
                 nact = (uint32_t)s_na;
-                const int nl = (int)TR.n_links;
-                for (int e = (int)threadIdx.x; e < nl; e += NTHR) {
+                auto init1 = [&](int e) {
                     const int c = ln[e];
                     if (c > 0) {
                         const double r0 = a.link_bw[TR.link_off + e] * bws;
@@ -1164,6 +1176,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                         lsh[e] = r0 / (double)c;
                         alg += 2;
                     }
+                };
+                if (lmask) {
+                    for (unsigned mm = um[threadIdx.x]; mm; mm &= mm - 1) init1((__ffs(mm) - 1) * NTHR + (int)threadIdx.x);
+                } else {
+                    for (int e = (int)threadIdx.x; e < nl; e += NTHR) init1(e);
                 }
                 __syncthreads();
                 PFM(3);
@@ -1178,17 +1195,18 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                     auto freeze_c = [&](Flow &F, bool in) {
                         if (in) {
                             F.rate = sm;
+                            auto f1 = [&](int e) { atomicAdd(&lk[e], 1); mark(dm, e); };
 #pragma unroll
                             for (int h = 0; h < MAX_HOPS; h++)
-                                if (h < F.len) atomicAdd(&lk[hop(F.hl, h)], 1);
-                            for (int h = MAX_HOPS; h < F.len; h++) atomicAdd(&lk[a.rt_links[F.roff + h]], 1);
+                                if (h < F.len) f1(hop(F.hl, h));
+                            for (int h = MAX_HOPS; h < F.len; h++) f1(a.rt_links[F.roff + h]);
                         }
                     };
                     freeze_c(FT, iT);
                     freeze_c(FD, iD);
                     freeze_c(FP, iP);
                     __syncthreads();
-                    for (int e = (int)threadIdx.x; e < nl; e += NTHR) {
+                    auto upd1 = [&](int e) {
                         const int kk = lk[e];
                         if (kk) {
                             const double r = lres[e] - sm * (double)kk;
@@ -1200,6 +1218,13 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
                             if (nn > 0) lsh[e] = rr / (double)nn;
                             alg += 5;
                         }
+                    };
+                    if (lmask) {
+                        const unsigned mm0 = dm[threadIdx.x];
+                        dm[threadIdx.x] = 0;   // (the next round's marks follow this round's closing barrier)
+                        for (unsigned mm = mm0; mm; mm &= mm - 1) upd1((__ffs(mm) - 1) * NTHR + (int)threadIdx.x);
+                    } else {
+                        for (int e = (int)threadIdx.x; e < nl; e += NTHR) upd1(e);
                     }
                     __syncthreads();
                     rounds++;
