@@ -118,11 +118,12 @@ def make(name, procs):
           f"({os.path.getsize(out)} B); statuses {np.bincount(rec['status'])}", flush=True)
 
 
-def finalize_partial(name):
-    """<name>.npz from <name>.partial.npz: the finished points' oracle records plus the `have` mask."""
+def finalize_partial(name, where=HERE):
+    """<name>.npz from <name>.partial.npz (both in `where`): the finished points' oracle records plus the
+    `have` mask."""
     sw = SWEEPS[name]()
     n = len(sw.points)
-    z = np.load(os.path.join(HERE, f"{name}.partial.npz"))
+    z = np.load(os.path.join(where, f"{name}.partial.npz"))
     cache = {pb.tobytes(): (rb, float(sc)) for pb, rb, sc in zip(z["points"], z["records"], z["secs"])}
     rec = np.zeros(n, W.RESULT_DTYPE)
     secs = np.zeros(n)
@@ -133,8 +134,9 @@ def finalize_partial(name):
             rec[i] = h[0].view(W.RESULT_DTYPE)[0]
             secs[i] = h[1]
             have[i] = True
-    out = os.path.join(HERE, f"{name}.npz")
+    out = os.path.join(where, f"{name}.npz")
     np.savez_compressed(out, records=rec.view(np.uint8), n=n, digest=sweep_digest(sw), oracle_s=secs, have=have)
+    return out
     print(f"{name}: {int(have.sum())} of {n} points finished by the oracle -> {out}; pending: "
           f"{np.flatnonzero(~have).tolist()}", flush=True)
 
