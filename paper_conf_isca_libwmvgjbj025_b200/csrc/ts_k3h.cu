@@ -203,10 +203,11 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
     __shared__ unsigned long long s_red64[2][NW];
     // CTA: each lane's group progress D (TP, DP), published with an event-loop pass's first barrier
     __shared__ int s_dx[2][NW == 1 ? 1 : SL];
-    // CTA: one round of cross-warp group votes per pass and group -- members done, and ready under either
-    // outcome (21-bit fields) -- in a rotating triple buffer indexed by group slot (a group that spans warps
-    // has >= 2 members, so its slot is < SL / 2)
-    __shared__ unsigned long long s_gc3[3][NW == 1 ? 1 : SL / 2];
+    // CTA: one round of cross-warp group votes per pass and group -- members done | ready now (16-bit fields),
+    // and ready after this collective -- in a rotating triple buffer indexed by group slot (a group that spans
+    // warps has >= 2 members, so its slot is < SL / 2).  32-bit adds: a 64-bit shared add is a CAS loop, which
+    // an 84-member group turned into a 35 % slower wafer sweep
+    __shared__ unsigned s_gca[3][NW == 1 ? 1 : SL / 2], s_gcb[3][NW == 1 ? 1 : SL / 2];
     __shared__ uint8_t s_fl[2][NW == 1 ? 1 : SL];      // tree flags exchange (CTA)
     __shared__ uint32_t s_item;
     __shared__ int s_na;                               // CTA water-filling: active flows of the call
@@ -228,7 +229,10 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
         lk[q - seg * LMAX] = 0;
     }
     if constexpr (NW > 1) {
-        if (threadIdx.x < SL / 2) s_gc3[0][threadIdx.x] = s_gc3[1][threadIdx.x] = s_gc3[2][threadIdx.x] = 0ull;
+        if (threadIdx.x < SL / 2) {
+            s_gca[0][threadIdx.x] = s_gca[1][threadIdx.x] = s_gca[2][threadIdx.x] = 0u;
+            s_gcb[0][threadIdx.x] = s_gcb[1][threadIdx.x] = s_gcb[2][threadIdx.x] = 0u;
+        }
     }
     if (NW == 1 && PM > 0) {   // (a CTA overlays its tables on the link arrays: set up per photonic point)
         for (int k = 0; k < PM; k++) p_st[k * NTHR + threadIdx.x] = 0;
@@ -501,22 +505,24 @@ __global__ void __launch_bounds__(NW == 1 ? K3_THREADS : 32 * NW, 1) k3_hybrid(c
             // is group-uniform), so each member also reports readiness for the next collective
             const int cb = gcb3;
             gcb3 = gcb3 == 2 ? 0 : gcb3 + 1;
-            if (threadIdx.x < SL / 2) s_gc3[gcb3][threadIdx.x] = 0ull;   // next call's buffer (its last readers
-                                                                          // passed a barrier since)
+            if (threadIdx.x < SL / 2) {   // next call's buffer (its last readers passed a barrier since)
+                s_gca[gcb3][threadIdx.x] = 0u;
+                s_gcb[gcb3][threadIdx.x] = 0u;
+            }
             if (G.member) {
-                const unsigned long long v = (G.ldone ? 1ull : 0ull) | (G.trig > G.cur ? (1ull << 21) : 0ull) |
-                                             (G.trig > G.cur + 1 ? (1ull << 42) : 0ull);
-                if (v) atomicAdd(&s_gc3[cb][G.slot], v);
+                const unsigned va = (G.ldone ? 1u : 0u) | (G.trig > G.cur ? (1u << 16) : 0u);
+                if (va) atomicAdd(&s_gca[cb][G.slot], va);
+                if (G.trig > G.cur + 1) atomicAdd(&s_gcb[cb][G.slot], 1u);
             }
             __syncthreads();
-            const unsigned long long c = s_gc3[cb][G.slot], M = (1ull << 21) - 1ull, P = (unsigned long long)G.p;
-            allfin = !G.member || (c & M) == P;
+            const unsigned ca = s_gca[cb][G.slot], cbv = s_gcb[cb][G.slot], P = (unsigned)G.p;
+            allfin = !G.member || (ca & 0xffffu) == P;
             const bool adv = G.member && G.running && allfin;
             if (adv) {
                 G.running = false;
                 G.cur++;
             }
-            allrdy = !G.member || ((c >> (adv ? 42 : 21)) & M) == P;
+            allrdy = !G.member || (adv ? cbv : (ca >> 16)) == P;
         } else {
             allfin = gall(G, G.ldone);
             if (G.member && G.running && allfin) {
