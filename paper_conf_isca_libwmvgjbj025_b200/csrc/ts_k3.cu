@@ -501,11 +501,24 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                         // interleaves), the ones past n masked out of the sum
                         const bool split = 2 * p <= W;
                         const bool twin = split && li >= W / 2 && li - W / 2 < p;
+                        // mix64 of the eight instant times: the same in every lane of the segment, so with W >= 8
+                        // segment lane j computes instant j's and the others read it by shuffle (the block's
+                        // control flow is segment-uniform: every lane of the segment is here)
+                        uint64_t tmx[8];
+                        if constexpr (W >= 8) {
+                            const int j = li & 7;
+                            double tj = ti[0];
+#pragma unroll
+                            for (int i = 1; i < 8; i++) tj = j == i ? ti[i] : tj;
+                            const uint64_t mj = mix64((uint64_t)__double_as_longlong(tj));
+#pragma unroll
+                            for (int i = 0; i < 8; i++) tmx[i] = __shfl_sync(smask, mj, sbase + i);
+                        }
                         if (used || twin) {
                             const uint64_t cb = ((uint64_t)cur << 32) | (uint64_t)(twin ? li - W / 2 : li);
-                            // instant of parity `odd` (0 activation, 1 delivery + release) of step k
-                            auto term = [&](double tv, bool odd, int kk) -> uint64_t {
-                                const uint64_t m = mix64((uint64_t)__double_as_longlong(tv));
+                            // instant of parity `odd` (0 activation, 1 delivery + release) of step k, m = mix64 of
+                            // its time
+                            auto term = [&](uint64_t m, bool odd, int kk) -> uint64_t {
                                 const uint64_t k = (uint64_t)kk;
                                 if (!odd)
                                     return mix64(m ^ (((uint64_t)EV_ACTIVATE << 60) | cb | (k << 16)));
@@ -517,13 +530,19 @@ __global__ void __launch_bounds__(K3_THREADS, TS_K3_MINB) k3_timeline(const K3Ar
                                 const int off = twin ? 4 : 0;
 #pragma unroll
                                 for (int i = 0; i < 4; i++) {
-                                    const uint64_t tr = term(twin ? ti[i + 4] : ti[i], (i & 1) != 0, D0 + ((i + off) >> 1));
+                                    uint64_t m;
+                                    if constexpr (W >= 8) m = twin ? tmx[i + 4] : tmx[i];
+                                    else m = mix64((uint64_t)__double_as_longlong(twin ? ti[i + 4] : ti[i]));
+                                    const uint64_t tr = term(m, (i & 1) != 0, D0 + ((i + off) >> 1));
                                     add += i + off < n ? tr : 0ull;
                                 }
                             } else {
 #pragma unroll
                                 for (int i = 0; i < 8; i++) {
-                                    const uint64_t tr = term(ti[i], (i & 1) != 0, D0 + (i >> 1));
+                                    uint64_t m;
+                                    if constexpr (W >= 8) m = tmx[i];
+                                    else m = mix64((uint64_t)__double_as_longlong(ti[i]));
+                                    const uint64_t tr = term(m, (i & 1) != 0, D0 + (i >> 1));
                                     add += i < n ? tr : 0ull;
                                 }
                             }
